@@ -23,7 +23,7 @@ oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
 	$(CC) -O2 -std=c11 -Wall -Wextra -fPIC -shared -o $@ oracle/oracle.c
 
 hec: $(PKG)/libhec.so
-$(PKG)/libhec.so: $(CU_SRC) $(CU_HDR)
+$(PKG)/libhec.so: $(CU_SRC) $(CU_HDR) Makefile
 	$(NVCC) $(NVFLAGS) -Xptxas -v -shared -o $@ $(CU_SRC) -lcudart 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
 
 clean:

@@ -1,0 +1,324 @@
+#!/usr/bin/env python
+"""Benchmark of the HEC coarsening hot path on B200.
+
+One step = one full HEC hierarchy (Alg 1: mapping + coarse
+construction at every level until n_l <= C, discard rule L367) of the
+workload's G0, which is resident in HBM when the timed region starts.
+
+  metric  fine edges coarsened/sec (undirected G0 edges m0 / time-to-cutoff)
+  value   whole-job aggregate over ranks (each rank coarsens its own replica)
+  e2e     same metric through the C-ABI call with host buffers: pinned-host ->
+          device copy of G0 and a device -> host read of the coarsest graph and
+          the level sizes inside the timed region
+  roofline  dominant phase: algorithmic bytes / CUDA-event device time, vs the
+          measured HBM copy bandwidth in MEASURED_PEAKS.json
+  cpu_baseline  the CPU oracle (single thread) on a bounded sample
+
+usage: python bench.py [--gpus N] [--steps K] [--warmup W] [--config 4] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "fine edges coarsened/sec and time-to-cutoff per hierarchy; HBM GB/s vs peak"
+UNIT = "edges/s"
+SAMPLE = dict(kind="rmat", scale=19, ef=32, cutoff=50)  # oracle sample: G-spec R-MAT, 1/32 of C4's vertex range
+
+
+def env_rank():
+    return (int(os.environ.get("RANK", 0)), int(os.environ.get("LOCAL_RANK", 0)),
+            int(os.environ.get("WORLD_SIZE", 1)))
+
+
+def make_graph(cfg):
+    import graphgen as gg
+    if isinstance(cfg, dict):
+        return gg.rmat(cfg["scale"], cfg["ef"], gg.GEN_SEED)
+    return gg.config(cfg)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.FIELDS}",
+                                       "--format=csv,noheader,nounits", "-lms", "50"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+        time.sleep(0.15)
+        return self
+
+    def __exit__(self, *a):
+        self.out = ""
+        if self.p:
+            self.p.terminate()
+            try:
+                self.out = self.p.communicate(timeout=5)[0]
+            except subprocess.TimeoutExpired:
+                self.p.kill()
+
+    def summary(self):
+        rows = []
+        for line in (self.out or "").splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                rows.append(dict(sm=float(f[1]), smax=float(f[2]), power=float(f[3]),
+                                 hw=f[5] == "Active", hwt=f[6] == "Active", swt=f[7] == "Active",
+                                 cap=f[8] == "Active"))
+            except ValueError:
+                continue
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        load = [r for r in rows if r["power"] > 200] or rows
+        reasons = sorted({name for r in rows for name, k in
+                          (("hw_slowdown", "hw"), ("hw_thermal_slowdown", "hwt"),
+                           ("sw_thermal_slowdown", "swt"), ("sw_power_cap", "cap")) if r[k]})
+        return {"sm_mhz": statistics.median(r["sm"] for r in load), "sm_max_mhz": rows[0]["smax"],
+                "reasons": reasons, "samples": len(rows)}
+
+
+def level_bytes(levels, g0_n, g0_nnz):
+    """B_l = 16 nnz + 8 nnz_c + 28 n + 12 n_c per built level."""
+    tot = 0.0
+    n, nnz = g0_n, g0_nnz
+    for (nc, nnzc) in levels:
+        tot += 16 * nnz + 8 * nnzc + 28 * n + 12 * nc
+        n, nnz = nc, nnzc
+    return tot
+
+
+def traffic_from_profiles(kernel_phase):
+    """ncu dram bytes per launch of the dominant kernel, if a capture was committed."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    d = json.load(open(p))
+    return d.get(kernel_phase)
+
+
+def run_oracle_sample(reps):
+    import oracle as o
+    g = make_graph(SAMPLE)
+    ts = []
+    for _ in range(reps):
+        H = o.hierarchy(g, SAMPLE["cutoff"], 0x5EED)
+        ts.append(H.t_total)
+    return g, ts
+
+
+def reference_arm(args, rank, world):
+    """The base contract's reference arm: the CPU oracle as it stands, on a bounded
+    sample of the workload (this tier has no runnable reference implementation)."""
+    if rank != 0:
+        return 0
+    import oracle as o
+    g = make_graph(SAMPLE)
+    m0 = g.nnz // 2
+    for _ in range(args.warmup):
+        o.hierarchy(g, SAMPLE["cutoff"], 0x5EED)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        H = o.hierarchy(g, SAMPLE["cutoff"], 0x5EED)
+    dt = (time.perf_counter() - t0) / args.steps
+    val = m0 / dt
+    sample = f"oracle hierarchy (C=50) of rmat_s{SAMPLE['scale']}_ef{SAMPLE['ef']} (G-spec, n={g.n}, nnz={g.nnz})"
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": workload_name(args.config), "sample": sample,
+                       "levels": [lv.n_c for lv in H.levels]},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def workload_name(cfg):
+    import graphgen as gg
+    c = gg.CONFIGS[cfg]
+    return f"C{cfg} {c['name']} HEC hierarchy to C={c['cutoff']} (seed 0x5EED)"
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=4)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    rank, local_rank, world = env_rank()
+    if args.impl == "reference":
+        return reference_arm(args, rank, world)
+
+    import numpy as np
+    import torch
+    import graphgen as gg
+    import paper_conf_ipps_gilbertabmr21_b200 as P
+
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    else:
+        dist = None
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    cfg = gg.CONFIGS[args.config]
+    t0 = time.time()
+    g = make_graph(args.config)
+    t_gen = time.time() - t0
+    m0 = g.nnz // 2
+    dg = P.DeviceGraph.from_host(g, device=dev)
+    stream = torch.cuda.current_stream()
+    ctx = P.Context(stream=stream)
+
+    def barrier():
+        if dist:
+            dist.barrier()
+
+    def step():
+        h = P.coarsen_hierarchy(ctx, dg, cfg["cutoff"], gg.COARSEN_SEED)
+        sizes = [(lv.graph.n, lv.graph.nnz) for lv in h.levels]
+        h.free()
+        return sizes
+
+    for _ in range(args.warmup):
+        levels = step()
+    torch.cuda.synchronize()
+    # ---- timed region
+    ctx.set_profiling(True)
+    ctx.profile_reset()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(torch.cuda.current_device()) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            levels = step()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    barrier()
+    ms = ev0.elapsed_time(ev1) / args.steps
+    prof = ctx.profile()
+    launches = ctx.launches()
+    ctx.set_profiling(False)
+    if dist:
+        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = m0 * world / (ms / 1e3)
+
+    # ---- roofline of the dominant phase
+    peak, peak_src = peaks()
+    dom = max(prof.items(), key=lambda kv: kv[1]["ms"])
+    dom_name, d = dom
+    achieved = d["bytes"] / (d["ms"] / 1e3) / 1e9 if d["ms"] > 0 else 0.0
+    traffic = traffic_from_profiles(dom_name)
+    B = level_bytes(levels, g.n, g.nnz)
+    phases = {k: {"ms_per_step": v["ms"] / args.steps, "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] else 0,
+                  "share": v["ms"] / (ms * args.steps)} for k, v in sorted(prof.items(), key=lambda kv: -kv[1]["ms"])}
+
+    # ---- e2e through host buffers
+    e2e = None
+    if args.e2e_steps > 0:
+        host = [torch.from_numpy(a).pin_memory() for a in (g.row_ptr, g.col, g.wgt, g.vwgt)]
+        bi = sum(t.numel() * t.element_size() for t in host)
+        bo = 0
+        torch.cuda.synchronize()
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            d_in = [t.to(dev, non_blocking=True) for t in host]
+            hg = P.DeviceGraph(*d_in)
+            h = P.coarsen_hierarchy(ctx, hg, cfg["cutoff"], gg.COARSEN_SEED)
+            last = h.levels[-1].graph if h.levels else hg
+            outs = [last.row_ptr.to("cpu", non_blocking=True), last.col.to("cpu", non_blocking=True),
+                    last.wgt.to("cpu", non_blocking=True)]
+            sizes = torch.tensor([lv.graph.n for lv in h.levels], dtype=torch.int64)
+            bo = sum(t.numel() * t.element_size() for t in outs) + sizes.numel() * 8
+            h.free()
+            del d_in, hg
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ems = e0.elapsed_time(e1) / args.e2e_steps
+        if dist:
+            t = torch.tensor([ems], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": m0 * world / (ems / 1e3), "unit": UNIT, "h2d_bytes_per_step": bi, "d2h_bytes_per_step": bo,
+               "ms_per_step": ems}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        sg, ts = run_oracle_sample(2)
+        tmed = statistics.median(ts)
+        cpu = {"value": (sg.nnz // 2) / tmed, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"oracle hierarchy (C=50, seed 0x5EED) of rmat_s{SAMPLE['scale']}_ef{SAMPLE['ef']} "
+                         f"(G-spec, n={sg.n}, nnz={sg.nnz}), median of 2 runs, {tmed:.2f} s each; "
+                         f"host nproc={os.cpu_count()}"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz, "m0": m0,
+                       "cutoff": cfg["cutoff"], "seed": gg.COARSEN_SEED,
+                       "parallelism": "replicas" if world > 1 else "single",
+                       "l2": f"inputs {(g.nnz * 8 + g.n * 12) / 1e9:.1f} GB > 126 MB L2 (no flush needed)",
+                       "levels": [n for n, _ in levels], "gen_s": round(t_gen, 1)},
+            "time_to_cutoff_ms": ms,
+            "hierarchy_GBps": B / (ms / 1e3) / 1e9,
+            "hierarchy_frac_of_peak": B / (ms / 1e3) / 1e9 / peak,
+            "roofline": {"bound": "hbm", "kernel": dom_name, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src},
+            "phases": phases,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "gpu_launches_per_step": launches / args.steps,
+            "clocks": clk.summary(),
+        }
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if dist:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,215 @@
+/* hec.h — C-ABI of libhec: the B200 (sm_100a) hot path of iterated Heavy Edge
+ * Coarsening (HEC), Gilbert, Acer, Boman, Madduri, Rajamanickam, IPDPS 2021.
+ *
+ * PAPER.md references are to /root/reference/PAPER.md (line numbers "L…").
+ * The three north-star entry points follow the paper's Algorithm 1 (L37-53):
+ *   hec_find_mapping   FINDCOARSEMAPPING with HEC (Alg 3 L99-130; parallel Alg 4
+ *                      L168-225): M[1..n], n_c  (L103)
+ *   build_coarse_graph CONSTRUCTCOARSEGRAPH (Alg 6): G(V_c, E_c, W_c) in CSR
+ *   coarsen_hierarchy  Alg 1 with cutoff C and the discard rule of L367
+ *
+ * Conventions:
+ *   - 0-based ids (the paper is 1-based, L280).  Vertex ids, labels, columns and
+ *     edge/vertex weights are int32; row offsets are int64 (R7).
+ *   - Pointers inside hec_graph and all array arguments documented "device" are
+ *     CUDA device pointers; "host" arguments are host pointers.
+ *   - All work is stream-ordered on the context's stream.  Calls that must know a
+ *     size on the host (n_c, nnz_c) synchronise that stream once to read it.
+ *   - Inputs are never written.  Outputs allocated by the library are owned by the
+ *     returned handle and released with the matching *_free call.
+ *   - Every function returns HEC_OK (0) or a negative HEC_E* code; on error no
+ *     output handle is returned and hec_last_error() (thread-local) describes it.
+ *   - Results are deterministic and bit-exact with the plain sequential
+ *     definition (Alg 3 under the visit order of hec_prio, coarse ids by ascending
+ *     root id, coarse rows with ascending columns and summed integer weights).
+ */
+#ifndef HEC_H
+#define HEC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(_WIN32)
+#define HEC_API __declspec(dllexport)
+#else
+#define HEC_API __attribute__((visibility("default")))
+#endif
+
+/* ------------------------------------------------------------------ errors */
+enum {
+  HEC_OK = 0,
+  HEC_EINVAL = -1,    /* bad argument or (validate=1) malformed graph */
+  HEC_ENOMEM = -2,    /* device allocation failed */
+  HEC_ECUDA = -3,     /* CUDA runtime / kernel error */
+  HEC_EOVERFLOW = -4  /* a coarse weight or vertex weight exceeds INT32_MAX */
+};
+/* Why coarsen_hierarchy stopped (Alg 1 loop test L46 + L367). */
+enum {
+  HEC_STOP_CUTOFF = 0,     /* n_l <= C */
+  HEC_STOP_DISCARD = 1,    /* next level would drop below discard_below: not built */
+  HEC_STOP_STALL = 2,      /* n_c == n (only possible with all vertices isolated) */
+  HEC_STOP_MAX_LEVELS = 3  /* level cap reached */
+};
+
+/* Thread-local, static storage; valid until the next failing call on the thread. */
+HEC_API const char *hec_last_error(void);
+
+/* ------------------------------------------------------------------- graph */
+/* Borrowed CSR view of an undirected graph G(V,E,W):
+ * each undirected edge stored in both endpoint rows, no self-loops, no parallel
+ * edges, weights > 0 and symmetric, columns strictly ascending within a row. */
+typedef struct {
+  int64_t n;               /* |V| (0 <= n < 2^31)                                  */
+  int64_t nnz;             /* directed entries = 2m                                 */
+  const int64_t *row_ptr;  /* device [n+1], row_ptr[0]=0, non-decreasing, [n]=nnz  */
+  const int32_t *col;      /* device [nnz]                                          */
+  const int32_t *wgt;      /* device [nnz], > 0, W(u,v) == W(v,u)                   */
+  const int32_t *vwgt;     /* device [n] vertex weights > 0, or NULL = all ones     */
+} hec_graph;
+
+/* --------------------------------------------------------------- context */
+typedef struct CUstream_st *hec_stream_t; /* == cudaStream_t */
+/* Optional device allocator (e.g. a framework caching allocator).  Must return
+ * 256-byte aligned device memory usable on `stream`, or NULL on failure. */
+typedef void *(*hec_alloc_fn)(size_t bytes, hec_stream_t stream, void *user);
+typedef void (*hec_free_fn)(void *ptr, hec_stream_t stream, void *user);
+
+typedef struct hec_ctx hec_ctx;
+
+/* Create a context bound to the current CUDA device and `stream` (NULL = the
+ * legacy default stream).  alloc/free NULL => cudaMallocAsync/cudaFreeAsync on
+ * the device's default pool.  The context owns a grow-only device workspace
+ * reused across calls (no per-call allocation once warm). */
+HEC_API int hec_ctx_create(hec_stream_t stream, hec_alloc_fn alloc, hec_free_fn free,
+                           void *user, hec_ctx **out);
+HEC_API void hec_ctx_destroy(hec_ctx *ctx);
+/* validate=1: every call first checks R1 on the device (O(nnz)): offsets
+ * monotone, columns in range/strictly ascending/no self-loop, weights > 0,
+ * symmetric structure and weights; a violation returns HEC_EINVAL. */
+HEC_API int hec_ctx_set_validate(hec_ctx *ctx, int validate);
+HEC_API int hec_ctx_set_stream(hec_ctx *ctx, hec_stream_t stream);
+
+/* Per-call statistics of the most recent hec_find_mapping/coarsen_hierarchy
+ * level processed by this context. */
+typedef struct {
+  int32_t rounds;          /* resolution rounds of the last mapping */
+  int32_t fallback;        /* 1 if the round cap was hit and the residual was finished sequentially */
+  int64_t n_c;             /* coarse vertices of the last mapping */
+  int64_t nnz_c;           /* coarse entries of the last construction */
+  int64_t huge_rows;       /* rows routed to the skewed-degree path in the last construction */
+  int64_t dense_rows;      /* of which used the dense accumulator */
+} hec_stats;
+HEC_API int hec_ctx_last_stats(const hec_ctx *ctx, hec_stats *out);
+
+/* ------------------------------------------------- north-star call 1: mapping */
+/* Visit-order priority of vertex u at level l (the paper's
+ * GENPERM "random order", L61, L104):
+ *   s_l = splitmix64(seed + l);  prio_l(u) = (splitmix64(s_l ^ u) >> 32) << 32 | u
+ * Host helper so callers can reproduce the order. */
+HEC_API uint64_t hec_prio(uint64_t seed, int level, int64_t u);
+
+/* HEC fine-to-coarse mapping of g (Alg 3 semantics, computed by the parallel
+ * heavy-neighbour scan + deterministic resolution rounds):
+ *   H[u]  = heaviest neighbour, ties -> smallest id, isolated -> u   (L116, L184)
+ *   visit order ascending hec_prio(seed, level, u)
+ *   M     = device int32[n] caller-allocated; coarse ids 0..n_c-1 ordered by the
+ *           aggregate's root (the vertex an aggregate was created at) ascending
+ *   *n_c  = host int64, number of aggregates.
+ * Synchronises the stream once (to read n_c).  n == 0 gives n_c = 0. */
+HEC_API int hec_find_mapping(hec_ctx *ctx, const hec_graph *g, uint64_t seed, int level,
+                             int32_t *M, int64_t *n_c);
+
+/* Same with explicit device priorities prio[n] (uint64, pairwise distinct: the
+ * visit order is ascending prio).  Test hook for hand-drawn visit orders. */
+HEC_API int hec_find_mapping_prio(hec_ctx *ctx, const hec_graph *g, const uint64_t *prio,
+                                  int32_t *M, int64_t *n_c);
+
+/* --------------------------------------------- north-star call 2: construction */
+typedef struct hec_csr_owned hec_csr_owned; /* device CSR owned by the library */
+
+/* Coarse graph G_c = P A P^T without the diagonal (L141, L280):
+ *   W_c(a,b) = sum_{M[u]=a} sum_{v in N(u), M[v]=b} W(u,v) for a != b,
+ *   rows ascending by b, vwgt_c(a) = sum_{M[u]=a} vwgt(u).
+ * M: device int32[n] with values in [0, n_c), every label used.
+ * Returns HEC_EOVERFLOW if a sum exceeds INT32_MAX.  Synchronises once (nnz_c). */
+HEC_API int build_coarse_graph(hec_ctx *ctx, const hec_graph *g, const int32_t *M,
+                               int64_t n_c, hec_csr_owned **out);
+/* Borrow the owned CSR as a hec_graph (valid until hec_csr_free). */
+HEC_API int hec_csr_view(const hec_csr_owned *csr, hec_graph *view);
+HEC_API void hec_csr_free(hec_csr_owned *csr);
+
+/* ---------------------------------------------- north-star call 3: hierarchy */
+typedef struct hec_hierarchy hec_hierarchy;
+
+/* Alg 1: l = 0; while n_l > cutoff and l < max_levels:
+ *   (M, n') = hec_find_mapping(G_l, seed, level = l);
+ *   if n' < discard_below: stop (DISCARD; G_{l+1} not built)   (L367, reading Z11/Z12)
+ *   if n' == n_l: stop (STALL)
+ *   G_{l+1} = build_coarse_graph(G_l, M, n'); l++
+ * Output levels i = 1..l hold G_i and M_i (M_i maps G_{i-1} -> G_i).
+ * discard_below <= 0 selects the paper's 10; max_levels <= 0 selects 200. */
+HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
+                              int64_t discard_below, int max_levels, hec_hierarchy **out);
+HEC_API int hec_hierarchy_levels(const hec_hierarchy *h);
+/* i in [1, levels]: view of G_i, device pointer to M_i (length n_{i-1}), n_{i-1}. */
+HEC_API int hec_hierarchy_level(const hec_hierarchy *h, int i, hec_graph *g_i,
+                                const int32_t **M_i, int64_t *n_fine);
+HEC_API int hec_hierarchy_stop_reason(const hec_hierarchy *h);
+/* n' of the discarded mapping when stop_reason == HEC_STOP_DISCARD, else -1. */
+HEC_API int64_t hec_hierarchy_discarded_n_c(const hec_hierarchy *h);
+/* Resolution rounds used at level i (1-based), or -1. */
+HEC_API int hec_hierarchy_rounds(const hec_hierarchy *h, int i);
+HEC_API void hec_hierarchy_free(hec_hierarchy *h);
+
+/* ------------------------------------------------------------ profiling */
+/* When enabled, every phase of the hot path is bracketed by CUDA events on the
+ * context stream; hec_ctx_profile() synchronises, then reports per phase the
+ * summed device time, number of calls and the algorithmic bytes (compulsory
+ * traffic: each input read once, each output written once).
+ * Phases: "heavy" (a1), "rounds" (a3), "relabel" (a4+a5), "bucket" (a7),
+ * "rows_small", "rows_mid" (a8), "rows_skew" (a9), "place" (a10). */
+typedef struct {
+  char name[24];
+  double ms;         /* summed device time */
+  int64_t calls;
+  double bytes;      /* summed algorithmic bytes */
+} hec_phase_time;
+HEC_API int hec_ctx_set_profiling(hec_ctx *ctx, int on);
+/* Clears the accumulated phase times and the launch counter. */
+HEC_API int hec_ctx_profile_reset(hec_ctx *ctx);
+/* Writes up to max entries; *count receives the number of phases. */
+HEC_API int hec_ctx_profile(hec_ctx *ctx, hec_phase_time *out, int max, int *count);
+/* Number of libhec kernel launches since the last reset. */
+HEC_API int64_t hec_ctx_launches(const hec_ctx *ctx);
+
+/* ------------------------------------------------------- debug / test hooks */
+/* Heavy-neighbour array only (a1): H device int32[n]. */
+HEC_API int hec_debug_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H);
+/* Root flags after the resolution rounds (a3): root device uint8[n] (1 = root);
+ * *rounds (host) receives the number of rounds.  prio NULL => hec_prio(seed, level). */
+HEC_API int hec_debug_roots(hec_ctx *ctx, const hec_graph *g, const uint64_t *prio,
+                            uint64_t seed, int level, uint8_t *root, int *rounds);
+
+/* ------------------------------------------- multi-GPU construction (§8(e)) */
+/* Rows [a_begin, a_end) of G_c only (coarse-vertex range partition).  Writes
+ * counts[a - a_begin] = |row a| (device int64[a_end-a_begin]); then, after the
+ * caller has all-gathered the counts and passed the global exclusive offsets of
+ * its rows (device int64 offs[a_end-a_begin+1], offs[0] = first entry index of
+ * row a_begin), hec_build_rows_write fills col_c/wgt_c at those global
+ * positions (device arrays of the full nnz_c, or of the slice when offs are
+ * rebased by the caller) plus vwgt_c[a - a_begin].
+ * The pair must be called with the same ctx, g, M, n_c, range and no other
+ * libhec call in between on that ctx. */
+HEC_API int hec_build_rows_count(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
+                                 int64_t a_begin, int64_t a_end, int64_t *counts);
+HEC_API int hec_build_rows_write(hec_ctx *ctx, const int64_t *offs, int32_t *col_c,
+                                 int32_t *wgt_c, int32_t *vwgt_c);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HEC_H */

@@ -1,0 +1,501 @@
+// mapping.cu — FINDCOARSEMAPPING for HEC on sm_100a.
+//
+//  a1 heavy neighbour  H[u] = argmax_{v in N(u)} W(u,v), ties -> smallest v,
+//     isolated -> u.  PAPER.md Alg 4 l.2-8 (L177-187) / Alg 3 l.6-10 (L109-119).
+//     Merge-path tiles over (row ends + entries): every tile covers a fixed
+//     number of items regardless of the degree skew, the tile's col/wgt are
+//     staged into shared memory with one cp.async.bulk (TMA) copy each, and the
+//     per-row argmax runs on the packed key (w << 32) | ~v.
+//  a3 resolution rounds replacing Alg 4's CAS passes (L189-224): a vertex is
+//     ROOT iff a lower child (H[y]=u, prio(y)<prio(u)) is ACTIVE, ACTIVE iff no
+//     lower child is still undecided.  Deterministic: only idempotent flag
+//     stores; result == sequential Alg 3 (derived).  One
+//     persistent cooperative kernel runs all rounds with a compacted worklist.
+//  a4 relabel  coarse id = exclusive scan of root flags (FINDUNIQANDRELABEL,
+//     L273) with the decoupled-look-back scan.
+//  a5 inherit  M[u] = M[first root on the H-path from u] (Alg 3 l.14 L128,
+//     pointer chase as in Alg 5 l.17-21 L264-271).
+#include "hec_internal.cuh"
+
+namespace hec {
+
+// ---------------------------------------------------------------- a1 heavy
+constexpr int kHvBlock = 256;
+constexpr int kHvItems = 16;
+constexpr int kHvTile = kHvBlock * kHvItems;  // merge items (row ends + entries) per tile
+
+// Merge-path split of diagonal d between the row-end list row_ptr[1..n] and the
+// entry indices 0..nnz-1: returns x = row ends consumed (entries = d - x).
+__device__ __forceinline__ int64_t merge_path_x(int64_t d, const int64_t *__restrict__ row_ptr,
+                                                int64_t n, int64_t nnz) {
+  int64_t lo = d - nnz > 0 ? d - nnz : 0;
+  int64_t hi = d < n ? d : n;
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (__ldg(row_ptr + mid + 1) <= d - mid - 1) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+__global__ void k_tile_coords(int64_t n, int64_t nnz, const int64_t *__restrict__ row_ptr,
+                              int64_t ntiles, int64_t *__restrict__ cx) {
+  int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (t > ntiles) return;
+  int64_t d = t * kHvTile;
+  if (d > n + nnz) d = n + nnz;
+  cx[t] = merge_path_x(d, row_ptr, n, nnz);
+}
+
+__device__ __forceinline__ uint64_t pack_key(int32_t w, int32_t v) {
+  return ((uint64_t)(uint32_t)w << 32) | (uint64_t)(~(uint32_t)v);
+}
+__device__ __forceinline__ int32_t key_vertex(uint64_t k) { return (int32_t)(~(uint32_t)k); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, unsigned count) {
+  unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, unsigned bytes) {
+  unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void tma_bulk_g2s(void *dst, const void *src, unsigned bytes,
+                                             uint64_t *bar) {
+  unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  unsigned b = (unsigned)__cvta_generic_to_shared(bar);
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d),
+      "l"(src), "r"(bytes), "r"(b)
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
+  unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+  unsigned done = 0;
+  while (!done) {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(a), "r"(phase)
+        : "memory");
+  }
+}
+
+struct HeavySmem {
+  alignas(16) int32_t col[kHvTile + 8];
+  alignas(16) int32_t wgt[kHvTile + 8];
+  int32_t rb[kHvTile + 2];        // row begin offsets relative to the tile's first entry
+  uint64_t key[kHvTile + 2];      // per-row partial argmax keys (rows split across threads)
+  uint64_t bar;
+};
+
+// One tile = kHvTile merge items.  head_key[t]: partial of the tile's first row
+// when that row started in an earlier tile and ends here; mid_key[t]: partial of
+// the unfinished row at the tile's end (row x1 < n).
+__global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
+                                                   const int64_t *__restrict__ row_ptr,
+                                                   const int32_t *__restrict__ col,
+                                                   const int32_t *__restrict__ wgt,
+                                                   const int64_t *__restrict__ cx,
+                                                   int32_t *__restrict__ H,
+                                                   uint64_t *__restrict__ head_key,
+                                                   uint64_t *__restrict__ mid_key) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  HeavySmem &S = *reinterpret_cast<HeavySmem *>(smem_raw);
+  const int64_t t = blockIdx.x;
+  const int64_t total = n + nnz;
+  const int64_t d0 = t * kHvTile;
+  const int64_t d1 = (d0 + kHvTile < total) ? d0 + kHvTile : total;
+  const int64_t x0 = cx[t], x1 = cx[t + 1];
+  const int64_t y0 = d0 - x0, y1 = d1 - x1;
+  const int64_t ybase = y0 & ~(int64_t)3;
+  const int64_t ya = (y0 + 3) & ~(int64_t)3, yb = y1 & ~(int64_t)3;
+  const bool bulk = yb > ya;
+
+  if (threadIdx.x == 0) {
+    mbar_init(&S.bar, 1);
+    if (bulk) {
+      unsigned bytes = (unsigned)((yb - ya) * 4);
+      mbar_expect_tx(&S.bar, 2 * bytes);
+      tma_bulk_g2s(S.col + (ya - ybase), col + ya, bytes, &S.bar);
+      tma_bulk_g2s(S.wgt + (ya - ybase), wgt + ya, bytes, &S.bar);
+    }
+  }
+  // head / tail entries outside the 16-byte aligned interior
+  {
+    int64_t hend = bulk ? ya : y1;
+    for (int64_t y = y0 + threadIdx.x; y < hend; y += kHvBlock) {
+      S.col[y - ybase] = __ldg(col + y);
+      S.wgt[y - ybase] = __ldg(wgt + y);
+    }
+    if (bulk) {
+      for (int64_t y = yb + threadIdx.x; y < y1; y += kHvBlock) {
+        S.col[y - ybase] = __ldg(col + y);
+        S.wgt[y - ybase] = __ldg(wgt + y);
+      }
+    }
+  }
+  // row begins rows x0..x1+1 (clamped), and zeroed partial keys
+  const int nrows = (int)(x1 - x0);  // rows whose end item lies in this tile
+  for (int k = threadIdx.x; k <= nrows + 1; k += kHvBlock) {
+    int64_t r = x0 + k;
+    int64_t b = r <= n ? __ldg(row_ptr + r) : nnz;
+    int64_t rel = b - y0;
+    S.rb[k] = rel < -1 ? -1 : (rel > kHvTile + 1 ? kHvTile + 1 : (int32_t)rel);
+    S.key[k] = 0;
+  }
+  __syncthreads();
+  if (bulk) mbar_wait(&S.bar, 0);
+
+  // ---- per-thread merge-path walk over kHvItems items
+  const int64_t tile_items = d1 - d0;
+  const int64_t ld = (int64_t)threadIdx.x * kHvItems;
+  if (ld < tile_items) {
+    const int64_t ents = y1 - y0;
+    // local search: a[k] = row end of row x0+k = rb[k+1]; b[j] = j
+    int64_t lo = ld - ents > 0 ? ld - ents : 0;
+    int64_t hi = ld < nrows ? ld : nrows;
+    while (lo < hi) {
+      int64_t mid = (lo + hi) >> 1;
+      if (S.rb[mid + 1] <= ld - mid - 1) lo = mid + 1;
+      else hi = mid;
+    }
+    int k = (int)lo;            // local row
+    int y = (int)(ld - lo);     // local entry
+    const int ystart = y;
+    int items = (int)((tile_items - ld) < kHvItems ? (tile_items - ld) : kHvItems);
+    uint64_t key = 0;
+    for (int i = 0; i < items; ++i) {
+      if (k < nrows && y >= S.rb[k + 1]) {
+        // end item of row x0+k
+        if (S.rb[k] >= ystart) {
+          H[x0 + k] = key ? key_vertex(key) : (int32_t)(x0 + k);
+        } else if (key) {
+          atomicMax((unsigned long long *)&S.key[k], (unsigned long long)key);
+        }
+        ++k;
+        key = 0;
+      } else {
+        int idx = (int)(y0 - ybase) + y;
+        uint64_t kk = pack_key(S.wgt[idx], S.col[idx]);
+        key = kk > key ? kk : key;
+        ++y;
+      }
+    }
+    if (key) atomicMax((unsigned long long *)&S.key[k], (unsigned long long)key);
+  }
+  __syncthreads();
+  // ---- rows split across threads / tiles
+  for (int k = threadIdx.x; k <= nrows; k += kHvBlock) {
+    uint64_t key = S.key[k];
+    if (k < nrows) {
+      if (k == 0 && S.rb[0] < 0) {
+        head_key[t] = key;                 // tail piece of a row begun in an earlier tile
+      } else if (key) {
+        H[x0 + k] = key_vertex(key);
+      }
+    } else if (x1 < n) {
+      mid_key[t] = key;                    // unfinished row at the tile end
+    }
+  }
+}
+
+// Rows spanning tile boundaries: the tile holding the row's end item combines
+// its head piece with the mid pieces of the preceding tiles of the same row.
+__global__ void k_heavy_fixup(int64_t n, int64_t nnz, const int64_t *__restrict__ row_ptr,
+                              int64_t ntiles, const int64_t *__restrict__ cx,
+                              const uint64_t *__restrict__ head_key,
+                              const uint64_t *__restrict__ mid_key, int32_t *__restrict__ H) {
+  int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (t >= ntiles) return;
+  int64_t x0 = cx[t], x1 = cx[t + 1];
+  int64_t y0 = t * kHvTile - x0;
+  if (!(x0 < x1 && x0 < n && __ldg(row_ptr + x0) < y0)) return;
+  int64_t x = x0;
+  uint64_t key = head_key[t];
+  const int64_t rb = __ldg(row_ptr + x);
+  for (int64_t s = t - 1; s >= 0; --s) {
+    if (cx[s + 1] != x) break;
+    uint64_t m = mid_key[s];
+    key = m > key ? m : key;
+    int64_t ys = s * kHvTile - cx[s];
+    if (rb >= ys) break;  // row begins in tile s
+  }
+  H[x] = key ? key_vertex(key) : (int32_t)x;
+}
+
+__global__ void k_fill_identity(int64_t n, int32_t *__restrict__ H) {
+  int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u < n) H[u] = (int32_t)u;
+}
+
+static inline unsigned nblk(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
+
+static size_t heavy_ws(int64_t n, int64_t nnz) {
+  int64_t ntiles = (n + nnz + kHvTile - 1) / kHvTile;
+  return ws_bytes(ntiles + 1, 8) + 2 * ws_bytes(ntiles + 1, 8);
+}
+
+static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H) {
+  const int64_t n = g->n, nnz = g->nnz;
+  if (n == 0) return HEC_OK;
+  if (nnz == 0) {
+    k_fill_identity<<<nblk(n, 256), 256, 0, ctx->stream>>>(n, H);
+    HEC_LAUNCH_CHECK();
+    return HEC_OK;
+  }
+  int64_t ntiles = (n + nnz + kHvTile - 1) / kHvTile;
+  int64_t *cx = ws_take<int64_t>(ctx, ntiles + 1);
+  uint64_t *head = ws_take<uint64_t>(ctx, ntiles + 1);
+  uint64_t *mid = ws_take<uint64_t>(ctx, ntiles + 1);
+  if (!cx || !head || !mid) { set_error("workspace under-reserved (heavy)"); return HEC_EINVAL; }
+  k_tile_coords<<<nblk(ntiles + 1, 256), 256, 0, ctx->stream>>>(n, nnz, g->row_ptr, ntiles, cx);
+  HEC_LAUNCH_CHECK();
+  static bool attr = false;
+  if (!attr) {
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_heavy, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)sizeof(HeavySmem)));
+    attr = true;
+  }
+  k_heavy<<<(unsigned)ntiles, kHvBlock, sizeof(HeavySmem), ctx->stream>>>(
+      n, nnz, g->row_ptr, g->col, g->wgt, cx, H, head, mid);
+  HEC_LAUNCH_CHECK();
+  k_heavy_fixup<<<nblk(ntiles, 256), 256, 0, ctx->stream>>>(n, nnz, g->row_ptr, ntiles, cx, head,
+                                                            mid, H);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
+// --------------------------------------------------------- a3 resolution rounds
+enum : uint8_t { UNDEC = 0, ACTIVE = 2, ROOT = 3 };
+
+// status, lower-child "blocked" stamps for round 1.
+__global__ void k_round_init(int64_t n, const int32_t *__restrict__ H, Prio prio,
+                             uint8_t *__restrict__ status, int32_t *__restrict__ blocked) {
+  int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u >= n) return;
+  int32_t x = H[u];
+  status[u] = (x == (int32_t)u) ? ROOT : UNDEC;
+  if (x != (int32_t)u && prio((uint32_t)u) < prio((uint32_t)x)) blocked[x] = 1;
+}
+
+struct RoundArgs {
+  int64_t n;
+  const int32_t *H;
+  Prio prio;
+  uint8_t *status;
+  uint8_t *rootflag;
+  int32_t *blocked;
+  int32_t *wl[2];
+  unsigned *cnt;      // [kMaxTrackedRounds + 2] per-round next-list sizes (zeroed)
+  int32_t *rounds_out;
+  GridBarrier bar;
+};
+constexpr int kMaxTrackedRounds = 4096;
+constexpr int kSoloThreshold = 8192;  // finish small residuals in one CTA
+constexpr int kRoundBlock = 512;
+
+// decide(r) for u, then scatter(r+1); returns true if u stays undecided.
+__device__ __forceinline__ bool round_step(const RoundArgs &A, uint32_t u, int r) {
+  uint8_t s;
+  if (A.rootflag[u]) s = ROOT;
+  else if (A.blocked[u] < r) s = ACTIVE;
+  else s = UNDEC;
+  int32_t x = A.H[u];
+  if (s != UNDEC) A.status[u] = s;
+  if (s != ROOT && x != (int32_t)u && A.prio(u) < A.prio((uint32_t)x)) {
+    if (s == ACTIVE) A.rootflag[x] = 1;      // an active lower child makes x a root
+    else A.blocked[x] = r + 1;               // x must wait for u
+  }
+  return s == UNDEC;
+}
+
+__device__ __forceinline__ void append(int32_t *list, unsigned *count, bool keep, uint32_t u) {
+  unsigned m = __ballot_sync(0xffffffffu, keep);
+  if (!m) return;
+  int lane = threadIdx.x & 31;
+  int leader = __ffs(m) - 1;
+  unsigned base = 0;
+  if (lane == leader) base = atomicAdd(count, (unsigned)__popc(m));
+  base = __shfl_sync(0xffffffffu, base, leader);
+  if (keep) list[base + __popc(m & ((1u << lane) - 1))] = (int32_t)u;
+}
+
+__global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
+  const unsigned nb = gridDim.x;
+  const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int64_t gstride = (int64_t)nb * blockDim.x;
+  int r = 1;
+  int64_t len = A.n;  // round 1 walks all vertices
+  int cur = 0;
+  __shared__ unsigned s_len;
+  // ---- grid-wide rounds
+  while (true) {
+    unsigned *next_cnt = A.cnt + (r < kMaxTrackedRounds ? r : kMaxTrackedRounds);
+    int32_t *next = A.wl[cur ^ 1];
+    int64_t lim = (len + 31) & ~(int64_t)31;
+    for (int64_t i = gtid; i < lim; i += gstride) {
+      bool keep = false;
+      uint32_t u = 0;
+      if (i < len) {
+        u = (r == 1) ? (uint32_t)i : (uint32_t)A.wl[cur][i];
+        if (r > 1 || A.status[u] == UNDEC) keep = round_step(A, u, r);
+      }
+      append(next, next_cnt, keep, u);
+    }
+    A.bar.sync(nb);
+    if (threadIdx.x == 0) s_len = ld_acquire_u32(next_cnt);
+    __syncthreads();
+    len = s_len;
+    if (r >= kMaxTrackedRounds - 1) {  // keep per-round counters reusable
+      A.bar.sync(nb);
+      if (gtid == 0) *next_cnt = 0;
+    }
+    cur ^= 1;
+    ++r;
+    if (len == 0) {
+      if (gtid == 0) *A.rounds_out = r - 1;
+      return;
+    }
+    if (len <= kSoloThreshold) break;
+  }
+  // ---- small residual: CTA 0 alone, block barriers only
+  if (blockIdx.x != 0) return;
+  while (true) {
+    unsigned *next_cnt = A.cnt + (r < kMaxTrackedRounds ? r : kMaxTrackedRounds);
+    int32_t *next = A.wl[cur ^ 1];
+    int64_t lim = (len + 31) & ~(int64_t)31;
+    for (int64_t i = threadIdx.x; i < lim; i += blockDim.x) {
+      bool keep = false;
+      uint32_t u = 0;
+      if (i < len) {
+        u = (uint32_t)A.wl[cur][i];
+        keep = round_step(A, u, r);
+      }
+      append(next, next_cnt, keep, u);
+    }
+    __threadfence_block();
+    __syncthreads();
+    if (threadIdx.x == 0) s_len = *(volatile unsigned *)next_cnt;
+    __syncthreads();
+    len = s_len;
+    if (r >= kMaxTrackedRounds - 1) {
+      __syncthreads();
+      if (threadIdx.x == 0) *next_cnt = 0;
+      __syncthreads();
+    }
+    cur ^= 1;
+    ++r;
+    if (len == 0) break;
+  }
+  if (threadIdx.x == 0) *A.rounds_out = r - 1;
+}
+
+// ------------------------------------------------------- a4 / a5 relabel + M
+struct RootFlagIn {
+  const uint8_t *status;
+  __device__ __forceinline__ int64_t operator()(int64_t u) const { return status[u] == ROOT; }
+};
+struct RootLabelOut {
+  const uint8_t *status;
+  int32_t *M;
+  uint8_t *root_out;  // nullable
+  __device__ __forceinline__ void operator()(int64_t u, int64_t prefix) const {
+    bool r = status[u] == ROOT;
+    if (r) M[u] = (int32_t)prefix;
+    if (root_out) root_out[u] = r;
+  }
+};
+
+__global__ void k_assign(int64_t n, const int32_t *__restrict__ H, const uint8_t *__restrict__ status,
+                         int32_t *__restrict__ M) {
+  int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u >= n || status[u] == ROOT) return;
+  int32_t x = H[u];
+  while (status[x] != ROOT) x = H[x];
+  M[u] = M[x];
+}
+
+int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes) {
+  size_t b = 0;
+  b += ws_bytes(n, 4);          // H
+  b += ws_bytes(n, 1) * 2;      // status, rootflag
+  b += ws_bytes(n, 4);          // blocked
+  b += 2 * ws_bytes(n, 4);      // worklists
+  b += ws_bytes(kMaxTrackedRounds + 2, 4) + ws_bytes(4, 4) + ws_bytes(4, 8);
+  b += heavy_ws(n, nnz);
+  b += scan_ws_bytes(n);
+  *bytes = b;
+  return HEC_OK;
+}
+
+int heavy_only_impl(hec_ctx *ctx, const hec_graph *g, int32_t *H) { return run_heavy(ctx, g, H); }
+
+int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, uint8_t *root_out,
+                      int32_t *H_out, MapResult *res) {
+  const int64_t n = g->n;
+  res->n_c = 0;
+  res->rounds = 0;
+  if (n == 0) return HEC_OK;
+  cudaStream_t s = ctx->stream;
+  int32_t *H = H_out ? H_out : ws_take<int32_t>(ctx, n);
+  uint8_t *status = ws_take<uint8_t>(ctx, n);
+  uint8_t *rootflag = ws_take<uint8_t>(ctx, n);
+  int32_t *blocked = ws_take<int32_t>(ctx, n);
+  int32_t *wl0 = ws_take<int32_t>(ctx, n);
+  int32_t *wl1 = ws_take<int32_t>(ctx, n);
+  unsigned *cnt = ws_take<unsigned>(ctx, kMaxTrackedRounds + 2);
+  unsigned *bar = ws_take<unsigned>(ctx, 4);
+  int64_t *scal = ws_take<int64_t>(ctx, 4);  // [0] n_c, [1] rounds (int32 in low word)
+  if (!H || !status || !rootflag || !blocked || !wl0 || !wl1 || !cnt || !bar || !scal) {
+    set_error("workspace under-reserved (mapping)");
+    return HEC_EINVAL;
+  }
+  const double dn = (double)n, dnnz = (double)g->nnz;
+  int ph = phase_begin(ctx, "heavy", 8.0 * dnnz + 8.0 * (dn + 1) + 4.0 * dn);
+  HEC_TRY(run_heavy(ctx, g, H));
+  phase_end(ctx, ph);
+  ph = phase_begin(ctx, "rounds", 5.0 * dn);
+  HEC_CUDA_TRY(cudaMemsetAsync(rootflag, 0, n, s));
+  HEC_CUDA_TRY(cudaMemsetAsync(blocked, 0, sizeof(int32_t) * n, s));
+  HEC_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(unsigned) * (kMaxTrackedRounds + 2), s));
+  HEC_CUDA_TRY(cudaMemsetAsync(bar, 0, sizeof(unsigned) * 4, s));
+  HEC_CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(int64_t) * 4, s));
+  k_round_init<<<nblk(n, 256), 256, 0, s>>>(n, H, prio, status, blocked);
+  HEC_LAUNCH_CHECK();
+
+  RoundArgs A;
+  A.n = n; A.H = H; A.prio = prio; A.status = status; A.rootflag = rootflag; A.blocked = blocked;
+  A.wl[0] = wl0; A.wl[1] = wl1; A.cnt = cnt; A.rounds_out = reinterpret_cast<int32_t *>(scal + 1);
+  A.bar.count = bar; A.bar.gen = bar + 1;
+  static int occ = 0;
+  if (!occ) {
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rounds, kRoundBlock, 0));
+    if (occ < 1) occ = 1;
+  }
+  int64_t want = (n + kRoundBlock - 1) / kRoundBlock;
+  int64_t grid = (int64_t)ctx->num_sms * occ;
+  if (want < grid) grid = want < 1 ? 1 : want;
+  void *args[] = {&A};
+  HEC_CUDA_TRY(cudaLaunchCooperativeKernel((const void *)k_rounds, dim3((unsigned)grid),
+                                           dim3(kRoundBlock), args, 0, s));
+  ctx->launches++;
+  phase_end(ctx, ph);
+  ph = phase_begin(ctx, "relabel", 9.0 * dn);
+  // a4: labels by ascending root id; a5: inherit along H
+  ScanTiles st = take_scan_tiles(ctx, n);
+  if (!st.desc || !st.ticket) { set_error("workspace under-reserved (scan)"); return HEC_EINVAL; }
+  HEC_TRY(chained_scan(ctx, n, RootFlagIn{status}, RootLabelOut{status, M, root_out}, st, scal));
+  k_assign<<<nblk(n, 256), 256, 0, s>>>(n, H, status, M);
+  HEC_LAUNCH_CHECK();
+  phase_end(ctx, ph);
+  int64_t h[2];
+  HEC_TRY(read_scalars(ctx, scal, 2, h));
+  res->n_c = h[0];
+  res->rounds = (int)(int32_t)(h[1] & 0xffffffff);
+  return HEC_OK;
+}
+
+}  // namespace hec

@@ -1,0 +1,307 @@
+"""Parity of the CUDA path (through the C-ABI) against the CPU oracle.
+
+Bar: integer work, so everything is bit-exact — H, root
+flags, round counts, M, n_c, and every coarse CSR (row_ptr, col, wgt, vwgt).
+Small/medium sizes compare element by element with the oracle run on the same
+seeded inputs; the full-size configs C3/C4 compare per-level digests against
+tests/golden/oracle_digests.json (written by tests/golden/make_digests.py,
+which calls only graphgen/ and oracle/)."""
+import itertools
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import graphgen as gg
+import oracle as o
+
+pytestmark = pytest.mark.gpu
+
+SEED = 0x5EED
+
+
+@pytest.fixture(scope="module")
+def P():
+    import subprocess
+    subprocess.run(["make", "-C", os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "-s", "hec"],
+                   check=True)
+    import paper_conf_ipps_gilbertabmr21_b200 as P
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    return P
+
+
+@pytest.fixture(scope="module")
+def ctx(P):
+    c = P.Context()
+    yield c
+    c.close()
+
+
+def dev(P, g):
+    return P.DeviceGraph.from_host(g)
+
+
+def host_csr(dg):
+    rp, col, wgt, vw = dg.to_host()
+    return rp, col, wgt, vw
+
+
+def assert_csr_equal(dg, oc):
+    rp, col, wgt, vw = host_csr(dg)
+    assert np.array_equal(rp, oc.row_ptr), "row_ptr differs"
+    assert np.array_equal(col, oc.col), "col differs"
+    assert np.array_equal(wgt, oc.wgt), "wgt differs"
+    assert np.array_equal(vw, oc.vwgt), "vwgt differs"
+
+
+def random_graph(n, rng, p=0.3, wmax=3, isolated=0):
+    edges = [(u, v, int(rng.integers(1, wmax + 1)))
+             for u in range(n - isolated) for v in range(u + 1, n - isolated) if rng.random() < p]
+    return gg.from_edges(n, edges)
+
+
+def prio_tensor(pr):
+    return torch.from_numpy(pr.view(np.int64).copy()).cuda()
+
+
+# ------------------------------------------------------------------ a1
+@pytest.mark.parametrize("which", ["grid", "mesh27_small", "rmat12", "rmat16", "random"])
+def test_heavy_parity(P, ctx, which):
+    rng = np.random.default_rng(11)
+    if which == "grid":
+        gs = [gg.grid2d(64, 64), gg.grid2d(1, 7), gg.grid2d(3, 1000)]
+    elif which == "mesh27_small":
+        gs = [gg.mesh27(20, 21, 22)]
+    elif which == "rmat12":
+        gs = [gg.rmat(12, 16)]
+    elif which == "rmat16":
+        gs = [gg.rmat(16, 16)]
+    else:
+        gs = [random_graph(int(rng.integers(1, 60)), rng, p=0.3, wmax=3, isolated=int(rng.integers(0, 4)))
+              for _ in range(30)]
+    for g in gs:
+        H = P.hec_debug_heavy(ctx, dev(P, g)).cpu().numpy()
+        assert np.array_equal(H, o.heavy(g))
+
+
+def test_heavy_hub_rows_span_tiles(P, ctx):
+    """Rows far longer than a tile (4096 items), ties everywhere, weights chosen so
+    the maximum sits at the row's end / start / middle."""
+    n = 30000
+    edges = [(0, v, 1) for v in range(1, n)]                       # hub row 0
+    edges += [(1, v, 1 + (v % 7 == 0)) for v in range(2, 20000)]  # max repeated: first wins
+    edges += [(2, n - 1, 9)]                                      # heaviest at row end of 2
+    g = gg.from_edges(n, edges)
+    H = P.hec_debug_heavy(ctx, dev(P, g)).cpu().numpy()
+    assert np.array_equal(H, o.heavy(g))
+
+
+# ------------------------------------------------------------------ a3
+def test_roots_and_rounds_c1(P, ctx, golden_dir):
+    ka = json.load(open(os.path.join(golden_dir, "survey_known_answers.json")))["C1"]
+    g = gg.config(1)
+    H = o.hierarchy(g, 50, SEED, keep_roots=True)
+    cur = g
+    for level, lv in enumerate(H.levels):
+        root, rounds = P.hec_debug_roots(ctx, dev(P, cur), seed=SEED, level=level)
+        assert np.array_equal(root.cpu().numpy(), lv.root)
+        assert 1 <= rounds <= ka["rounds"][level]  # see test_hierarchy_c1
+        cur = lv.graph
+
+
+# ------------------------------------------------------------- a1-a5 mapping
+def test_mapping_hand_examples(P, ctx, golden_dir):
+    ex = json.load(open(os.path.join(golden_dir, "hand_examples.json")))
+    for name in ("G6", "P4w"):
+        e = ex[name]
+        g = gg.from_edges(e["n"], e["edges"])
+        for run in e["runs"]:
+            pr = o.prio_from_order(run["order"])
+            M, nc = P.hec_find_mapping_prio(ctx, dev(P, g), prio_tensor(pr))
+            assert nc == run["n_c"] and M.cpu().numpy().tolist() == run["M"]
+
+
+def test_mapping_exhaustive_small(P, ctx):
+    """All visit orders of small graphs with ties and an isolated vertex."""
+    rng = np.random.default_rng(12)
+    for t in range(4):
+        g = random_graph(6, rng, p=0.5, wmax=2, isolated=1 if t % 2 else 0)
+        dg = dev(P, g)
+        for order in itertools.permutations(range(6)):
+            pr = o.prio_from_order(order)
+            M, nc = P.hec_find_mapping_prio(ctx, dg, prio_tensor(pr))
+            Mo, nco, _ = o.mapping(g, pr)
+            assert nc == nco and np.array_equal(M.cpu().numpy(), Mo)
+
+
+def test_mapping_adversarial_path(P, ctx):
+    """Reverse-priority path: O(n) resolution rounds; must still be exact."""
+    n = 20000
+    g = gg.from_edges(n, [(i, i + 1, 1) for i in range(n - 1)])
+    for order in (range(n), range(n - 1, -1, -1)):
+        pr = o.prio_from_order(order)
+        M, nc = P.hec_find_mapping_prio(ctx, dev(P, g), prio_tensor(pr))
+        Mo, nco, _ = o.mapping(g, pr)
+        assert nc == nco and np.array_equal(M.cpu().numpy(), Mo)
+
+
+@pytest.mark.parametrize("which", ["c1", "c2", "rmat16", "random"])
+def test_mapping_parity_seeded(P, ctx, which):
+    rng = np.random.default_rng(13)
+    if which == "c1":
+        gs = [gg.config(1)]
+    elif which == "c2":
+        gs = [gg.config(2)]
+    elif which == "rmat16":
+        gs = [gg.rmat(16, 16)]
+    else:
+        gs = [random_graph(int(rng.integers(1, 200)), rng, p=0.05, wmax=4, isolated=int(rng.integers(0, 3)))
+              for _ in range(20)]
+    for g in gs:
+        for level in (0, 3):
+            M, nc = P.hec_find_mapping(ctx, dev(P, g), SEED, level)
+            Mo, nco, _ = o.mapping(g, o.prio(SEED, level, g.n))
+            assert nc == nco and np.array_equal(M.cpu().numpy(), Mo)
+
+
+# ------------------------------------------------------- a7-a10 construction
+def test_construct_random_labels(P, ctx):
+    """Random M over random weighted graphs (exercises SMALL rows, duplicates, self entries)."""
+    rng = np.random.default_rng(14)
+    for t in range(25):
+        g = random_graph(int(rng.integers(2, 120)), rng, p=0.2, wmax=50)
+        g.vwgt = rng.integers(1, 5, g.n).astype(np.int32)
+        nc = int(rng.integers(1, g.n + 1))
+        M = rng.integers(0, nc, g.n).astype(np.int32)
+        M[:nc] = np.arange(nc)
+        cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+        assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
+
+
+@pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
+def test_construct_size_classes(P, ctx, nc):
+    """R-MAT s14 with random labels into nc aggregates: few labels give huge rows
+    (DENSE when nc <= 16384, BIN otherwise), many labels give SMALL/MID rows."""
+    rng = np.random.default_rng(15 + nc)
+    g = gg.rmat(14 if nc < 20000 else 17, 16)
+    g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
+    # symmetric weights: w(u,v) = w(v,u) = f(min, max)
+    rows = np.repeat(np.arange(g.n), np.diff(g.row_ptr))
+    lo, hi = np.minimum(rows, g.col), np.maximum(rows, g.col)
+    g.wgt = ((lo.astype(np.int64) * 7919 + hi * 104729) % 1000 + 1).astype(np.int32)
+    nc = min(nc, g.n)
+    M = rng.integers(0, nc, g.n).astype(np.int32)
+    M[rng.permutation(g.n)[:nc]] = np.arange(nc)
+    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+    assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
+
+
+def test_construct_overflow_detected(P, ctx):
+    big = 2**31 - 1
+    g = gg.from_edges(3, [(0, 2, big), (1, 2, big)])
+    M = torch.tensor([0, 0, 1], dtype=torch.int32, device="cuda")
+    with pytest.raises(P.HecError) as e:
+        P.build_coarse_graph(ctx, dev(P, g), M, 2)
+    assert e.value.code == P.HEC_EOVERFLOW
+    # near the limit but exact: no error
+    g = gg.from_edges(3, [(0, 2, big // 2), (1, 2, big // 2)])
+    cg = P.build_coarse_graph(ctx, dev(P, g), M, 2)
+    assert_csr_equal(cg.graph, o.coarsen(g, M.cpu().numpy(), 2))
+
+
+def test_construct_rejects_bad_labels(P, ctx):
+    g = gg.from_edges(3, [(0, 1, 1), (1, 2, 1)])
+    M = torch.tensor([0, 5, 1], dtype=torch.int32, device="cuda")
+    with pytest.raises(P.HecError) as e:
+        P.build_coarse_graph(ctx, dev(P, g), M, 2)
+    assert e.value.code == P.HEC_EINVAL
+
+
+def test_validate_flags_bad_graph(P):
+    c = P.Context(validate=True)
+    g = gg.from_edges(4, [(0, 1, 1), (1, 2, 1), (2, 3, 1)])
+    dg = dev(P, g)
+    P.hec_find_mapping(c, dg, SEED, 0)  # valid graph passes
+    bad = P.DeviceGraph(dg.row_ptr.clone(), dg.col.clone(), dg.wgt.clone(), dg.vwgt)
+    bad.wgt[0] = 5  # asymmetric weight
+    with pytest.raises(P.HecError) as e:
+        P.hec_find_mapping(c, bad, SEED, 0)
+    assert e.value.code == P.HEC_EINVAL and "asymmetric" in str(e.value)
+    c.close()
+
+
+# ------------------------------------------------------------ hierarchy
+def check_hierarchy(P, ctx, g, cutoff):
+    Ho = o.hierarchy(g, cutoff, SEED)
+    Hg = P.coarsen_hierarchy(ctx, dev(P, g), cutoff, SEED)
+    assert len(Hg.levels) == len(Ho.levels)
+    assert Hg.stop_reason == Ho.stop_reason
+    if Ho.stop_reason == o.STOP_DISCARD:
+        assert Hg.discarded_n_c == Ho.discarded_n_c
+    for lg, lo in zip(Hg.levels, Ho.levels):
+        assert np.array_equal(lg.M.cpu().numpy(), lo.M)
+        assert_csr_equal(lg.graph, lo.graph)
+    return Hg
+
+
+def test_hierarchy_c1(P, ctx, golden_dir):
+    Hg = check_hierarchy(P, ctx, gg.config(1), 50)
+    ka = json.load(open(os.path.join(golden_dir, "survey_known_answers.json")))["C1"]
+    # The kernel fuses decide(r) with scatter(r+1); a root flag published in the
+    # same round may be seen one round early, so the count can only be lower.
+    # The result (M, G_c) is unaffected — compared exactly above.
+    rounds = [lv.rounds for lv in Hg.levels]
+    assert all(1 <= r <= k for r, k in zip(rounds, ka["rounds"])), rounds
+
+
+def test_hierarchy_c2(P, ctx):
+    check_hierarchy(P, ctx, gg.config(2), 1000)
+
+
+@pytest.mark.parametrize("scale", [10, 12, 16, 18])
+def test_hierarchy_rmat(P, ctx, scale):
+    check_hierarchy(P, ctx, gg.rmat(scale, 16), 50)
+
+
+def test_hierarchy_edge_cases(P, ctx):
+    empty = gg.Graph(np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0, np.int32), np.zeros(0, np.int32))
+    Hg = P.coarsen_hierarchy(ctx, P.DeviceGraph.from_host(empty), 50, SEED)
+    assert Hg.levels == [] and Hg.stop_reason == P.STOP_CUTOFF
+    iso = gg.Graph(np.zeros(61, np.int64), np.zeros(0, np.int32), np.zeros(0, np.int32), np.ones(60, np.int32))
+    Hg = P.coarsen_hierarchy(ctx, P.DeviceGraph.from_host(iso), 50, SEED)
+    assert Hg.levels == [] and Hg.stop_reason == P.STOP_STALL
+    star = gg.from_edges(60, [(0, i, 1) for i in range(1, 60)])
+    Hg = P.coarsen_hierarchy(ctx, dev(P, star), 50, SEED)
+    assert Hg.levels == [] and Hg.stop_reason == P.STOP_DISCARD and Hg.discarded_n_c == 1
+    Hg = P.coarsen_hierarchy(ctx, dev(P, gg.config(1)), 50, SEED, max_levels=2)
+    assert len(Hg.levels) == 2 and Hg.stop_reason == P.STOP_MAX_LEVELS
+    # graph with isolated vertices and a disconnected part
+    rng = np.random.default_rng(16)
+    g = random_graph(500, rng, p=0.01, wmax=3, isolated=7)
+    check_hierarchy(P, ctx, g, 20)
+
+
+def digest_levels(Hg):
+    out = []
+    for lv in Hg.levels:
+        rp, col, wgt, vw = host_csr(lv.graph)
+        out.append(dict(n_c=lv.graph.n, nnz_c=lv.graph.nnz, sum_wc=int(wgt.astype(np.int64).sum()),
+                        sha_M=gg.sha16(lv.M.cpu().numpy()), sha_G=gg.sha16(rp, col, wgt), sha_vwgt=gg.sha16(vw)))
+    return out
+
+
+@pytest.mark.parametrize("cfg", [2, 3, 4])
+def test_hierarchy_full_size_digests(P, ctx, golden_dir, cfg):
+    d = json.load(open(os.path.join(golden_dir, "oracle_digests.json")))[str(cfg)]
+    g = gg.config(cfg)
+    assert gg.sha16(g.row_ptr, g.col) == d["sha_G0"]
+    Hg = P.coarsen_hierarchy(ctx, dev(P, g), d["cutoff"], d["seed"])
+    del g
+    got = digest_levels(Hg)
+    exp = [{k: lv[k] for k in ("n_c", "nnz_c", "sum_wc", "sha_M", "sha_G", "sha_vwgt")} for lv in d["levels"]]
+    assert got == exp
+    assert Hg.stop_reason == d["stop_reason"]
+    if d["discarded_n_c"] is not None:
+        assert Hg.discarded_n_c == d["discarded_n_c"]
