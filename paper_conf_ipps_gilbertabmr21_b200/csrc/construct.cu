@@ -27,91 +27,14 @@
 //      order and each obtains its output offset with a decoupled look-back over
 //      block totals, then writes col_c/wgt_c/row_ptr_c/vwgt_c in place (no
 //      scratch + compaction pass).
-#include "hec_internal.cuh"
+#include <stdlib.h>
+
+#include "construct_common.cuh"
 
 namespace hec {
 
-constexpr int kT = 512;            // threads per CTA of the row kernels
-constexpr int kIt = 8;             // entries held per thread (registers)
-constexpr int kCap = kT * kIt;     // entries per work block (4096)
-constexpr int kWin = 2048;         // window weight; a block's weight is < 2*kWin
-constexpr int kRowW = 8;           // per-row weight: bounds rows per block
-constexpr int kMaxRows = 2 * kWin / kRowW;   // 512
-constexpr int kSmallMax = kWin - kRowW;      // rows with U <= 2040 are small
-constexpr int kMC = 1024;          // member-table chunk
-constexpr int kBucketAvg = 1024;   // target entries per BUCKET
-constexpr int kDenseMax = 32768;   // n_c bound of the DENSE skew path
 constexpr int kFbTab = 16384;      // fallback hash slots (int64 values)
 constexpr int kFbCap = 8192;       // fallback distinct keys per sub-range pass
-constexpr int32_t kEmpty = -1;
-
-enum : int32_t { B_SMALL = 0, B_BUCKET = 1, B_DENSE = 2 };
-
-static inline unsigned nblk(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
-
-// ----------------------------------------------------------------- helpers
-// largest i in [lo, hi) with a[i] <= x (a non-decreasing, a[lo] <= x)
-template <typename T>
-__device__ __forceinline__ int64_t last_le(const T *a, int64_t lo, int64_t hi, int64_t x) {
-  hi -= 1;
-  while (lo < hi) {
-    int64_t mid = (lo + hi + 1) >> 1;
-    if ((int64_t)a[mid] <= x) lo = mid;
-    else hi = mid - 1;
-  }
-  return lo;
-}
-
-// In-place exclusive scan of n <= kCap+1 int32 values in shared memory by a CTA
-// of kT threads; returns the total.  `tmp` holds >= 33 ints.
-__device__ int smem_exclusive_scan(int32_t *a, int n, int32_t *tmp) {
-  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
-  const int chunk = (n + kT - 1) / kT;
-  const int beg = t * chunk;
-  int local = 0;
-  for (int i = 0; i < chunk && beg + i < n; ++i) local += a[beg + i];
-  int x = local;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    int y = __shfl_up_sync(0xffffffffu, x, o);
-    if (lane >= o) x += y;
-  }
-  if (lane == 31) tmp[wid] = x;
-  __syncthreads();
-  if (wid == 0) {
-    int w = lane < kT / 32 ? tmp[lane] : 0;
-    int ws = w;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      int y = __shfl_up_sync(0xffffffffu, ws, o);
-      if (lane >= o) ws += y;
-    }
-    if (lane < kT / 32) tmp[lane] = ws - w;
-    if (lane == kT / 32 - 1) tmp[32] = ws;
-  }
-  __syncthreads();
-  int run = tmp[wid] + x - local;
-  for (int i = 0; i < chunk && beg + i < n; ++i) {
-    int v = a[beg + i];
-    a[beg + i] = run;
-    run += v;
-  }
-  int total = tmp[32];
-  __syncthreads();
-  return total;
-}
-
-__device__ __forceinline__ int block_sum(int v, int32_t *tmp) {
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-  if (lane == 0) tmp[wid] = v;
-  __syncthreads();
-  int s = 0;
-  for (int w = 0; w < kT / 32; ++w) s += tmp[w];
-  __syncthreads();
-  return s;
-}
 
 __device__ __forceinline__ unsigned hslot(int32_t b, unsigned mask) {
   return ((uint32_t)b * 0x9E3779B1u) >> 7 & mask;
@@ -140,6 +63,10 @@ __global__ void k_member_fill(int64_t n, int64_t n_c, const int32_t *__restrict_
   members[member_ptr[a] + k] = (int32_t)u;
 }
 
+struct BlkCntIn {
+  const int32_t *c;
+  __device__ __forceinline__ int64_t operator()(int64_t i) const { return c[i]; }
+};
 struct CountIn {
   const unsigned *c;
   __device__ __forceinline__ int64_t operator()(int64_t i) const { return c[i]; }
@@ -157,19 +84,6 @@ struct DegIn {
     int32_t u = members[i];
     return row_ptr[u + 1] - row_ptr[u];
   }
-};
-
-struct Layout {
-  int64_t n_c;
-  const int64_t *member_ptr;  // [n_c+1]
-  const int32_t *members;     // [n]
-  const int64_t *mpre;        // [n+1] member-edge prefix
-  const int64_t *row_ptr;
-  const int32_t *col;
-  const int32_t *wgt;
-  const int32_t *M;
-  __device__ __forceinline__ int64_t upos(int64_t a) const { return mpre[member_ptr[a]]; }
-  __device__ __forceinline__ int64_t U(int64_t a) const { return upos(a + 1) - upos(a); }
 };
 
 // window weight of small rows (U + kRowW), 0 for big rows
@@ -236,13 +150,6 @@ struct BlockCountIn {
   }
 };
 
-struct BlockDesc {
-  int32_t kind;
-  int32_t row0;  // first row (SMALL) / the row (BUCKET, DENSE)
-  int32_t row1;  // one past the last row (SMALL)
-  int32_t sub;   // bucket index within the row / dense key chunk
-};
-
 __global__ void k_block_desc(Layout L, const int64_t *__restrict__ blk_ptr, const int32_t *__restrict__ big_idx,
                              bool dense, BlockDesc *__restrict__ blk) {
   int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -261,378 +168,6 @@ __global__ void k_block_ends(int64_t nblocks, int64_t n_c, BlockDesc *__restrict
   int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= nblocks) return;
   if (blk[k].kind == B_SMALL) blk[k].row1 = (k + 1 < nblocks) ? blk[k + 1].row0 : (int32_t)n_c;
-}
-
-// ------------------------------------------------------------- expansion
-struct MemberTab {
-  int64_t mstart[kMC];     // row_ptr[u] of the member
-  int32_t moff[kMC + 1];   // member's first position relative to the window start
-  int32_t mrow[kMC];       // local row of the member
-};
-
-// Expand the member-edge window [P0, P0+nP) (nP <= kCap), whose members are
-// [m0, m1), into registers: slot s = tid + kT*k holds (b = M[v], w, local row).
-// Slots without an entry keep kb = -1.  s_mptr[0..R]: member_ptr slice of the
-// rows (nullptr => one row, index 0).
-__device__ __forceinline__ void expand_window(const Layout &L, MemberTab &T, int64_t P0, int nP, int64_t m0,
-                                              int64_t m1, const int64_t *s_mptr, int R, int32_t (&kb)[kIt],
-                                              int32_t (&kw)[kIt], int32_t (&kr)[kIt]) {
-  const int t = threadIdx.x;
-#pragma unroll
-  for (int k = 0; k < kIt; ++k) { kb[k] = -1; kw[k] = 0; kr[k] = 0; }
-  for (int64_t cm = m0; cm < m1; cm += kMC) {
-    const int nm = (int)((m1 - cm) < kMC ? (m1 - cm) : kMC);
-    for (int i = t; i < nm; i += kT) {
-      int32_t u = L.members[cm + i];
-      T.mstart[i] = L.row_ptr[u];
-      T.moff[i] = (int32_t)(L.mpre[cm + i] - P0);
-      T.mrow[i] = s_mptr ? (int32_t)last_le(s_mptr, 0, R, cm + i) : 0;
-    }
-    if (t == 0) {
-      int64_t e = L.mpre[cm + nm] - P0;
-      T.moff[nm] = (int32_t)(e > (int64_t)kCap + 1 ? kCap + 1 : e);
-    }
-    __syncthreads();
-    const int lo = T.moff[0] > 0 ? T.moff[0] : 0;
-    const int hi = T.moff[nm] < nP ? T.moff[nm] : nP;
-    unsigned fresh = 0;
-    int64_t ev[kIt];
-#pragma unroll
-    for (int k = 0; k < kIt; ++k) {
-      const int s = t + kT * k;
-      ev[k] = 0;
-      if (s >= lo && s < hi) {
-        int i = (int)last_le(T.moff, 0, nm, s);
-        ev[k] = T.mstart[i] + (s - T.moff[i]);
-        kr[k] = T.mrow[i];
-        fresh |= 1u << k;
-      }
-    }
-#pragma unroll
-    for (int k = 0; k < kIt; ++k)
-      if (fresh & (1u << k)) { kb[k] = __ldg(L.col + ev[k]); kw[k] = __ldg(L.wgt + ev[k]); }
-#pragma unroll
-    for (int k = 0; k < kIt; ++k)
-      if (fresh & (1u << k)) kb[k] = __ldg(L.M + kb[k]);
-    __syncthreads();
-  }
-}
-
-// Members of a big row covering the window [P0, P0+nP): [m0, m1).
-__device__ __forceinline__ void window_members(const Layout &L, int32_t a, int64_t P0, int nP, int64_t *m0,
-                                               int64_t *m1) {
-  const int64_t m0r = L.member_ptr[a], m1r = L.member_ptr[a + 1];
-  *m0 = last_le(L.mpre, m0r, m1r, P0);
-  int64_t lo = *m0, hi = m1r - 1;  // last member i with mpre[i] < P0 + nP
-  while (lo < hi) {
-    int64_t mid = (lo + hi + 1) >> 1;
-    if (L.mpre[mid] < P0 + nP) lo = mid;
-    else hi = mid - 1;
-  }
-  *m1 = lo + 1;
-}
-
-// ---------------------------------------------------- bucket sort + dedup
-struct RowsSmem {
-  MemberTab T;
-  int64_t mptr[kMaxRows + 1];
-  int32_t row_id[kMaxRows];
-  int32_t kmin[kMaxRows];
-  int32_t kmax[kMaxRows];
-  int32_t bbase[kMaxRows + 1];
-  float bscale[kMaxRows];
-  int32_t hist[kCap + 1];  // bucket histogram -> bucket offsets
-  int32_t ucnt[kCap + 1];  // unique count per bucket -> output offsets
-  int32_t pb[kCap];        // pairs in bucket order
-  int32_t pw[kCap];
-  int32_t tmp[40];
-  int64_t prefix;
-  int32_t blk;
-  int32_t nbins;
-};
-
-__device__ __forceinline__ int warp_min(int v) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, o));
-  return v;
-}
-__device__ __forceinline__ int warp_max(int v) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v = max(v, __shfl_xor_sync(0xffffffffu, v, o));
-  return v;
-}
-
-// Key range per local row over the valid register entries.
-__device__ __forceinline__ void row_key_range(RowsSmem &S, const int32_t (&kb)[kIt], const int32_t (&kr)[kIt]) {
-#pragma unroll
-  for (int k = 0; k < kIt; ++k) {
-    const bool valid = kb[k] >= 0;
-    const int r = valid ? kr[k] : -1;
-    const int r0 = __shfl_sync(0xffffffffu, r, 0);
-    if (__all_sync(0xffffffffu, r == r0)) {
-      if (r0 >= 0) {
-        int mn = warp_min(kb[k]), mx = warp_max(kb[k]);
-        if ((threadIdx.x & 31) == 0) { atomicMin(&S.kmin[r0], mn); atomicMax(&S.kmax[r0], mx); }
-      }
-    } else if (valid) {
-      atomicMin(&S.kmin[r], kb[k]);
-      atomicMax(&S.kmax[r], kb[k]);
-    }
-  }
-}
-
-// Bucket-sort the register entries of rows 0..R-1 (key ranges in kmin/kmax,
-// entry bounds rowU) and merge duplicates.  Leaves S.hist = bucket offsets into
-// pb/pw, S.ucnt = exclusive offsets of the unique entries per bucket (S.ucnt[nbins]
-// = total), returns the number of unique entries.  A merged weight above
-// INT32_MAX sets err bit 2 (exact: sums are int64).
-__device__ int sort_dedup(RowsSmem &S, int R, const int64_t *rowU, int32_t (&kb)[kIt], int32_t (&kw)[kIt],
-                          int32_t (&kr)[kIt], int *err) {
-  const int t = threadIdx.x;
-  for (int r = t; r < R; r += kT) {
-    int lo = S.kmin[r], hi = S.kmax[r];
-    int nb = 0;
-    if (hi >= lo) {
-      int64_t span = (int64_t)hi - lo + 1;
-      int64_t lim = rowU[r] < span ? rowU[r] : span;
-      nb = 1;
-      while ((int64_t)nb * 2 <= lim && nb * 2 <= kCap) nb *= 2;
-      S.bscale[r] = (float)nb / (float)span;
-    } else {
-      S.bscale[r] = 0.f;
-    }
-    S.bbase[r] = nb;
-  }
-  __syncthreads();
-  const int nbins = smem_exclusive_scan(S.bbase, R, S.tmp);
-  if (t == 0) S.bbase[R] = nbins;
-  for (int i = t; i <= nbins; i += kT) S.hist[i] = 0;
-  __syncthreads();
-  // bucket (monotone in the key within a row) and rank inside the bucket
-#pragma unroll
-  for (int k = 0; k < kIt; ++k) {
-    if (kb[k] >= 0) {
-      const int r = kr[k];
-      const int nb = S.bbase[r + 1] - S.bbase[r];
-      int off = (int)((float)(kb[k] - S.kmin[r]) * S.bscale[r]);
-      off = off < nb - 1 ? off : nb - 1;
-      const int bin = S.bbase[r] + off;
-      const int rank = atomicAdd(&S.hist[bin], 1);
-      kr[k] = (bin << 12) | rank;
-    }
-  }
-  __syncthreads();
-  smem_exclusive_scan(S.hist, nbins + 1, S.tmp);
-#pragma unroll
-  for (int k = 0; k < kIt; ++k) {
-    if (kb[k] >= 0) {
-      const int q = S.hist[kr[k] >> 12] + (kr[k] & 4095);
-      S.pb[q] = kb[k];
-      S.pw[q] = kw[k];
-    }
-  }
-  __syncthreads();
-  for (int bin = t; bin < nbins; bin += kT) {
-    const int lo = S.hist[bin], hi = S.hist[bin + 1];
-    for (int i = lo + 1; i < hi; ++i) {
-      int kk = S.pb[i], ww = S.pw[i];
-      int j = i - 1;
-      while (j >= lo && S.pb[j] > kk) {
-        S.pb[j + 1] = S.pb[j];
-        S.pw[j + 1] = S.pw[j];
-        --j;
-      }
-      S.pb[j + 1] = kk;
-      S.pw[j + 1] = ww;
-    }
-    int out = lo;
-    int i = lo;
-    while (i < hi) {
-      int kk = S.pb[i];
-      long long acc = 0;
-      while (i < hi && S.pb[i] == kk) acc += S.pw[i++];
-      if (acc > 0x7fffffffLL) atomicOr(err, 2);
-      S.pb[out] = kk;
-      S.pw[out] = (int32_t)acc;
-      ++out;
-    }
-    S.ucnt[bin] = out - lo;
-  }
-  __syncthreads();
-  const int T = smem_exclusive_scan(S.ucnt, nbins, S.tmp);
-  if (t == 0) { S.ucnt[nbins] = T; S.nbins = nbins; }
-  __syncthreads();
-  return T;
-}
-
-// unique entry q of the block -> (b, w); the largest bucket whose unique offset
-// is <= q is never empty, so it holds q.
-__device__ __forceinline__ void emit(const RowsSmem &S, int nbins, int T, int64_t O, int32_t *__restrict__ col_c,
-                                     int32_t *__restrict__ wgt_c) {
-  for (int q = threadIdx.x; q < T; q += kT) {
-    int bin = (int)last_le(S.ucnt, 0, nbins, q);
-    int src = S.hist[bin] + (q - S.ucnt[bin]);
-    col_c[O + q] = S.pb[src];
-    wgt_c[O + q] = S.pw[src];
-  }
-}
-
-struct RowsArgs {
-  Layout L;
-  const BlockDesc *blk;
-  int64_t nblocks;
-  unsigned *ticket;
-  uint64_t *desc;  // look-back descriptors [nblocks]
-  const unsigned long long *vw64;
-  const int32_t *big_idx;
-  // BUCKET mode
-  const int64_t *bkt_ptr;      // [nbig+1] first bucket of big row h
-  const int64_t *bkt_off;      // [nbkt+1] pair offsets
-  const int32_t *pb_g, *pw_g;  // partitioned pairs
-  const int32_t *fb_cnt;       // fallback unique count per bucket (-1: not overflowed)
-  const int64_t *fb_off;       // fallback scratch offset per bucket
-  const int32_t *fb_b, *fb_w;
-  // DENSE mode
-  const unsigned long long *dense;  // [nbig][n_c]
-  // outputs
-  int64_t *row_ptr_c;
-  int32_t *col_c, *wgt_c, *vwgt_c;
-  int *err;
-};
-
-__device__ __forceinline__ void write_vwgt(const RowsArgs &A, int32_t a) {
-  unsigned long long s = A.vw64[a];
-  if (s > 0x7fffffffull) atomicOr(A.err, 2);
-  A.vwgt_c[a] = (int32_t)s;
-}
-
-// keys b with floor(b * nb / n_c) == k: [ceil(k n_c / nb), ceil((k+1) n_c / nb))
-__device__ __forceinline__ void bucket_range(int64_t k, int64_t nb, int64_t n_c, int32_t *lo, int32_t *hi) {
-  *lo = (int32_t)((k * n_c + nb - 1) / nb);
-  int64_t h = ((k + 1) * n_c + nb - 1) / nb;
-  *hi = (int32_t)(h < n_c ? h : n_c);
-}
-
-__global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  RowsSmem &S = *reinterpret_cast<RowsSmem *>(smem_raw);
-  const int t = threadIdx.x;
-  const Layout &L = A.L;
-  int64_t *rowU = reinterpret_cast<int64_t *>(S.T.mstart);  // member table is free after expansion
-  while (true) {
-    if (t == 0) S.blk = (int32_t)atomicAdd(A.ticket, 1u);
-    __syncthreads();
-    const int64_t bi = S.blk;
-    if (bi >= A.nblocks) return;
-    const BlockDesc d = A.blk[bi];
-    int32_t kb[kIt], kw[kIt], kr[kIt];
-    int T = 0, nbins = 0, R = 1;
-    bool direct = false;  // DENSE / fallback: uniques already in key order
-    if (d.kind == B_SMALL) {
-      R = d.row1 - d.row0;
-      for (int r = t; r <= R; r += kT) {
-        S.mptr[r] = L.member_ptr[d.row0 + r];
-        if (r < R) { S.row_id[r] = d.row0 + r; S.kmin[r] = INT32_MAX; S.kmax[r] = -1; }
-      }
-      __syncthreads();
-      const int64_t m0 = S.mptr[0], m1 = S.mptr[R];
-      const int64_t P0 = L.mpre[m0];
-      const int nP = (int)(L.mpre[m1] - P0);
-      expand_window(L, S.T, P0, nP, m0, m1, S.mptr, R, kb, kw, kr);
-#pragma unroll
-      for (int k = 0; k < kIt; ++k)
-        if (kb[k] >= 0 && kb[k] == S.row_id[kr[k]]) kb[k] = -1;  // self entries are dropped (L280)
-      row_key_range(S, kb, kr);
-      for (int r = t; r < R; r += kT) rowU[r] = L.mpre[S.mptr[r + 1]] - L.mpre[S.mptr[r]];
-      __syncthreads();
-      T = sort_dedup(S, R, rowU, kb, kw, kr, A.err);
-      nbins = S.nbins;
-    } else if (d.kind == B_BUCKET) {
-      const int32_t h = A.big_idx[d.row0];
-      const int64_t bk = A.bkt_ptr[h] + d.sub;
-      const int64_t q0 = A.bkt_off[bk], cnt = A.bkt_off[bk + 1] - q0;
-      if (A.fb_cnt[bk] >= 0) {
-        T = A.fb_cnt[bk];
-        direct = true;
-      } else {
-        const int64_t nb = A.bkt_ptr[h + 1] - A.bkt_ptr[h];
-        int32_t lo, hi;
-        bucket_range(d.sub, nb, L.n_c, &lo, &hi);
-#pragma unroll
-        for (int k = 0; k < kIt; ++k) {
-          const int s = t + kT * k;
-          kb[k] = -1;
-          kr[k] = 0;
-          kw[k] = 0;
-          if (s < cnt) { kb[k] = A.pb_g[q0 + s]; kw[k] = A.pw_g[q0 + s]; }
-        }
-        if (t == 0) { S.kmin[0] = lo; S.kmax[0] = hi - 1; rowU[0] = cnt; }
-        __syncthreads();
-        T = sort_dedup(S, 1, rowU, kb, kw, kr, A.err);
-        nbins = S.nbins;
-      }
-    } else {  // B_DENSE: key chunk [k0, k0 + kCap) of a dense row, in key order
-      const int32_t h = A.big_idx[d.row0];
-      const int64_t k0 = (int64_t)d.sub * kCap;
-      const unsigned long long *row = A.dense + (int64_t)h * L.n_c;
-      unsigned long long v[kIt];
-      int c = 0;
-#pragma unroll
-      for (int k = 0; k < kIt; ++k) {  // blocked: thread t owns keys k0 + t*kIt + k
-        const int64_t key = k0 + (int64_t)t * kIt + k;
-        v[k] = key < L.n_c ? row[key] : 0ull;
-        c += v[k] != 0;
-      }
-      S.ucnt[t] = c;
-      __syncthreads();
-      T = smem_exclusive_scan(S.ucnt, kT, S.tmp);
-      int pos = S.ucnt[t];
-#pragma unroll
-      for (int k = 0; k < kIt; ++k) {
-        if (v[k] != 0) {
-          if (v[k] > 0x7fffffffull) atomicOr(A.err, 2);
-          S.pb[pos] = (int32_t)(k0 + (int64_t)t * kIt + k);
-          S.pw[pos] = (int32_t)v[k];
-          ++pos;
-        }
-      }
-      __syncthreads();
-      direct = true;
-    }
-    // ---- a10: decoupled look-back over block totals, then write in place
-    if (t < 32) {
-      int64_t p = lookback(A.desc, (int)bi, T);
-      if (t == 0) S.prefix = p;
-    }
-    __syncthreads();
-    const int64_t O = S.prefix;
-    if (!direct) {
-      emit(S, nbins, T, O, A.col_c, A.wgt_c);
-    } else if (d.kind == B_BUCKET) {
-      const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
-      const int64_t f0 = A.fb_off[bk];
-      for (int q = t; q < T; q += kT) {
-        A.col_c[O + q] = A.fb_b[f0 + q];
-        A.wgt_c[O + q] = A.fb_w[f0 + q];
-      }
-    } else {
-      for (int q = t; q < T; q += kT) {
-        A.col_c[O + q] = S.pb[q];
-        A.wgt_c[O + q] = S.pw[q];
-      }
-    }
-    if (d.kind == B_SMALL) {
-      for (int r = t; r < R; r += kT) {
-        A.row_ptr_c[S.row_id[r]] = O + S.ucnt[S.bbase[r]];
-        write_vwgt(A, S.row_id[r]);
-      }
-    } else if (d.sub == 0 && t == 0) {
-      A.row_ptr_c[d.row0] = O;
-      write_vwgt(A, d.row0);
-    }
-    if (bi == A.nblocks - 1 && t == 0) A.row_ptr_c[L.n_c] = O + T;
-    __syncthreads();
-  }
 }
 
 // ------------------------------------------------------- a9 BUCKET partition
@@ -1063,9 +598,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   ctx->stats.huge_rows = nbig;
   ctx->stats.dense_rows = dense ? nbig : 0;
 
-  // ---- second arena: block list, look-back descriptors, skew-path buffers
+  // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
-    size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + ws_bytes(nblocks + 1, 8);
+    size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 2 * ws_bytes(nblocks + 1, 4) +
+                ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
+                2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
     if (nbig > 0 && dense) b2 += ws_bytes((size_t)nbig * n_c, 8);
     if (nbig > 0 && !dense) {
       b2 += 2 * ws_bytes(nbkt + 1, 4) + 2 * ws_bytes(nbkt + 1, 8) + ws_bytes(nbkt + 1, 4);
@@ -1077,8 +614,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
   Arena &W2 = ctx->ws2;
   BlockDesc *blk = arena_take<BlockDesc>(W2, nblocks + 1);
-  uint64_t *desc = arena_take<uint64_t>(W2, nblocks + 1);
-  HEC_CUDA_TRY(cudaMemsetAsync(desc, 0, sizeof(uint64_t) * (nblocks + 1), s));
+  int32_t *blk_cnt = arena_take<int32_t>(W2, nblocks + 1);
+  int32_t *need_wide = arena_take<int32_t>(W2, nblocks + 1);
+  int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
+  ScanTiles st_blk = take_scan_tiles(W2, nblocks);
+  // SMALL staging is indexed by member-edge position (the space of all rows)
+  int32_t *sc_col = arena_take<int32_t>(W2, (size_t)(small_vol + big_vol) + 1);
+  int32_t *sc_wgt = arena_take<int32_t>(W2, (size_t)(small_vol + big_vol) + 1);
+  if (!sc_wgt) { set_error("workspace under-reserved (blocks)"); return HEC_EINVAL; }
+  HEC_CUDA_TRY(cudaMemsetAsync(need_wide, 0, sizeof(int32_t) * (nblocks + 1), s));
   k_block_desc<<<nblk(n_c, 256), 256, 0, s>>>(L, blk_ptr, big_idx, dense, blk);
   HEC_LAUNCH_CHECK();
   k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, n_c, blk);
@@ -1089,7 +633,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   A.blk = blk;
   A.nblocks = nblocks;
   A.ticket = counts + 1;
-  A.desc = desc;
+  A.blk_cnt = blk_cnt;
+  A.need_wide = need_wide;
+  A.blk_off = blk_off;
+  A.sc_col = sc_col;
+  A.sc_wgt = sc_wgt;
   A.vw64 = vw64;
   A.big_idx = big_idx;
   A.bkt_ptr = bkt_ptr;
@@ -1097,7 +645,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
 
   static bool attr = false;
   if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_rows, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(RowsSmem)));
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(PartSmem)));
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1162,34 +709,58 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
   phase_end(ctx, ph_skew);
 
-  // ---- outputs: nnz_c is known only after the ordered pass; allocate the upper
-  // bound sum(U) <= nnz (the tail beyond nnz_c is never read).
-  const int64_t cap_out = small_vol + big_vol;
+  // ---- work blocks (a8/a9 output), then placement (a10)
   HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_c + 1)));
-  HEC_TRY(dev_alloc(ctx, (void **)&out->col, sizeof(int32_t) * (cap_out > 0 ? cap_out : 1)));
-  HEC_TRY(dev_alloc(ctx, (void **)&out->wgt, sizeof(int32_t) * (cap_out > 0 ? cap_out : 1)));
   HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * n_c));
   A.row_ptr_c = out->row_ptr;
-  A.col_c = out->col;
-  A.wgt_c = out->wgt;
   A.vwgt_c = out->vwgt;
-  const int ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
-  {
-    int grid = ctx->num_sms * 2;
-    if (nblocks < grid) grid = (int)(nblocks > 0 ? nblocks : 1);
-    k_rows<<<grid, kT, sizeof(RowsSmem), s>>>(A);
-    HEC_LAUNCH_CHECK();
+  long long *trace = nullptr;
+  if (getenv("HEC_TRACE_ROWS")) {
+    HEC_TRY(dev_alloc(ctx, (void **)&trace, sizeof(long long) * 4 * (nblocks + 1)));
+    A.trace = trace;
   }
+  const int ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
+  HEC_TRY(launch_rows(ctx, A, false));
   phase_end(ctx, ph_rows);
-  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 12, out->row_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+  if (trace) {
+    std::vector<long long> h(4 * nblocks);
+    HEC_CUDA_TRY(cudaMemcpyAsync(h.data(), trace, sizeof(long long) * 4 * nblocks, cudaMemcpyDeviceToHost, s));
+    HEC_CUDA_TRY(cudaStreamSynchronize(s));
+    char fn[256];
+    snprintf(fn, sizeof fn, "%s_%lld.bin", getenv("HEC_TRACE_ROWS"), (long long)n_c);
+    FILE *f = fopen(fn, "wb");
+    if (f) { fwrite(h.data(), sizeof(long long), h.size(), f); fclose(f); }
+    dev_free(ctx, trace);
+  }
+  HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks));
+  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 12, blk_off + nblocks, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
   int64_t r2[13];
   HEC_TRY(read_scalars(ctx, scal, 13, r2));
+  if ((int)(r2[0] & 0xffffffff) & ERR_WIDE) {
+    // some block's total weight exceeds int32: those blocks (flagged, inputs left
+    // untouched) are redone with int64 sums
+    HEC_CUDA_TRY(cudaMemsetAsync(counts + 1, 0, sizeof(unsigned), s));
+    HEC_CUDA_TRY(cudaMemsetAsync(err, 0, sizeof(int), s));
+    HEC_TRY(launch_rows(ctx, A, true));
+    HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks));
+    HEC_CUDA_TRY(cudaMemcpyAsync(scal + 12, blk_off + nblocks, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+    HEC_TRY(read_scalars(ctx, scal, 13, r2));
+  }
   out->nnz_c = r2[12];
-  phase_set_bytes(ctx, ph_rows, 8.0 * (double)small_vol + 8.0 * (double)out->nnz_c + 12.0 * dnc);
-  if ((int)(r2[0] & 0xffffffff) & 2) {
+  if ((int)(r2[0] & 0xffffffff) & ERR_OVERFLOW) {
     set_error("build_coarse_graph: a coarse weight exceeds INT32_MAX");
     return HEC_EOVERFLOW;
   }
+  const int64_t nnz_c = out->nnz_c;
+  HEC_TRY(dev_alloc(ctx, (void **)&out->col, sizeof(int32_t) * (nnz_c > 0 ? nnz_c : 1)));
+  HEC_TRY(dev_alloc(ctx, (void **)&out->wgt, sizeof(int32_t) * (nnz_c > 0 ? nnz_c : 1)));
+  A.col_c = out->col;
+  A.wgt_c = out->wgt;
+  const int ph_place = phase_begin(ctx, "place", 16.0 * (double)nnz_c + 16.0 * dnc);
+  HEC_TRY(launch_place(ctx, A));
+  phase_end(ctx, ph_place);
+  phase_set_bytes(ctx, ph_rows, 8.0 * (double)small_vol + 12.0 * dnc);
+  if (nblocks == 0) HEC_CUDA_TRY(cudaMemsetAsync(out->row_ptr, 0, sizeof(int64_t) * (n_c + 1), s));
   ctx->stats.nnz_c = out->nnz_c;
   return HEC_OK;
 }

@@ -1,0 +1,227 @@
+// construct_common.cuh — shared pieces of CONSTRUCTCOARSEGRAPH (construct*.cu):
+// sizes, the member-edge layout, shared-memory member tables and the
+// edge-balanced expansion of fine entries into (b = M[v], w) register tuples.
+#pragma once
+#include "hec_internal.cuh"
+
+namespace hec {
+
+constexpr int kT = 512;            // threads per CTA of the row kernels
+constexpr int kIt = 8;             // entries held per thread (registers)
+constexpr int kCap = kT * kIt;     // entries per work block (4096)
+constexpr int kHash = kCap + kCap / 2 + 8;  // hash slots per work block (regions of 1.5 U + 1)
+constexpr int kWin = 2048;         // window weight; a block's weight is < 2*kWin
+constexpr int kRowW = 8;           // per-row weight: bounds rows per block
+constexpr int kMaxRows = 2 * kWin / kRowW;  // 512
+constexpr int kSmallMax = kWin - kRowW;     // rows with U <= 2040 are small
+constexpr int kMC = 1024;          // member-table chunk
+constexpr int kBucketAvg = 1024;   // target entries per BUCKET
+constexpr int kDenseMax = 32768;   // n_c bound of the DENSE skew path
+constexpr int32_t kEmpty = -1;
+
+enum : int32_t { B_SMALL = 0, B_BUCKET = 1, B_DENSE = 2 };
+enum : int { ERR_LABEL = 1, ERR_OVERFLOW = 2, ERR_WIDE = 4 };
+
+inline unsigned nblk(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
+
+// largest i in [lo, hi) with a[i] <= x (a non-decreasing, a[lo] <= x)
+template <typename T>
+__device__ __forceinline__ int64_t last_le(const T *a, int64_t lo, int64_t hi, int64_t x) {
+  hi -= 1;
+  while (lo < hi) {
+    int64_t mid = (lo + hi + 1) >> 1;
+    if ((int64_t)a[mid] <= x) lo = mid;
+    else hi = mid - 1;
+  }
+  return lo;
+}
+
+// In-place exclusive scan of n <= kCap+1 int32 values in shared memory by a CTA
+// of kT threads; returns the total.  `tmp` holds >= 33 ints.
+__device__ __forceinline__ int smem_exclusive_scan(int32_t *a, int n, int32_t *tmp) {
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  const int chunk = (n + kT - 1) / kT;
+  const int beg = t * chunk;
+  int local = 0;
+  for (int i = 0; i < chunk && beg + i < n; ++i) local += a[beg + i];
+  int x = local;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) tmp[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    int w = lane < kT / 32 ? tmp[lane] : 0;
+    int ws = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int y = __shfl_up_sync(0xffffffffu, ws, o);
+      if (lane >= o) ws += y;
+    }
+    if (lane < kT / 32) tmp[lane] = ws - w;
+    if (lane == kT / 32 - 1) tmp[32] = ws;
+  }
+  __syncthreads();
+  int run = tmp[wid] + x - local;
+  for (int i = 0; i < chunk && beg + i < n; ++i) {
+    int v = a[beg + i];
+    a[beg + i] = run;
+    run += v;
+  }
+  int total = tmp[32];
+  __syncthreads();
+  return total;
+}
+
+// CTA-wide sum of a 64-bit value; `tmp` holds >= kT/32 long longs.
+__device__ __forceinline__ long long block_sum64(long long v, long long *tmp) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  if (lane == 0) tmp[wid] = v;
+  __syncthreads();
+  long long s = 0;
+  for (int w = 0; w < kT / 32; ++w) s += tmp[w];
+  __syncthreads();
+  return s;
+}
+
+struct Layout {
+  int64_t n_c;
+  const int64_t *member_ptr;  // [n_c+1]
+  const int32_t *members;     // [n]
+  const int64_t *mpre;        // [n+1] member-edge prefix
+  const int64_t *row_ptr;
+  const int32_t *col;
+  const int32_t *wgt;
+  const int32_t *M;
+  __device__ __forceinline__ int64_t upos(int64_t a) const { return mpre[member_ptr[a]]; }
+  __device__ __forceinline__ int64_t U(int64_t a) const { return upos(a + 1) - upos(a); }
+};
+
+struct MemberTab {
+  int64_t mstart[kMC];    // row_ptr[u] of the member
+  int32_t moff[kMC + 1];  // member's first position relative to the window start
+  int32_t mrow[kMC];      // local row of the member
+};
+
+// Expand the member-edge window [P0, P0+nP) (nP <= kCap), whose members are
+// [m0, m1), into registers: slot s = tid + kT*k holds (b = M[v], w, local row).
+// Slots without an entry keep kb = -1.  s_mptr[0..R]: member_ptr slice of the
+// rows (nullptr => one row, index 0).
+__device__ __forceinline__ void expand_window(const Layout &L, MemberTab &T, int64_t P0, int nP, int64_t m0,
+                                              int64_t m1, const int64_t *s_mptr, int R, int32_t (&kb)[kIt],
+                                              int32_t (&kw)[kIt], int32_t (&kr)[kIt]) {
+  const int t = threadIdx.x;
+#pragma unroll
+  for (int k = 0; k < kIt; ++k) { kb[k] = -1; kw[k] = 0; kr[k] = 0; }
+  for (int64_t cm = m0; cm < m1; cm += kMC) {
+    const int nm = (int)((m1 - cm) < kMC ? (m1 - cm) : kMC);
+    for (int i = t; i < nm; i += kT) {
+      int32_t u = L.members[cm + i];
+      T.mstart[i] = L.row_ptr[u];
+      T.moff[i] = (int32_t)(L.mpre[cm + i] - P0);
+      T.mrow[i] = s_mptr ? (int32_t)last_le(s_mptr, 0, R, cm + i) : 0;
+    }
+    if (t == 0) {
+      int64_t e = L.mpre[cm + nm] - P0;
+      T.moff[nm] = (int32_t)(e > (int64_t)kCap + 1 ? kCap + 1 : e);
+    }
+    __syncthreads();
+    const int lo = T.moff[0] > 0 ? T.moff[0] : 0;
+    const int hi = T.moff[nm] < nP ? T.moff[nm] : nP;
+    unsigned fresh = 0;
+    int64_t ev[kIt];
+#pragma unroll
+    for (int k = 0; k < kIt; ++k) {
+      const int s = t + kT * k;
+      ev[k] = 0;
+      if (s >= lo && s < hi) {
+        int i = (int)last_le(T.moff, 0, nm, s);
+        ev[k] = T.mstart[i] + (s - T.moff[i]);
+        kr[k] = T.mrow[i];
+        fresh |= 1u << k;
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < kIt; ++k)
+      if (fresh & (1u << k)) { kb[k] = __ldg(L.col + ev[k]); kw[k] = __ldg(L.wgt + ev[k]); }
+#pragma unroll
+    for (int k = 0; k < kIt; ++k)
+      if (fresh & (1u << k)) kb[k] = __ldg(L.M + kb[k]);
+    __syncthreads();
+  }
+}
+
+// Members of big row a covering the window [P0, P0+nP): [m0, m1).
+__device__ __forceinline__ void window_members(const Layout &L, int32_t a, int64_t P0, int nP, int64_t *m0,
+                                               int64_t *m1) {
+  const int64_t m0r = L.member_ptr[a], m1r = L.member_ptr[a + 1];
+  *m0 = last_le(L.mpre, m0r, m1r, P0);
+  int64_t lo = *m0, hi = m1r - 1;  // last member i with mpre[i] < P0 + nP
+  while (lo < hi) {
+    int64_t mid = (lo + hi + 1) >> 1;
+    if (L.mpre[mid] < P0 + nP) lo = mid;
+    else hi = mid - 1;
+  }
+  *m1 = lo + 1;
+}
+
+struct BlockDesc {
+  int32_t kind;
+  int32_t row0;  // first row (SMALL) / the row (BUCKET, DENSE)
+  int32_t row1;  // one past the last row (SMALL)
+  int32_t sub;   // bucket index within the row / dense key chunk
+};
+
+// Arguments of the work-block kernels (construct_rows.cu).  Each block leaves
+// its sorted distinct (b, w) in a staging place that depends on its kind:
+//   SMALL   sc_col/sc_wgt at the block's first member-edge position
+//   BUCKET  in place over its partitioned pairs pb_g/pw_g
+//   DENSE   interleaved (b, w) int32 pairs over its chunk of the dense row
+//   fallback buckets: fb_b/fb_w (written by k_bucket_fallback)
+// and its count in blk_cnt; row_ptr_c holds row offsets relative to the block.
+// An exclusive scan of blk_cnt then gives every block's output offset and
+// k_place copies the staged entries into the final CSR (coalesced).
+struct RowsArgs {
+  Layout L;
+  const BlockDesc *blk;
+  int64_t nblocks;
+  unsigned *ticket;
+  int32_t *blk_cnt;                 // [nblocks] distinct entries per block
+  int32_t *need_wide;               // [nblocks] 1: redo with 64-bit sums (zeroed)
+  const int64_t *blk_off;           // [nblocks+1] exclusive scan of blk_cnt (k_place)
+  const unsigned long long *vw64;
+  const int32_t *big_idx;
+  int32_t *sc_col, *sc_wgt;         // SMALL staging, member-edge space [nnz]
+  // BUCKET mode
+  const int64_t *bkt_ptr;           // [nbig+1] first bucket of big row h
+  const int64_t *bkt_off;           // [nbkt+1] pair offsets
+  int32_t *pb_g, *pw_g;             // partitioned pairs (sorted uniques written back in place)
+  const int32_t *fb_cnt;            // fallback unique count per bucket (-1: not overflowed)
+  const int64_t *fb_off;            // fallback scratch offset per bucket
+  const int32_t *fb_b, *fb_w;
+  // DENSE mode
+  unsigned long long *dense;        // [nbig][n_c] sums, then staged pairs
+  // outputs
+  int64_t *row_ptr_c;
+  int32_t *col_c, *wgt_c, *vwgt_c;
+  int *err;
+  long long *trace;  // debug: per block (compute cycles, 0, kind, T); nullable
+};
+
+// keys b with floor(b * nb / n_c) == k: [ceil(k n_c / nb), ceil((k+1) n_c / nb))
+__host__ __device__ __forceinline__ void bucket_range(int64_t k, int64_t nb, int64_t n_c, int32_t *lo,
+                                                      int32_t *hi) {
+  *lo = (int32_t)((k * n_c + nb - 1) / nb);
+  int64_t h = ((k + 1) * n_c + nb - 1) / nb;
+  *hi = (int32_t)(h < n_c ? h : n_c);
+}
+
+// Work-block kernel and placement launchers (construct_rows.cu).
+int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide);
+int launch_place(hec_ctx *ctx, const RowsArgs &A);
+
+}  // namespace hec

@@ -1,0 +1,417 @@
+// construct_rows.cu — the ordered work-block kernel of CONSTRUCTCOARSEGRAPH
+// (SURVEY §8 rows a8, a9 output, a10).
+//
+// Persistent CTAs take work blocks through a ticket (dynamic balancing):
+//  1. entries (b = M[v], w) of the block's rows arrive in registers (expansion of
+//     the member rows, or a partitioned bucket of a skewed row);
+//  2. per-row shared-memory hash tables (regions of 1.5*U slots) merge duplicate
+//     keys — DEDUPWITHWTS's hash variant.  The thread whose CAS
+//     created a key owns it from then on;
+//  3. owned keys are bucket-sorted per row in shared memory (one bucket per
+//     distinct key of the row on average, bucket = scaled key within the row's
+//     key range, rank from one smem atomic, insertion sort inside buckets);
+//  4. the sorted distinct entries are staged (see RowsArgs), the block's count
+//     goes to blk_cnt; after an exclusive scan of the counts, k_place copies
+//     every block to its final CSR position (no CTA ever waits for another).
+// Sums are exact: int32 accumulators are used only when the block's total
+// weight fits in int32; otherwise the block is flagged and the host reruns the
+// flagged blocks with the 64-bit (WIDE) instantiation.
+#include <type_traits>
+
+#include "construct_common.cuh"
+
+namespace hec {
+
+template <bool WIDE>
+struct RowsSmemT {
+  // phase-aliased areas: [expansion: member table] -> [hash keys] -> [bucket histogram]
+  union {
+    MemberTab T;
+    int32_t hkey[kHash];
+    int32_t hist[kCap + 1];
+  } a;
+  // [hash values] -> [sorted pairs]
+  union {
+    typename std::conditional<WIDE, unsigned long long, unsigned>::type hval[kHash];
+    struct {
+      int32_t pb[kCap];
+      int32_t pw[kCap];
+    } p;
+  } v;
+  int64_t mptr[kMaxRows + 1];
+  int32_t kmin[kMaxRows];
+  int32_t kmax[kMaxRows];
+  int32_t hbase[kMaxRows + 1];  // hash region offsets
+  int32_t ucnt[kMaxRows + 1];   // distinct keys per row -> exclusive offsets
+  float bscale[kMaxRows];
+  int32_t tmp[40];
+  unsigned long long wtot;
+  long long tx[2];  // trace: expansion / hashing cycles
+  int32_t blk;
+};
+
+__device__ __forceinline__ int warp_min(int v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ int warp_max(int v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = max(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+// min/max of key over lanes with row r >= 0; one atomic per warp when uniform.
+__device__ __forceinline__ void range_update(int32_t *kmin, int32_t *kmax, int r, int32_t key) {
+  const int r0 = __shfl_sync(0xffffffffu, r, 0);
+  if (__all_sync(0xffffffffu, r == r0)) {
+    if (r0 >= 0) {
+      int mn = warp_min(key), mx = warp_max(key);
+      if ((threadIdx.x & 31) == 0) { atomicMin(kmin + r0, mn); atomicMax(kmax + r0, mx); }
+    }
+  } else if (r >= 0) {
+    atomicMin(kmin + r, key);
+    atomicMax(kmax + r, key);
+  }
+}
+
+// count of lanes with `flag` per row r; one atomic per warp when uniform.
+__device__ __forceinline__ void count_update(int32_t *cnt, int r, bool flag) {
+  const unsigned m = __ballot_sync(0xffffffffu, flag);
+  if (!m) return;
+  const int leader = __ffs(m) - 1;
+  const int r0 = __shfl_sync(0xffffffffu, r, leader);
+  if (__all_sync(0xffffffffu, !flag || r == r0)) {
+    if ((int)(threadIdx.x & 31) == leader) atomicAdd(cnt + r0, __popc(m));
+  } else if (flag) {
+    atomicAdd(cnt + r, 1);
+  }
+}
+
+template <bool WIDE>
+__global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
+  using V = typename std::conditional<WIDE, unsigned long long, unsigned>::type;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  RowsSmemT<WIDE> &S = *reinterpret_cast<RowsSmemT<WIDE> *>(smem_raw);
+  int32_t *pb = S.v.p.pb;
+  int32_t *pw = S.v.p.pw;
+  const int t = threadIdx.x;
+  const Layout &L = A.L;
+  while (true) {
+    if (t == 0) S.blk = (int32_t)atomicAdd(A.ticket, 1u);
+    __syncthreads();
+    const int64_t bi = S.blk;
+    if (bi >= A.nblocks) return;
+    if (WIDE && !A.need_wide[bi]) {  // the 64-bit pass redoes only flagged blocks
+      __syncthreads();
+      continue;
+    }
+    const BlockDesc d = A.blk[bi];
+    const long long c0 = A.trace ? clock64() : 0;
+    int T = 0, R = 1;
+    bool from_fallback = false;
+    int64_t fb0 = 0;
+    if (d.kind == B_DENSE) {
+      // key chunk [k0, k0 + kCap) of a dense row, already in key order
+      const int32_t h = A.big_idx[d.row0];
+      const int64_t k0 = (int64_t)d.sub * kCap;
+      const unsigned long long *row = A.dense + (int64_t)h * L.n_c;
+      unsigned long long v[kIt];
+      int c = 0;
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) {  // blocked: thread t owns keys k0 + t*kIt + k
+        const int64_t key = k0 + (int64_t)t * kIt + k;
+        v[k] = key < L.n_c ? row[key] : 0ull;
+        c += v[k] != 0;
+      }
+      S.a.hist[t] = c;
+      __syncthreads();
+      T = smem_exclusive_scan(S.a.hist, kT, S.tmp);
+      int pos = S.a.hist[t];
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) {
+        if (v[k] != 0) {
+          if (v[k] > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
+          pb[pos] = (int32_t)(k0 + (int64_t)t * kIt + k);
+          pw[pos] = (int32_t)v[k];
+          ++pos;
+        }
+      }
+    } else if (d.kind == B_BUCKET && A.fb_cnt[A.bkt_ptr[A.big_idx[d.row0]] + d.sub] >= 0) {
+      const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
+      T = A.fb_cnt[bk];
+      fb0 = A.fb_off[bk];
+      from_fallback = true;
+    } else {
+      // ---- 1. entries into registers
+      int32_t kb[kIt], kw[kIt], kr[kIt];
+      if (d.kind == B_SMALL) {
+        R = d.row1 - d.row0;
+        for (int r = t; r <= R; r += kT) S.mptr[r] = L.member_ptr[d.row0 + r];
+        if (t == 0) S.wtot = 0;
+        __syncthreads();
+        for (int r = t; r < R; r += kT) {
+          S.kmin[r] = INT32_MAX;
+          S.kmax[r] = -1;
+          S.ucnt[r] = 0;
+          const int32_t U = (int32_t)(L.mpre[S.mptr[r + 1]] - L.mpre[S.mptr[r]]);
+          S.hbase[r] = U + (U >> 1) + 1;
+        }
+        const int64_t m0 = S.mptr[0], m1 = S.mptr[R];
+        const int64_t P0 = L.mpre[m0];
+        const int nP = (int)(L.mpre[m1] - P0);
+        expand_window(L, S.a.T, P0, nP, m0, m1, S.mptr, R, kb, kw, kr);  // ends with a barrier
+#pragma unroll
+        for (int k = 0; k < kIt; ++k)
+          if (kb[k] >= 0 && kb[k] == d.row0 + kr[k]) kb[k] = -1;  // self entries are dropped (L280)
+      } else {  // B_BUCKET: partitioned pairs of one skewed row (self entries already dropped)
+        const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
+        const int64_t q0 = A.bkt_off[bk], cnt = A.bkt_off[bk + 1] - q0;
+#pragma unroll
+        for (int k = 0; k < kIt; ++k) {
+          const int s = t + kT * k;
+          kb[k] = -1;
+          kw[k] = 0;
+          kr[k] = 0;
+          if (s < cnt) { kb[k] = A.pb_g[q0 + s]; kw[k] = A.pw_g[q0 + s]; }
+        }
+        if (t == 0) {
+          S.kmin[0] = INT32_MAX;
+          S.kmax[0] = -1;
+          S.ucnt[0] = 0;
+          S.hbase[0] = (int32_t)(cnt + (cnt >> 1) + 1);
+          S.wtot = 0;
+        }
+        __syncthreads();
+      }
+      // ---- 2. per-row hash regions; the creating thread owns each key
+      const int Hs = smem_exclusive_scan(S.hbase, R, S.tmp);
+      if (t == 0) S.hbase[R] = Hs;
+      for (int i = t; i < Hs; i += kT) { S.a.hkey[i] = kEmpty; S.v.hval[i] = 0; }
+      {
+        long long ws = 0;
+#pragma unroll
+        for (int k = 0; k < kIt; ++k) ws += kb[k] >= 0 ? kw[k] : 0;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(0xffffffffu, ws, o);
+        if ((t & 31) == 0 && ws) atomicAdd(&S.wtot, (unsigned long long)ws);
+      }
+      __syncthreads();
+      if (!WIDE && S.wtot > 0x7fffffffull) {
+        // a merged weight could exceed int32: leave the inputs untouched and let
+        // the 64-bit pass redo this block
+        if (t == 0) {
+          A.need_wide[bi] = 1;
+          atomicOr(A.err, ERR_WIDE);
+        }
+        __syncthreads();
+        continue;
+      }
+      const long long c_exp = A.trace ? clock64() : 0;
+      int32_t ks[kIt];  // owned slot or -1
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) {
+        bool fresh = false;
+        ks[k] = -1;
+        const int r = kr[k];
+        if (kb[k] >= 0) {
+          const int32_t b = kb[k];
+          const int hb = S.hbase[r], hs = S.hbase[r + 1] - hb;
+          int s = hb + (int)(((uint64_t)((uint32_t)b * 0x9E3779B1u) * (uint32_t)hs) >> 32);
+          while (true) {
+            int32_t cur = ((volatile int32_t *)S.a.hkey)[s];
+            if (cur == b) break;
+            if (cur == kEmpty) {
+              int32_t old = atomicCAS(S.a.hkey + s, kEmpty, b);
+              if (old == kEmpty) { fresh = true; break; }
+              if (old == b) break;
+            }
+            if (++s == hb + hs) s = hb;
+          }
+          atomicAdd(S.v.hval + s, (V)kw[k]);
+          if (fresh) ks[k] = s;
+        }
+        count_update(S.ucnt, r, fresh);
+        if (!fresh) kb[k] = -1;  // not an owner
+      }
+      __syncthreads();
+      T = smem_exclusive_scan(S.ucnt, R, S.tmp);
+      if (A.trace && t == 0) { S.tx[0] = c_exp - c0; S.tx[1] = clock64() - c_exp; }
+      if (t == 0) S.ucnt[R] = T;
+      // ---- 3. owned keys: key range per row, buckets, ranks
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) range_update(S.kmin, S.kmax, kb[k] >= 0 ? kr[k] : -1, kb[k]);
+      __syncthreads();
+      for (int r = t; r < R; r += kT) {
+        const int lo = S.kmin[r], hi = S.kmax[r];
+        const int cnt = S.ucnt[r + 1] - S.ucnt[r];
+        S.bscale[r] = hi >= lo ? (float)cnt / (float)((int64_t)hi - lo + 1) : 0.f;
+      }
+      for (int i = t; i <= T; i += kT) S.a.hist[i] = 0;  // hash keys are dead
+      __syncthreads();
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) {
+        if (kb[k] >= 0) {
+          const int r = kr[k];
+          const int nb = S.ucnt[r + 1] - S.ucnt[r];  // one bucket per distinct key
+          int off = (int)((float)(kb[k] - S.kmin[r]) * S.bscale[r]);
+          off = off < nb - 1 ? off : nb - 1;
+          const int bin = S.ucnt[r] + off;
+          kr[k] = (bin << 12) | atomicAdd(&S.a.hist[bin], 1);
+          const V wv = S.v.hval[ks[k]];
+          if (WIDE && (unsigned long long)wv > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
+          kw[k] = (int32_t)wv;  // final sum, read before the pairs overwrite the values
+        }
+      }
+      __syncthreads();
+      smem_exclusive_scan(S.a.hist, T + 1, S.tmp);
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) {
+        if (kb[k] >= 0) {
+          const int q = S.a.hist[kr[k] >> 12] + (kr[k] & 4095);
+          pb[q] = kb[k];
+          pw[q] = kw[k];
+        }
+      }
+      __syncthreads();
+      // insertion sort inside each bucket (distinct keys, ~1 per bucket)
+      for (int bin = t; bin < T; bin += kT) {
+        const int lo = S.a.hist[bin], hi = S.a.hist[bin + 1];
+        for (int i = lo + 1; i < hi; ++i) {
+          const int32_t kk = pb[i], ww = pw[i];
+          int j = i - 1;
+          while (j >= lo && pb[j] > kk) {
+            pb[j + 1] = pb[j];
+            pw[j + 1] = pw[j];
+            --j;
+          }
+          pb[j + 1] = kk;
+          pw[j + 1] = ww;
+        }
+      }
+    }
+    __syncthreads();
+    // ---- 4. stage the block's sorted distinct entries; k_place moves them
+    const long long c1 = A.trace ? clock64() : 0;
+    if (d.kind == B_SMALL) {
+      const int64_t P0 = L.mpre[S.mptr[0]];
+      for (int q = t; q < T; q += kT) {
+        A.sc_col[P0 + q] = pb[q];
+        A.sc_wgt[P0 + q] = pw[q];
+      }
+      for (int r = t; r < R; r += kT) {
+        const int32_t a = d.row0 + r;
+        A.row_ptr_c[a] = S.ucnt[r];  // relative to the block's output offset
+        const unsigned long long s = A.vw64[a];
+        if (s > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
+        A.vwgt_c[a] = (int32_t)s;
+      }
+    } else {
+      if (d.kind == B_BUCKET && !from_fallback) {
+        const int64_t q0 = A.bkt_off[A.bkt_ptr[A.big_idx[d.row0]] + d.sub];
+        for (int q = t; q < T; q += kT) {  // in place over the bucket's own pairs
+          A.pb_g[q0 + q] = pb[q];
+          A.pw_g[q0 + q] = pw[q];
+        }
+      } else if (d.kind == B_DENSE) {
+        int32_t *st = reinterpret_cast<int32_t *>(A.dense + (int64_t)A.big_idx[d.row0] * L.n_c +
+                                                  (int64_t)d.sub * kCap);
+        for (int q = t; q < T; q += kT) {
+          st[2 * q] = pb[q];
+          st[2 * q + 1] = pw[q];
+        }
+      }
+      if (d.sub == 0 && t == 0) {
+        const unsigned long long s = A.vw64[d.row0];
+        if (s > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
+        A.vwgt_c[d.row0] = (int32_t)s;
+      }
+    }
+    if (t == 0) {
+      A.blk_cnt[bi] = T;
+      if (A.trace) {
+        A.trace[4 * bi] = c1 - c0;
+        // expansion cycles << 32 | hashing cycles (0 for DENSE / fallback blocks)
+        A.trace[4 * bi + 1] = (d.kind == B_DENSE || from_fallback) ? 0 : (S.tx[0] << 32) | (S.tx[1] & 0xffffffff);
+        A.trace[4 * bi + 2] = d.kind * 100000 + (d.kind == B_SMALL ? R : d.sub);
+        A.trace[4 * bi + 3] = T;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// One CTA per work block: copy its staged entries to the final CSR position.
+constexpr int kPlaceT = 256;
+__global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
+  const int64_t bi = blockIdx.x;
+  const BlockDesc d = A.blk[bi];
+  const Layout &L = A.L;
+  const int64_t O = A.blk_off[bi];
+  const int T = A.blk_cnt[bi];
+  const int t = threadIdx.x;
+  if (d.kind == B_SMALL) {
+    const int64_t P0 = L.mpre[L.member_ptr[d.row0]];
+    for (int q = t; q < T; q += kPlaceT) {
+      A.col_c[O + q] = A.sc_col[P0 + q];
+      A.wgt_c[O + q] = A.sc_wgt[P0 + q];
+    }
+    for (int a = d.row0 + t; a < d.row1; a += kPlaceT) A.row_ptr_c[a] += O;
+  } else {
+    const int64_t bk = d.kind == B_BUCKET ? A.bkt_ptr[A.big_idx[d.row0]] + d.sub : 0;
+    if (d.kind == B_DENSE) {
+      const int32_t *st = reinterpret_cast<const int32_t *>(A.dense + (int64_t)A.big_idx[d.row0] * L.n_c +
+                                                            (int64_t)d.sub * kCap);
+      for (int q = t; q < T; q += kPlaceT) {
+        A.col_c[O + q] = st[2 * q];
+        A.wgt_c[O + q] = st[2 * q + 1];
+      }
+    } else if (A.fb_cnt[bk] >= 0) {
+      const int64_t f0 = A.fb_off[bk];
+      for (int q = t; q < T; q += kPlaceT) {
+        A.col_c[O + q] = A.fb_b[f0 + q];
+        A.wgt_c[O + q] = A.fb_w[f0 + q];
+      }
+    } else {
+      const int64_t q0 = A.bkt_off[bk];
+      for (int q = t; q < T; q += kPlaceT) {
+        A.col_c[O + q] = A.pb_g[q0 + q];
+        A.wgt_c[O + q] = A.pw_g[q0 + q];
+      }
+    }
+    if (d.sub == 0 && t == 0) A.row_ptr_c[d.row0] = O;
+  }
+  if (bi == A.nblocks - 1 && t == 0) A.row_ptr_c[L.n_c] = O + T;
+}
+
+int launch_place(hec_ctx *ctx, const RowsArgs &A) {
+  if (A.nblocks <= 0) return HEC_OK;
+  k_place<<<(unsigned)A.nblocks, kPlaceT, 0, ctx->stream>>>(A);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
+int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide) {
+  static int occ[2] = {0, 0};
+  if (!occ[0]) {
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_rows<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)sizeof(RowsSmemT<false>)));
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_rows<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)sizeof(RowsSmemT<true>)));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_rows<false>, kT,
+                                                               sizeof(RowsSmemT<false>)));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_rows<true>, kT,
+                                                               sizeof(RowsSmemT<true>)));
+    if (occ[0] < 1) occ[0] = 1;
+    if (occ[1] < 1) occ[1] = 1;
+  }
+  // persistent: every CTA holding a ticket must be resident (look-back progress)
+  int64_t grid = (int64_t)ctx->num_sms * occ[wide ? 1 : 0];
+  if (A.nblocks < grid) grid = A.nblocks > 0 ? A.nblocks : 1;
+  if (wide) k_rows<true><<<(unsigned)grid, kT, sizeof(RowsSmemT<true>), ctx->stream>>>(A);
+  else k_rows<false><<<(unsigned)grid, kT, sizeof(RowsSmemT<false>), ctx->stream>>>(A);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
+}  // namespace hec

@@ -218,35 +218,68 @@ __device__ __forceinline__ int64_t block_exclusive_sum(int64_t v, int64_t *total
   return r;
 }
 
-// Warp 0 resolves the exclusive prefix of `tile` given its aggregate.
-__device__ __forceinline__ int64_t lookback(uint64_t *desc, int tile, int64_t agg) {
+// Publish the aggregate of `tile` (tile 0 publishes its inclusive prefix).
+__device__ __forceinline__ void lookback_publish(uint64_t *desc, int tile, int64_t agg) {
+  st_release(desc + tile, (tile == 0 ? kFlagP : kFlagA) | (uint64_t)agg);
+}
+
+// Warp 0 resolves the exclusive prefix of `tile` whose aggregate `agg` was
+// already published, then publishes the inclusive prefix.
+__device__ __forceinline__ int64_t lookback_resolve(uint64_t *desc, int tile, int64_t agg) {
   const int lane = threadIdx.x & 31;
-  if (tile == 0) {
-    if (lane == 0) st_release(desc, kFlagP | (uint64_t)agg);
-    return 0;
-  }
-  if (lane == 0) st_release(desc + tile, kFlagA | (uint64_t)agg);
+  if (tile == 0) return 0;
+  // Windows of 32 x kLB predecessors per round: with hundreds of blocks in
+  // flight the nearest inclusive prefix is typically ~that far back, so a wide
+  // window resolves in one or two L2 round trips.  Predecessor at distance
+  // lane + 32*i (i < kLB) is examined by `lane`.
+  constexpr int kLB = 8;
   int64_t prefix = 0;
   int base = tile - 1;
   while (true) {
-    int j = base - lane;
-    uint64_t d = 0;
-    if (j >= 0) {
-      do { d = ld_acquire(desc + j); } while ((d >> 62) == 0);
-    } else {
-      d = kFlagP;  // virtual inclusive prefix 0 before tile 0
+    uint64_t d[kLB];
+#pragma unroll
+    for (int i = 0; i < kLB; ++i) {
+      const int j = base - lane - 32 * i;
+      d[i] = j >= 0 ? ld_acquire(desc + j) : kFlagP;  // virtual prefix 0 before tile 0
     }
-    unsigned pmask = __ballot_sync(0xffffffffu, (d >> 62) == 2);
-    int first_p = pmask ? __ffs(pmask) - 1 : 32;  // nearest inclusive prefix
-    int64_t v = (lane <= first_p) ? (int64_t)(d & kValMask) : 0;
+#pragma unroll
+    for (int i = 0; i < kLB; ++i) {
+      const int j = base - lane - 32 * i;
+      // poll with backoff: hundreds of CTAs spinning on L2 would otherwise steal
+      // request bandwidth from the predecessors they wait for
+      unsigned ns = 32;
+      while ((d[i] >> 62) == 0) {
+        __nanosleep(ns);
+        ns = ns < 1024 ? ns * 2 : ns;
+        d[i] = ld_acquire(desc + j);
+      }
+    }
+    // nearest predecessor holding an inclusive prefix: smallest distance
+    int near = 32 * kLB;
+#pragma unroll
+    for (int i = kLB - 1; i >= 0; --i)
+      if ((d[i] >> 62) == 2) near = lane + 32 * i;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) near = min(near, __shfl_xor_sync(0xffffffffu, near, o));
+    int64_t v = 0;
+#pragma unroll
+    for (int i = 0; i < kLB; ++i)
+      if (lane + 32 * i <= near) v += (int64_t)(d[i] & kValMask);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
     prefix += v;
-    if (pmask) break;
-    base -= 32;
+    if (near < 32 * kLB) break;
+    base -= 32 * kLB;
   }
   if (lane == 0) st_release(desc + tile, kFlagP | (uint64_t)(prefix + agg));
   return prefix;
+}
+
+// Warp 0: publish the aggregate and resolve the exclusive prefix.
+__device__ __forceinline__ int64_t lookback(uint64_t *desc, int tile, int64_t agg) {
+  if ((threadIdx.x & 31) == 0) lookback_publish(desc, tile, agg);
+  __syncwarp();
+  return lookback_resolve(desc, tile, agg);
 }
 
 // Exclusive scan over i in [0, N): out(i, prefix_i) with in(i) >= 0.
