@@ -194,19 +194,43 @@ HEC_API int hec_debug_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H);
 HEC_API int hec_debug_roots(hec_ctx *ctx, const hec_graph *g, const uint64_t *prio,
                             uint64_t seed, int level, uint8_t *root, int *rounds);
 
-/* ------------------------------------------- multi-GPU construction (§8(e)) */
-/* Rows [a_begin, a_end) of G_c only (coarse-vertex range partition).  Writes
- * counts[a - a_begin] = |row a| (device int64[a_end-a_begin]); then, after the
- * caller has all-gathered the counts and passed the global exclusive offsets of
- * its rows (device int64 offs[a_end-a_begin+1], offs[0] = first entry index of
- * row a_begin), hec_build_rows_write fills col_c/wgt_c at those global
- * positions (device arrays of the full nnz_c, or of the slice when offs are
- * rebased by the caller) plus vwgt_c[a - a_begin].
- * The pair must be called with the same ctx, g, M, n_c, range and no other
- * libhec call in between on that ctx. */
+/* ------------------------------------------- multi-GPU building blocks (§8(e)) */
+/* The partitioned hierarchy level (one process per GPU; the collectives are the
+ * caller's, e.g. torch.distributed over NCCL):
+ *   1. hec_heavy_range on the rank's fine-vertex slice, all-gather H;
+ *   2. hec_mapping_from_heavy (rounds + relabel are replicated, cheap, vertex-
+ *      only), M written for the rank's slice, all-gather M;
+ *   3. hec_balance_rows: every rank derives the same coarse-row ranges;
+ *   4. hec_build_rows_count on the rank's coarse rows, all-gather the counts;
+ *   5. hec_build_rows_write at the slice's global entry offset.
+ * Every result is identical to the single-GPU calls (bit-exact). */
+
+/* H[u] for u in [u_begin, u_end) only (same definition as hec_debug_heavy);
+ * H is a device int32[n] array indexed by global vertex id. */
+HEC_API int hec_heavy_range(hec_ctx *ctx, const hec_graph *g, int64_t u_begin, int64_t u_end,
+                            int32_t *H);
+/* Mapping from a complete heavy-neighbour array H (device int32[n]): the
+ * resolution rounds and the relabel run over all vertices; M (device int32[n])
+ * is written for [u_begin, u_end) only.  *n_c (host) as hec_find_mapping. */
+HEC_API int hec_mapping_from_heavy(hec_ctx *ctx, const hec_graph *g, const int32_t *H,
+                                   uint64_t seed, int level, int64_t u_begin, int64_t u_end,
+                                   int32_t *M, int64_t *n_c);
+/* Split the coarse rows into `parts` contiguous ranges of about equal member-
+ * edge volume (sum of fine degrees of the members): host bounds[parts+1],
+ * bounds[0] = 0, bounds[parts] = n_c. */
+HEC_API int hec_balance_rows(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
+                             int parts, int64_t *bounds);
+/* Build coarse rows [a_begin, a_end) of G_c (the same rows build_coarse_graph
+ * produces).  counts (device int64[a_end-a_begin], may be NULL) receives the
+ * row lengths, *nnz_slice (host) their sum.  The slice is kept in ctx until
+ * hec_build_rows_write (no other libhec call on ctx in between). */
 HEC_API int hec_build_rows_count(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
-                                 int64_t a_begin, int64_t a_end, int64_t *counts);
-HEC_API int hec_build_rows_write(hec_ctx *ctx, const int64_t *offs, int32_t *col_c,
+                                 int64_t a_begin, int64_t a_end, int64_t *counts,
+                                 int64_t *nnz_slice);
+/* Write the pending slice: row_ptr_c[0..rows] = offset + local offsets (device
+ * int64[rows+1]), col_c/wgt_c[0..nnz_slice) and vwgt_c[0..rows) (device int32);
+ * pass pointers already advanced to the slice's global position. */
+HEC_API int hec_build_rows_write(hec_ctx *ctx, int64_t offset, int64_t *row_ptr_c, int32_t *col_c,
                                  int32_t *wgt_c, int32_t *vwgt_c);
 
 #ifdef __cplusplus

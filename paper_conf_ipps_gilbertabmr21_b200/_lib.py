@@ -18,7 +18,8 @@ EXPORTS = [
     "coarsen_hierarchy", "hec_hierarchy_levels", "hec_hierarchy_level",
     "hec_hierarchy_stop_reason", "hec_hierarchy_discarded_n_c", "hec_hierarchy_rounds",
     "hec_hierarchy_free", "hec_debug_heavy", "hec_debug_roots", "hec_build_rows_count",
-    "hec_build_rows_write", "hec_ctx_set_profiling", "hec_ctx_profile_reset", "hec_ctx_profile",
+    "hec_build_rows_write", "hec_heavy_range", "hec_mapping_from_heavy", "hec_balance_rows",
+    "hec_ctx_set_profiling", "hec_ctx_profile_reset", "hec_ctx_profile",
     "hec_ctx_launches",
 ]
 
@@ -79,8 +80,11 @@ def load():
         "hec_hierarchy_free": (None, [p]),
         "hec_debug_heavy": (i32, [p, G, p]),
         "hec_debug_roots": (i32, [p, G, p, u64, i32, p, ctypes.POINTER(i32)]),
-        "hec_build_rows_count": (i32, [p, G, p, i64, i64, i64, p]),
-        "hec_build_rows_write": (i32, [p, p, p, p, p]),
+        "hec_build_rows_count": (i32, [p, G, p, i64, i64, i64, p, ctypes.POINTER(i64)]),
+        "hec_build_rows_write": (i32, [p, i64, p, p, p, p]),
+        "hec_heavy_range": (i32, [p, G, i64, i64, p]),
+        "hec_mapping_from_heavy": (i32, [p, G, p, u64, i32, i64, i64, p, ctypes.POINTER(i64)]),
+        "hec_balance_rows": (i32, [p, G, p, i64, i32, ctypes.POINTER(i64)]),
         "hec_ctx_set_profiling": (i32, [p, i32]),
         "hec_ctx_profile_reset": (i32, [p]),
         "hec_ctx_profile": (i32, [p, ctypes.POINTER(HecPhaseTime), i32, ctypes.POINTER(i32)]),

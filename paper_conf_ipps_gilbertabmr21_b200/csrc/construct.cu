@@ -90,6 +90,7 @@ struct DegIn {
 struct RowWeightIn {
   Layout L;
   __device__ __forceinline__ int64_t operator()(int64_t a) const {
+    if (!L.active(a)) return 0;
     int64_t U = L.U(a);
     return U <= kSmallMax ? U + kRowW : 0;
   }
@@ -100,8 +101,9 @@ __global__ void k_big_rows(Layout L, int32_t *__restrict__ big_list, int32_t *__
                            unsigned *__restrict__ nbig, unsigned long long *__restrict__ vol) {
   int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   bool in = a < L.n_c;
-  int64_t U = in ? L.U(a) : 0;
-  bool big = in && U > kSmallMax;
+  const bool act = in && L.active(a);
+  int64_t U = act ? L.U(a) : 0;
+  bool big = act && U > kSmallMax;
   unsigned m = __ballot_sync(0xffffffffu, big);
   int lane = threadIdx.x & 31;
   unsigned base = 0;
@@ -142,9 +144,10 @@ struct BlockCountIn {
   const int64_t *S;  // exclusive scan of RowWeightIn
   bool dense;
   __device__ __forceinline__ int64_t operator()(int64_t a) const {
+    if (!L.active(a)) return 0;
     int64_t U = L.U(a);
     if (U > kSmallMax) return dense ? dense_chunks(L.n_c) : row_buckets(U, L.n_c);
-    if (a == 0) return 1;
+    if (a == L.a_lo) return 1;
     if (L.U(a - 1) > kSmallMax) return 1;
     return (S[a] / kWin) != (S[a - 1] / kWin) ? 1 : 0;
   }
@@ -163,11 +166,11 @@ __global__ void k_block_desc(Layout L, const int64_t *__restrict__ blk_ptr, cons
     blk[b0] = BlockDesc{B_SMALL, (int32_t)a, -1, 0};
   }
 }
-// row1 of SMALL blocks = first row of the next block (or n_c)
-__global__ void k_block_ends(int64_t nblocks, int64_t n_c, BlockDesc *__restrict__ blk) {
+// row1 of SMALL blocks = first row of the next block (or the end of the range)
+__global__ void k_block_ends(int64_t nblocks, int64_t a_hi, BlockDesc *__restrict__ blk) {
   int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= nblocks) return;
-  if (blk[k].kind == B_SMALL) blk[k].row1 = (k + 1 < nblocks) ? blk[k + 1].row0 : (int32_t)n_c;
+  if (blk[k].kind == B_SMALL) blk[k].row1 = (k + 1 < nblocks) ? blk[k + 1].row0 : (int32_t)a_hi;
 }
 
 // ------------------------------------------------------- a9 BUCKET partition
@@ -513,7 +516,9 @@ size_t ws_bytes_construct(int64_t n, int64_t nnz, int64_t n_c) {
   return b;
 }
 
-int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, CoarseOut *out) {
+int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, CoarseOut *out,
+                      int64_t a_lo, int64_t a_hi) {
+  if (a_hi < 0) a_hi = n_c;
   cudaStream_t s = ctx->stream;
   const int64_t n = g->n;
   out->n_c = n_c;
@@ -568,7 +573,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_LAUNCH_CHECK();
   }
   HEC_TRY(chained_scan(ctx, n, DegIn{members, g->row_ptr, member_ptr + n_c}, PtrOut{mpre}, st[1], mpre + n));
-  Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M};
+  if (a_lo < 0 || a_lo > a_hi || a_hi > n_c) {
+    set_error("coarse row range [%lld, %lld) outside [0, %lld)", (long long)a_lo, (long long)a_hi, (long long)n_c);
+    return HEC_EINVAL;
+  }
+  const int64_t n_out = a_hi - a_lo;  // rows produced by this call
+  Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi};
   k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));
   HEC_LAUNCH_CHECK();
@@ -625,7 +635,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   HEC_CUDA_TRY(cudaMemsetAsync(need_wide, 0, sizeof(int32_t) * (nblocks + 1), s));
   k_block_desc<<<nblk(n_c, 256), 256, 0, s>>>(L, blk_ptr, big_idx, dense, blk);
   HEC_LAUNCH_CHECK();
-  k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, n_c, blk);
+  k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
   HEC_LAUNCH_CHECK();
 
   RowsArgs A{};
@@ -710,8 +720,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   phase_end(ctx, ph_skew);
 
   // ---- work blocks (a8/a9 output), then placement (a10)
-  HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_c + 1)));
-  HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * n_c));
+  HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
+  HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
+  out->n_c = n_out;
   A.row_ptr_c = out->row_ptr;
   A.vwgt_c = out->vwgt;
   long long *trace = nullptr;
@@ -760,8 +771,43 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   HEC_TRY(launch_place(ctx, A));
   phase_end(ctx, ph_place);
   phase_set_bytes(ctx, ph_rows, 8.0 * (double)small_vol + 12.0 * dnc);
-  if (nblocks == 0) HEC_CUDA_TRY(cudaMemsetAsync(out->row_ptr, 0, sizeof(int64_t) * (n_c + 1), s));
+  if (nblocks == 0) HEC_CUDA_TRY(cudaMemsetAsync(out->row_ptr, 0, sizeof(int64_t) * (n_out + 1), s));
   ctx->stats.nnz_c = out->nnz_c;
+  return HEC_OK;
+}
+
+}  // namespace hec
+
+namespace hec {
+
+__global__ void k_row_volume(int64_t n, const int32_t *__restrict__ M, int64_t n_c,
+                             const int64_t *__restrict__ row_ptr, unsigned long long *__restrict__ U,
+                             int *__restrict__ err) {
+  int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u >= n) return;
+  int32_t a = M[u];
+  if (a < 0 || a >= n_c) { atomicOr(err, ERR_LABEL); return; }
+  atomicAdd(U + a, (unsigned long long)(row_ptr[u + 1] - row_ptr[u]));
+}
+
+int row_volume_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, int64_t *U) {
+  int *err = nullptr;
+  HEC_TRY(dev_alloc(ctx, (void **)&err, 64));
+  HEC_CUDA_TRY(cudaMemsetAsync(err, 0, 64, ctx->stream));
+  HEC_CUDA_TRY(cudaMemsetAsync(U, 0, sizeof(int64_t) * n_c, ctx->stream));
+  if (g->n > 0) {
+    k_row_volume<<<nblk(g->n, 256), 256, 0, ctx->stream>>>(g->n, M, n_c, g->row_ptr,
+                                                          reinterpret_cast<unsigned long long *>(U), err);
+    HEC_LAUNCH_CHECK();
+  }
+  int64_t r[1];
+  int rc = read_scalars(ctx, reinterpret_cast<int64_t *>(err), 1, r);
+  dev_free(ctx, err);
+  HEC_TRY(rc);
+  if ((int)(r[0] & 0xffffffff) & ERR_LABEL) {
+    set_error("M has values outside [0, n_c)");
+    return HEC_EINVAL;
+  }
   return HEC_OK;
 }
 

@@ -97,6 +97,8 @@ struct Layout {
   const int32_t *col;
   const int32_t *wgt;
   const int32_t *M;
+  int64_t a_lo, a_hi;  // coarse rows produced by this call (range partition, §8(e))
+  __device__ __forceinline__ bool active(int64_t a) const { return a >= a_lo && a < a_hi; }
   __device__ __forceinline__ int64_t upos(int64_t a) const { return mpre[member_ptr[a]]; }
   __device__ __forceinline__ int64_t U(int64_t a) const { return upos(a + 1) - upos(a); }
 };
@@ -205,7 +207,7 @@ struct RowsArgs {
   const int32_t *fb_b, *fb_w;
   // DENSE mode
   unsigned long long *dense;        // [nbig][n_c] sums, then staged pairs
-  // outputs
+  // outputs (row-indexed outputs start at row L.a_lo)
   int64_t *row_ptr_c;
   int32_t *col_c, *wgt_c, *vwgt_c;
   int *err;

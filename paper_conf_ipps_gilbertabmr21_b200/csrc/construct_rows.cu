@@ -301,10 +301,10 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
       }
       for (int r = t; r < R; r += kT) {
         const int32_t a = d.row0 + r;
-        A.row_ptr_c[a] = S.ucnt[r];  // relative to the block's output offset
+        A.row_ptr_c[a - L.a_lo] = S.ucnt[r];  // relative to the block's output offset
         const unsigned long long s = A.vw64[a];
         if (s > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
-        A.vwgt_c[a] = (int32_t)s;
+        A.vwgt_c[a - L.a_lo] = (int32_t)s;
       }
     } else {
       if (d.kind == B_BUCKET && !from_fallback) {
@@ -324,7 +324,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
       if (d.sub == 0 && t == 0) {
         const unsigned long long s = A.vw64[d.row0];
         if (s > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
-        A.vwgt_c[d.row0] = (int32_t)s;
+        A.vwgt_c[d.row0 - L.a_lo] = (int32_t)s;
       }
     }
     if (t == 0) {
@@ -356,7 +356,7 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
       A.col_c[O + q] = A.sc_col[P0 + q];
       A.wgt_c[O + q] = A.sc_wgt[P0 + q];
     }
-    for (int a = d.row0 + t; a < d.row1; a += kPlaceT) A.row_ptr_c[a] += O;
+    for (int a = d.row0 + t; a < d.row1; a += kPlaceT) A.row_ptr_c[a - L.a_lo] += O;
   } else {
     const int64_t bk = d.kind == B_BUCKET ? A.bkt_ptr[A.big_idx[d.row0]] + d.sub : 0;
     if (d.kind == B_DENSE) {
@@ -379,9 +379,9 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
         A.wgt_c[O + q] = A.pw_g[q0 + q];
       }
     }
-    if (d.sub == 0 && t == 0) A.row_ptr_c[d.row0] = O;
+    if (d.sub == 0 && t == 0) A.row_ptr_c[d.row0 - L.a_lo] = O;
   }
-  if (bi == A.nblocks - 1 && t == 0) A.row_ptr_c[L.n_c] = O + T;
+  if (bi == A.nblocks - 1 && t == 0) A.row_ptr_c[L.a_hi - L.a_lo] = O + T;
 }
 
 int launch_place(hec_ctx *ctx, const RowsArgs &A) {

@@ -368,8 +368,17 @@ struct CoarseOut {
   int32_t *col = nullptr, *wgt = nullptr, *vwgt = nullptr;
 };
 size_t ws_bytes_construct(int64_t n, int64_t nnz, int64_t n_c);
+// Coarse rows [a_lo, a_hi) only (a_hi < 0: all rows); out->n_c = a_hi - a_lo and
+// row_ptr/vwgt are indexed from a_lo, row_ptr[0] = 0 (range partition, §8(e)).
 int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
-                      CoarseOut *out);
+                      CoarseOut *out, int64_t a_lo = 0, int64_t a_hi = -1);
+// Heavy neighbours of fine rows [u0, u1) only (H indexed globally).
+int heavy_range_impl(hec_ctx *ctx, const hec_graph *g, int64_t u0, int64_t u1, int32_t *H);
+// Resolution rounds + relabel from a full heavy array H; M written for [u0, u1).
+int mapping_from_heavy_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio prio, int64_t u0,
+                            int64_t u1, int32_t *M, MapResult *res);
+// Member-edge volume U(a) of every coarse row (int64, device) for range balancing.
+int row_volume_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, int64_t *U);
 int validate_graph(hec_ctx *ctx, const hec_graph *g);
 
 }  // namespace hec

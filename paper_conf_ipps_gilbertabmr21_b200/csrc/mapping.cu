@@ -27,24 +27,26 @@ constexpr int kHvTile = kHvBlock * kHvItems;  // merge items (row ends + entries
 // Merge-path split of diagonal d between the row-end list row_ptr[1..n] and the
 // entry indices 0..nnz-1: returns x = row ends consumed (entries = d - x).
 __device__ __forceinline__ int64_t merge_path_x(int64_t d, const int64_t *__restrict__ row_ptr,
-                                                int64_t n, int64_t nnz) {
+                                                int64_t n, int64_t nnz, int64_t ebase) {
   int64_t lo = d - nnz > 0 ? d - nnz : 0;
   int64_t hi = d < n ? d : n;
   while (lo < hi) {
     int64_t mid = (lo + hi) >> 1;
-    if (__ldg(row_ptr + mid + 1) <= d - mid - 1) lo = mid + 1;
+    if (__ldg(row_ptr + mid + 1) - ebase <= d - mid - 1) lo = mid + 1;
     else hi = mid;
   }
   return lo;
 }
 
-__global__ void k_tile_coords(int64_t n, int64_t nnz, const int64_t *__restrict__ row_ptr,
+// Rows [vbase, vbase + n) of a CSR whose entries of those rows start at ebase:
+// row_ptr arguments point at row vbase, values are absolute (minus ebase here).
+__global__ void k_tile_coords(int64_t n, int64_t nnz, const int64_t *__restrict__ row_ptr, int64_t ebase,
                               int64_t ntiles, int64_t *__restrict__ cx) {
   int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (t > ntiles) return;
   int64_t d = t * kHvTile;
   if (d > n + nnz) d = n + nnz;
-  cx[t] = merge_path_x(d, row_ptr, n, nnz);
+  cx[t] = merge_path_x(d, row_ptr, n, nnz, ebase);
 }
 
 __device__ __forceinline__ uint64_t pack_key(int32_t w, int32_t v) {
@@ -95,7 +97,8 @@ struct HeavySmem {
 // when that row started in an earlier tile and ends here; mid_key[t]: partial of
 // the unfinished row at the tile's end (row x1 < n).
 __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
-                                                   const int64_t *__restrict__ row_ptr,
+                                                   const int64_t *__restrict__ row_ptr, int64_t ebase,
+                                                   int64_t vbase,
                                                    const int32_t *__restrict__ col,
                                                    const int32_t *__restrict__ wgt,
                                                    const int64_t *__restrict__ cx,
@@ -141,7 +144,7 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
   const int nrows = (int)(x1 - x0);  // rows whose end item lies in this tile
   for (int k = threadIdx.x; k <= nrows + 1; k += kHvBlock) {
     int64_t r = x0 + k;
-    int64_t b = r <= n ? __ldg(row_ptr + r) : nnz;
+    int64_t b = r <= n ? __ldg(row_ptr + r) - ebase : nnz;
     int64_t rel = b - y0;
     S.rb[k] = rel < -1 ? -1 : (rel > kHvTile + 1 ? kHvTile + 1 : (int32_t)rel);
     S.key[k] = 0;
@@ -171,7 +174,7 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
       if (k < nrows && y >= S.rb[k + 1]) {
         // end item of row x0+k
         if (S.rb[k] >= ystart) {
-          H[x0 + k] = key ? key_vertex(key) : (int32_t)(x0 + k);
+          H[vbase + x0 + k] = key ? key_vertex(key) : (int32_t)(vbase + x0 + k);
         } else if (key) {
           atomicMax((unsigned long long *)&S.key[k], (unsigned long long)key);
         }
@@ -194,7 +197,7 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
       if (k == 0 && S.rb[0] < 0) {
         head_key[t] = key;                 // tail piece of a row begun in an earlier tile
       } else if (key) {
-        H[x0 + k] = key_vertex(key);
+        H[vbase + x0 + k] = key_vertex(key);
       }
     } else if (x1 < n) {
       mid_key[t] = key;                    // unfinished row at the tile end
@@ -204,18 +207,18 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
 
 // Rows spanning tile boundaries: the tile holding the row's end item combines
 // its head piece with the mid pieces of the preceding tiles of the same row.
-__global__ void k_heavy_fixup(int64_t n, int64_t nnz, const int64_t *__restrict__ row_ptr,
-                              int64_t ntiles, const int64_t *__restrict__ cx,
+__global__ void k_heavy_fixup(int64_t n, int64_t nnz, const int64_t *__restrict__ row_ptr, int64_t ebase,
+                              int64_t vbase, int64_t ntiles, const int64_t *__restrict__ cx,
                               const uint64_t *__restrict__ head_key,
                               const uint64_t *__restrict__ mid_key, int32_t *__restrict__ H) {
   int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (t >= ntiles) return;
   int64_t x0 = cx[t], x1 = cx[t + 1];
   int64_t y0 = t * kHvTile - x0;
-  if (!(x0 < x1 && x0 < n && __ldg(row_ptr + x0) < y0)) return;
+  if (!(x0 < x1 && x0 < n && __ldg(row_ptr + x0) - ebase < y0)) return;
   int64_t x = x0;
   uint64_t key = head_key[t];
-  const int64_t rb = __ldg(row_ptr + x);
+  const int64_t rb = __ldg(row_ptr + x) - ebase;
   for (int64_t s = t - 1; s >= 0; --s) {
     if (cx[s + 1] != x) break;
     uint64_t m = mid_key[s];
@@ -223,12 +226,12 @@ __global__ void k_heavy_fixup(int64_t n, int64_t nnz, const int64_t *__restrict_
     int64_t ys = s * kHvTile - cx[s];
     if (rb >= ys) break;  // row begins in tile s
   }
-  H[x] = key ? key_vertex(key) : (int32_t)x;
+  H[vbase + x] = key ? key_vertex(key) : (int32_t)(vbase + x);
 }
 
-__global__ void k_fill_identity(int64_t n, int32_t *__restrict__ H) {
+__global__ void k_fill_identity(int64_t n, int64_t vbase, int32_t *__restrict__ H) {
   int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (u < n) H[u] = (int32_t)u;
+  if (u < n) H[vbase + u] = (int32_t)(vbase + u);
 }
 
 static inline unsigned nblk(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
@@ -238,11 +241,25 @@ static size_t heavy_ws(int64_t n, int64_t nnz) {
   return ws_bytes(ntiles + 1, 8) + 2 * ws_bytes(ntiles + 1, 8);
 }
 
-static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H) {
-  const int64_t n = g->n, nnz = g->nnz;
-  if (n == 0) return HEC_OK;
+// Heavy neighbours of rows [u0, u1): ebase = row_ptr[u0] and nnz of the range are
+// read from the device when the range is partial (one small synchronous read).
+static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 0, int64_t u1 = -1) {
+  if (u1 < 0) u1 = g->n;
+  const int64_t n = u1 - u0;
+  int64_t nnz = g->nnz, ebase = 0;
+  if (n <= 0) return HEC_OK;
+  if (u0 != 0 || u1 != g->n) {
+    HEC_CUDA_TRY(cudaMemcpyAsync(ctx->h_pinned, g->row_ptr + u0, sizeof(int64_t), cudaMemcpyDeviceToHost,
+                                 ctx->stream));
+    HEC_CUDA_TRY(cudaMemcpyAsync(ctx->h_pinned + 1, g->row_ptr + u1, sizeof(int64_t), cudaMemcpyDeviceToHost,
+                                 ctx->stream));
+    HEC_CUDA_TRY(cudaStreamSynchronize(ctx->stream));
+    ebase = ctx->h_pinned[0];
+    nnz = ctx->h_pinned[1] - ebase;
+  }
+  const int64_t *rp = g->row_ptr + u0;
   if (nnz == 0) {
-    k_fill_identity<<<nblk(n, 256), 256, 0, ctx->stream>>>(n, H);
+    k_fill_identity<<<nblk(n, 256), 256, 0, ctx->stream>>>(n, u0, H);
     HEC_LAUNCH_CHECK();
     return HEC_OK;
   }
@@ -251,7 +268,7 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H) {
   uint64_t *head = ws_take<uint64_t>(ctx, ntiles + 1);
   uint64_t *mid = ws_take<uint64_t>(ctx, ntiles + 1);
   if (!cx || !head || !mid) { set_error("workspace under-reserved (heavy)"); return HEC_EINVAL; }
-  k_tile_coords<<<nblk(ntiles + 1, 256), 256, 0, ctx->stream>>>(n, nnz, g->row_ptr, ntiles, cx);
+  k_tile_coords<<<nblk(ntiles + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, ntiles, cx);
   HEC_LAUNCH_CHECK();
   static bool attr = false;
   if (!attr) {
@@ -260,9 +277,9 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H) {
     attr = true;
   }
   k_heavy<<<(unsigned)ntiles, kHvBlock, sizeof(HeavySmem), ctx->stream>>>(
-      n, nnz, g->row_ptr, g->col, g->wgt, cx, H, head, mid);
+      n, nnz, rp, ebase, u0, g->col + ebase, g->wgt + ebase, cx, H, head, mid);
   HEC_LAUNCH_CHECK();
-  k_heavy_fixup<<<nblk(ntiles, 256), 256, 0, ctx->stream>>>(n, nnz, g->row_ptr, ntiles, cx, head,
+  k_heavy_fixup<<<nblk(ntiles, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, u0, ntiles, cx, head,
                                                             mid, H);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
@@ -400,22 +417,28 @@ struct RootFlagIn {
 };
 struct RootLabelOut {
   const uint8_t *status;
-  int32_t *M;
+  int32_t *lab;       // coarse id of each root (M itself when M covers all vertices)
   uint8_t *root_out;  // nullable
   __device__ __forceinline__ void operator()(int64_t u, int64_t prefix) const {
     bool r = status[u] == ROOT;
-    if (r) M[u] = (int32_t)prefix;
+    if (r) lab[u] = (int32_t)prefix;
     if (root_out) root_out[u] = r;
   }
 };
 
-__global__ void k_assign(int64_t n, const int32_t *__restrict__ H, const uint8_t *__restrict__ status,
+// M[u] for u in [u0, u1): the label of the first root on u's H-path.
+__global__ void k_assign(int64_t u0, int64_t u1, const int32_t *__restrict__ H,
+                         const uint8_t *__restrict__ status, const int32_t *__restrict__ lab,
                          int32_t *__restrict__ M) {
-  int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (u >= n || status[u] == ROOT) return;
+  int64_t u = u0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u >= u1) return;
+  if (status[u] == ROOT) {
+    if (lab != M) M[u] = lab[u];
+    return;
+  }
   int32_t x = H[u];
   while (status[x] != ROOT) x = H[x];
-  M[u] = M[x];
+  M[u] = lab[x];
 }
 
 int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes) {
@@ -427,20 +450,18 @@ int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes) {
   b += ws_bytes(kMaxTrackedRounds + 2, 4) + ws_bytes(4, 4) + ws_bytes(4, 8);
   b += heavy_ws(n, nnz);
   b += scan_ws_bytes(n);
+  b += ws_bytes(n, 4);          // labels (partial-range mapping)
   *bytes = b;
   return HEC_OK;
 }
 
 int heavy_only_impl(hec_ctx *ctx, const hec_graph *g, int32_t *H) { return run_heavy(ctx, g, H); }
 
-int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, uint8_t *root_out,
-                      int32_t *H_out, MapResult *res) {
+// a3-a5 from a full heavy-neighbour array H; M written for [u0, u1).
+static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio prio, int64_t u0, int64_t u1,
+                        int32_t *M, uint8_t *root_out, MapResult *res) {
   const int64_t n = g->n;
-  res->n_c = 0;
-  res->rounds = 0;
-  if (n == 0) return HEC_OK;
   cudaStream_t s = ctx->stream;
-  int32_t *H = H_out ? H_out : ws_take<int32_t>(ctx, n);
   uint8_t *status = ws_take<uint8_t>(ctx, n);
   uint8_t *rootflag = ws_take<uint8_t>(ctx, n);
   int32_t *blocked = ws_take<int32_t>(ctx, n);
@@ -449,15 +470,14 @@ int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, u
   unsigned *cnt = ws_take<unsigned>(ctx, kMaxTrackedRounds + 2);
   unsigned *bar = ws_take<unsigned>(ctx, 4);
   int64_t *scal = ws_take<int64_t>(ctx, 4);  // [0] n_c, [1] rounds (int32 in low word)
-  if (!H || !status || !rootflag || !blocked || !wl0 || !wl1 || !cnt || !bar || !scal) {
+  const bool full = u0 == 0 && u1 == n;
+  int32_t *lab = full ? M : ws_take<int32_t>(ctx, n);
+  if (!status || !rootflag || !blocked || !wl0 || !wl1 || !cnt || !bar || !scal || !lab) {
     set_error("workspace under-reserved (mapping)");
     return HEC_EINVAL;
   }
-  const double dn = (double)n, dnnz = (double)g->nnz;
-  int ph = phase_begin(ctx, "heavy", 8.0 * dnnz + 8.0 * (dn + 1) + 4.0 * dn);
-  HEC_TRY(run_heavy(ctx, g, H));
-  phase_end(ctx, ph);
-  ph = phase_begin(ctx, "rounds", 5.0 * dn);
+  const double dn = (double)n;
+  int ph = phase_begin(ctx, "rounds", 5.0 * dn);
   HEC_CUDA_TRY(cudaMemsetAsync(rootflag, 0, n, s));
   HEC_CUDA_TRY(cudaMemsetAsync(blocked, 0, sizeof(int32_t) * n, s));
   HEC_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(unsigned) * (kMaxTrackedRounds + 2), s));
@@ -487,15 +507,47 @@ int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, u
   // a4: labels by ascending root id; a5: inherit along H
   ScanTiles st = take_scan_tiles(ctx, n);
   if (!st.desc || !st.ticket) { set_error("workspace under-reserved (scan)"); return HEC_EINVAL; }
-  HEC_TRY(chained_scan(ctx, n, RootFlagIn{status}, RootLabelOut{status, M, root_out}, st, scal));
-  k_assign<<<nblk(n, 256), 256, 0, s>>>(n, H, status, M);
-  HEC_LAUNCH_CHECK();
+  HEC_TRY(chained_scan(ctx, n, RootFlagIn{status}, RootLabelOut{status, lab, root_out}, st, scal));
+  if (u1 > u0) {
+    k_assign<<<nblk(u1 - u0, 256), 256, 0, s>>>(u0, u1, H, status, lab, M);
+    HEC_LAUNCH_CHECK();
+  }
   phase_end(ctx, ph);
   int64_t h[2];
   HEC_TRY(read_scalars(ctx, scal, 2, h));
   res->n_c = h[0];
   res->rounds = (int)(int32_t)(h[1] & 0xffffffff);
   return HEC_OK;
+}
+
+int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, uint8_t *root_out,
+                      int32_t *H_out, MapResult *res) {
+  const int64_t n = g->n;
+  res->n_c = 0;
+  res->rounds = 0;
+  if (n == 0) return HEC_OK;
+  int32_t *H = H_out ? H_out : ws_take<int32_t>(ctx, n);
+  if (!H) { set_error("workspace under-reserved (mapping)"); return HEC_EINVAL; }
+  const double dn = (double)n, dnnz = (double)g->nnz;
+  int ph = phase_begin(ctx, "heavy", 8.0 * dnnz + 8.0 * (dn + 1) + 4.0 * dn);
+  HEC_TRY(run_heavy(ctx, g, H));
+  phase_end(ctx, ph);
+  return resolve_impl(ctx, g, H, prio, 0, n, M, root_out, res);
+}
+
+int heavy_range_impl(hec_ctx *ctx, const hec_graph *g, int64_t u0, int64_t u1, int32_t *H) {
+  int ph = phase_begin(ctx, "heavy", 0);
+  int rc = run_heavy(ctx, g, H, u0, u1);
+  phase_end(ctx, ph);
+  return rc;
+}
+
+int mapping_from_heavy_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio prio, int64_t u0,
+                            int64_t u1, int32_t *M, MapResult *res) {
+  res->n_c = 0;
+  res->rounds = 0;
+  if (g->n == 0) return HEC_OK;
+  return resolve_impl(ctx, g, H, prio, u0, u1, M, nullptr, res);
 }
 
 }  // namespace hec
