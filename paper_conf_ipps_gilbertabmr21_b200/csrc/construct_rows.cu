@@ -294,7 +294,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
     // ---- 4. stage the block's sorted distinct entries; k_place moves them
     const long long c1 = A.trace ? clock64() : 0;
     if (d.kind == B_SMALL) {
-      const int64_t P0 = L.mpre[S.mptr[0]];
+      const int64_t P0 = L.mpre[S.mptr[0]] - L.upos(L.a_lo);  // staging covers the active rows only
       for (int q = t; q < T; q += kT) {
         A.sc_col[P0 + q] = pb[q];
         A.sc_wgt[P0 + q] = pw[q];
@@ -351,7 +351,7 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   const int T = A.blk_cnt[bi];
   const int t = threadIdx.x;
   if (d.kind == B_SMALL) {
-    const int64_t P0 = L.mpre[L.member_ptr[d.row0]];
+    const int64_t P0 = L.mpre[L.member_ptr[d.row0]] - L.upos(L.a_lo);
     for (int q = t; q < T; q += kPlaceT) {
       A.col_c[O + q] = A.sc_col[P0 + q];
       A.wgt_c[O + q] = A.sc_wgt[P0 + q];

@@ -98,7 +98,7 @@ struct HeavySmem {
 // the unfinished row at the tile's end (row x1 < n).
 __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
                                                    const int64_t *__restrict__ row_ptr, int64_t ebase,
-                                                   int64_t vbase,
+                                                   int64_t vbase, int64_t esh,
                                                    const int32_t *__restrict__ col,
                                                    const int32_t *__restrict__ wgt,
                                                    const int64_t *__restrict__ cx,
@@ -113,8 +113,11 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
   const int64_t d1 = (d0 + kHvTile < total) ? d0 + kHvTile : total;
   const int64_t x0 = cx[t], x1 = cx[t + 1];
   const int64_t y0 = d0 - x0, y1 = d1 - x1;
-  const int64_t ybase = y0 & ~(int64_t)3;
-  const int64_t ya = (y0 + 3) & ~(int64_t)3, yb = y1 & ~(int64_t)3;
+  // col/wgt point 16-byte aligned at entry ebase - esh: local entry y is element
+  // y + esh there, so TMA sources stay 16-byte aligned for any range start
+  const int64_t y0a = y0 + esh, y1a = y1 + esh;
+  const int64_t ybase = y0a & ~(int64_t)3;
+  const int64_t ya = (y0a + 3) & ~(int64_t)3, yb = y1a & ~(int64_t)3;
   const bool bulk = yb > ya;
 
   if (threadIdx.x == 0) {
@@ -128,13 +131,13 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
   }
   // head / tail entries outside the 16-byte aligned interior
   {
-    int64_t hend = bulk ? ya : y1;
-    for (int64_t y = y0 + threadIdx.x; y < hend; y += kHvBlock) {
+    int64_t hend = bulk ? ya : y1a;
+    for (int64_t y = y0a + threadIdx.x; y < hend; y += kHvBlock) {
       S.col[y - ybase] = __ldg(col + y);
       S.wgt[y - ybase] = __ldg(wgt + y);
     }
     if (bulk) {
-      for (int64_t y = yb + threadIdx.x; y < y1; y += kHvBlock) {
+      for (int64_t y = yb + threadIdx.x; y < y1a; y += kHvBlock) {
         S.col[y - ybase] = __ldg(col + y);
         S.wgt[y - ybase] = __ldg(wgt + y);
       }
@@ -181,7 +184,7 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
         ++k;
         key = 0;
       } else {
-        int idx = (int)(y0 - ybase) + y;
+        int idx = (int)(y0a - ybase) + y;
         uint64_t kk = pack_key(S.wgt[idx], S.col[idx]);
         key = kk > key ? kk : key;
         ++y;
@@ -277,7 +280,8 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
     attr = true;
   }
   k_heavy<<<(unsigned)ntiles, kHvBlock, sizeof(HeavySmem), ctx->stream>>>(
-      n, nnz, rp, ebase, u0, g->col + ebase, g->wgt + ebase, cx, H, head, mid);
+      n, nnz, rp, ebase, u0, ebase & 3, g->col + (ebase & ~(int64_t)3), g->wgt + (ebase & ~(int64_t)3), cx, H,
+      head, mid);
   HEC_LAUNCH_CHECK();
   k_heavy_fixup<<<nblk(ntiles, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, u0, ntiles, cx, head,
                                                             mid, H);
