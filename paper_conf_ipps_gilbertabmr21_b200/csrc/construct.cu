@@ -54,13 +54,15 @@ __global__ void k_member_count(int64_t n, const int32_t *__restrict__ M, int64_t
 
 __global__ void k_member_fill(int64_t n, int64_t n_c, const int32_t *__restrict__ M,
                               const int64_t *__restrict__ member_ptr, unsigned *__restrict__ mcount,
-                              int32_t *__restrict__ members) {
+                              int32_t *__restrict__ members, const int64_t *__restrict__ row_ptr,
+                              int64_t *__restrict__ mstart) {
   int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (u >= n) return;
   int32_t a = M[u];
   if (a < 0 || a >= n_c) return;  // reported through err by k_member_count
   unsigned k = atomicSub(mcount + a, 1u) - 1u;
   members[member_ptr[a] + k] = (int32_t)u;
+  mstart[member_ptr[a] + k] = row_ptr[u];
 }
 
 struct BlkCntIn {
@@ -189,72 +191,134 @@ struct BucketsIn {
   __device__ __forceinline__ int64_t operator()(int64_t h) const { return row_buckets(L.U(big_list[h]), L.n_c); }
 };
 
+// ------------------------------------------------------------ expansion
+// Every member-edge position p in [P_lo, P_hi) (the active rows) gets its
+// fine entry's (b = M[v], w): Sb/Sw[p - P_lo].  One streaming pass with warp-level
+// member walks (no CTA barriers); all later construction kernels read these
+// arrays with coalesced loads.  Self entries are kept (b == own row): the
+// consumers know their row and drop them.
+constexpr int kXT = 256;       // threads per CTA
+constexpr int kXChunk = 2048;  // positions per warp task
+
+__global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restrict__ mstart,
+                                              int32_t *__restrict__ Sb, int32_t *__restrict__ Sw) {
+  __shared__ WarpExpTab W[kXT / 32];
+  const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
+  const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t gw = (int64_t)blockIdx.x * (kXT / 32) + wid;
+  const int64_t nw = (int64_t)gridDim.x * (kXT / 32);
+  for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
+    int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
+    int64_t i0 = warp_find_member(L, m_lo, m_hi, P);
+    int64_t q = P;
+    while (q < Pend) {
+      int32_t b4[4], w4[4];
+      int64_t m4[4];
+      const int got = warp_expand(L, mstart, m_hi, q, Pend, i0, W[wid], b4, w4, m4);
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const int off = lane + 32 * t;
+        if (off < got) {
+          Sb[q + off - P_lo] = b4[t];
+          Sw[q + off - P_lo] = w4[t];
+        }
+      }
+      q += got;
+    }
+  }
+}
+
+// ------------------------------------------------------- a9 BUCKET partition
+// Work units: big row h (list index) split into ceil(U/kCap) windows of kCap
+// member-edge positions; unit_ptr = exclusive scan over big rows.
+constexpr int kPartHist = 4096;  // buckets of a row counted in smem (more: global atomics)
+
 struct PartSmem {
-  MemberTab T;
-  int32_t hist[8192];
-  int64_t base[8192];
+  int32_t hist[kPartHist];
+  int64_t base[kPartHist];
 };
 
-// Expand unit `unit` into registers; kr = bucket of each entry (self dropped).
-__device__ __forceinline__ void unit_expand(const Layout &L, PartSmem &S, const int32_t *big_list, int64_t nbig,
-                                            const int64_t *unit_ptr, const int64_t *bkt_ptr, int64_t unit,
-                                            int64_t *h_out, int64_t *nb_out, int32_t (&kb)[kIt],
-                                            int32_t (&kw)[kIt], int32_t (&kr)[kIt]) {
-  const int64_t h = last_le(unit_ptr, 0, nbig, unit);
-  const int32_t a = big_list[h];
-  const int64_t P0 = L.upos(a) + (unit - unit_ptr[h]) * kCap;
+// floor(x / d) for x < 2^62 with a precomputed 64-bit reciprocal rcp = ceil(2^64 / d)
+__device__ __forceinline__ int64_t div_rcp(uint64_t x, uint64_t d, uint64_t rcp) {
+  uint64_t q = __umul64hi(x, rcp);
+  if (q * d > x) --q;
+  else if ((q + 1) * d <= x) ++q;
+  return (int64_t)q;
+}
+
+struct PartArgs {
+  Layout L;
+  const int32_t *big_list;
+  int64_t nbig;
+  const int64_t *unit_ptr;
+  const int64_t *bkt_ptr;
+  const int32_t *Sb, *Sw;   // expanded entries, indexed from upos(a_lo)
+  uint64_t nc_rcp;          // ceil(2^64 / n_c)
+};
+
+// Registers of a unit: bucket (kr) of each entry of big row h, self entries dropped.
+__device__ __forceinline__ void unit_load(const PartArgs &A, int64_t unit, int64_t *h_out, int64_t *nb_out,
+                                          int32_t (&kb)[kIt], int32_t (&kw)[kIt], int32_t (&kr)[kIt]) {
+  const Layout &L = A.L;
+  const int64_t h = last_le(A.unit_ptr, 0, A.nbig, unit);
+  const int32_t a = A.big_list[h];
+  const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kCap;
   const int64_t Pend = L.upos(a + 1);
-  const int nP = (int)((Pend - P0) < kCap ? (Pend - P0) : kCap);
-  int64_t m0, m1;
-  window_members(L, a, P0, nP, &m0, &m1);
-  expand_window(L, S.T, P0, nP, m0, m1, nullptr, 1, kb, kw, kr);
-  const int64_t nb = bkt_ptr[h + 1] - bkt_ptr[h];
+  const int64_t nb = A.bkt_ptr[h + 1] - A.bkt_ptr[h];
+  const int64_t P_lo = L.upos(L.a_lo);
 #pragma unroll
   for (int k = 0; k < kIt; ++k) {
-    if (kb[k] == a) kb[k] = -1;
-    kr[k] = kb[k] >= 0 ? (int32_t)(((int64_t)kb[k] * nb) / L.n_c) : 0;
+    const int64_t p = P0 + threadIdx.x + (int64_t)kT * k;
+    kb[k] = -1;
+    kw[k] = 0;
+    kr[k] = 0;
+    if (p < Pend) {
+      const int32_t b = A.Sb[p - P_lo];
+      if (b != a) {
+        kb[k] = b;
+        kw[k] = A.Sw[p - P_lo];
+        kr[k] = (int32_t)div_rcp((uint64_t)b * (uint64_t)nb, (uint64_t)L.n_c, A.nc_rcp);
+      }
+    }
   }
   *h_out = h;
   *nb_out = nb;
 }
 
-__global__ void __launch_bounds__(kT) k_part_count(Layout L, const int32_t *__restrict__ big_list, int64_t nbig,
-                                                   const int64_t *__restrict__ unit_ptr,
-                                                   const int64_t *__restrict__ bkt_ptr,
-                                                   unsigned *__restrict__ bkt_cnt) {
+__global__ void __launch_bounds__(kT) k_part_count(PartArgs A, unsigned *__restrict__ bkt_cnt) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   int32_t kb[kIt], kw[kIt], kr[kIt];
   int64_t h, nb;
-  unit_expand(L, S, big_list, nbig, unit_ptr, bkt_ptr, blockIdx.x, &h, &nb, kb, kw, kr);
-  const bool sh = nb <= 8192;
+  unit_load(A, blockIdx.x, &h, &nb, kb, kw, kr);
+  const bool sh = nb <= kPartHist;
   if (sh)
     for (int i = threadIdx.x; i < nb; i += kT) S.hist[i] = 0;
   __syncthreads();
+  const int64_t b0 = A.bkt_ptr[h];
 #pragma unroll
   for (int k = 0; k < kIt; ++k)
     if (kb[k] >= 0) {
       if (sh) atomicAdd(&S.hist[kr[k]], 1);
-      else atomicAdd(bkt_cnt + bkt_ptr[h] + kr[k], 1u);
+      else atomicAdd(bkt_cnt + b0 + kr[k], 1u);
     }
   __syncthreads();
   if (sh)
     for (int i = threadIdx.x; i < nb; i += kT)
-      if (S.hist[i]) atomicAdd(bkt_cnt + bkt_ptr[h] + i, (unsigned)S.hist[i]);
+      if (S.hist[i]) atomicAdd(bkt_cnt + b0 + i, (unsigned)S.hist[i]);
 }
 
-__global__ void __launch_bounds__(kT) k_part_write(Layout L, const int32_t *__restrict__ big_list, int64_t nbig,
-                                                   const int64_t *__restrict__ unit_ptr,
-                                                   const int64_t *__restrict__ bkt_ptr,
-                                                   const int64_t *__restrict__ bkt_off, unsigned *__restrict__ bkt_cur,
-                                                   int32_t *__restrict__ pb, int32_t *__restrict__ pw) {
+__global__ void __launch_bounds__(kT) k_part_write(PartArgs A, const int64_t *__restrict__ bkt_off,
+                                                   unsigned *__restrict__ bkt_cur, int32_t *__restrict__ pb,
+                                                   int32_t *__restrict__ pw) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   int32_t kb[kIt], kw[kIt], kr[kIt];
   int64_t h, nb;
-  unit_expand(L, S, big_list, nbig, unit_ptr, bkt_ptr, blockIdx.x, &h, &nb, kb, kw, kr);
-  const int64_t b0 = bkt_ptr[h];
-  if (nb <= 8192) {
+  unit_load(A, blockIdx.x, &h, &nb, kb, kw, kr);
+  const int64_t b0 = A.bkt_ptr[h];
+  if (nb <= kPartHist) {
     for (int i = threadIdx.x; i < nb; i += kT) S.hist[i] = 0;
     __syncthreads();
     int rank[kIt];
@@ -437,16 +501,19 @@ struct DenseArgs {
   int64_t nunits;
   unsigned *ticket;
   unsigned long long *dense;  // [nbig][n_c] (zeroed)
+  const int32_t *Sb, *Sw;     // expanded entries, indexed from upos(a_lo)
 };
 
 __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  MemberTab &T = *reinterpret_cast<MemberTab *>(smem_raw);
-  int32_t *acc = reinterpret_cast<int32_t *>(smem_raw + sizeof(MemberTab));
+  int32_t *acc = reinterpret_cast<int32_t *>(smem_raw);
   __shared__ int64_t s_unit;
+  __shared__ long long s_w[kT / 32];
   const Layout &L = A.L;
   const int nc = (int)L.n_c;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   for (int b = threadIdx.x; b < nc; b += kT) acc[b] = 0;
+  const int64_t P_lo = L.upos(L.a_lo);
   int64_t cur_h = -1;
   long long running = 0;  // weight accumulated since the last merge
   while (true) {
@@ -454,31 +521,29 @@ __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
     __syncthreads();
     const int64_t unit = s_unit;
     const int64_t h = unit < A.nunits ? last_le(A.unit_ptr, 0, A.nbig, unit) : -1;
-    int32_t kb[kIt], kw[kIt], kr[kIt];
-    int a = -1;
+    int32_t kb[kIt], kw[kIt];
+    long long usum = 0;  // exact weight of this thread's slots
+#pragma unroll
+    for (int k = 0; k < kIt; ++k) { kb[k] = -1; kw[k] = 0; }
     if (h >= 0) {
-      a = A.big_list[h];
+      const int32_t a = A.big_list[h];
       const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kCap;
       const int64_t Pend = L.upos(a + 1);
-      const int nP = (int)((Pend - P0) < kCap ? (Pend - P0) : kCap);
-      int64_t m0, m1;
-      window_members(L, a, P0, nP, &m0, &m1);
-      expand_window(L, T, P0, nP, m0, m1, nullptr, 1, kb, kw, kr);
-    }
-    long long usum = 0;  // exact weight of this unit
-    if (h >= 0) {
 #pragma unroll
-      for (int k = 0; k < kIt; ++k)
-        if (kb[k] >= 0 && kb[k] != a) usum += kw[k];
+      for (int k = 0; k < kIt; ++k) {
+        const int64_t p = P0 + threadIdx.x + (int64_t)kT * k;
+        if (p < Pend) {
+          const int32_t b = A.Sb[p - P_lo];
+          if (b != a) { kb[k] = b; kw[k] = A.Sw[p - P_lo]; usum += kw[k]; }
+        }
+      }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) usum += __shfl_xor_sync(0xffffffffu, usum, o);
-    __shared__ long long s_w[kT / 32];
-    if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = usum;
+    if (lane == 0) s_w[wid] = usum;
     __syncthreads();
     long long unit_w = 0;
     for (int w = 0; w < kT / 32; ++w) unit_w += s_w[w];
-    __syncthreads();
     if (cur_h >= 0 && (h != cur_h || running + unit_w > 0x7fffffffLL)) {  // merge the accumulator
       unsigned long long *dst = A.dense + cur_h * (int64_t)nc;
       for (int b = threadIdx.x; b < nc; b += kT) {
@@ -493,7 +558,7 @@ __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
     running += unit_w;
 #pragma unroll
     for (int k = 0; k < kIt; ++k)
-      if (kb[k] >= 0 && kb[k] != a) atomicAdd(acc + kb[k], kw[k]);
+      if (kb[k] >= 0) atomicAdd(acc + kb[k], kw[k]);
     __syncthreads();
   }
 }
@@ -506,6 +571,7 @@ size_t ws_bytes_construct(int64_t n, int64_t nnz, int64_t n_c) {
   b += ws_bytes(n_c + 1, 8);      // vw64
   b += ws_bytes(n_c + 1, 8);      // member_ptr
   b += ws_bytes(n + 1, 4);        // members
+  b += ws_bytes(n + 1, 8);        // mstart
   b += ws_bytes(n + 1, 8);        // mpre
   b += ws_bytes(n_c + 1, 8);      // window scan
   b += ws_bytes(n_c + 1, 8);      // blk_ptr
@@ -536,6 +602,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   unsigned long long *vw64 = ws_take<unsigned long long>(ctx, n_c + 1);
   int64_t *member_ptr = ws_take<int64_t>(ctx, n_c + 1);
   int32_t *members = ws_take<int32_t>(ctx, n + 1);
+  int64_t *mstart = ws_take<int64_t>(ctx, n + 1);
   int64_t *mpre = ws_take<int64_t>(ctx, n + 1);
   int64_t *Sw = ws_take<int64_t>(ctx, n_c + 1);
   int64_t *blk_ptr = ws_take<int64_t>(ctx, n_c + 1);
@@ -550,7 +617,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   int64_t *scal = ws_take<int64_t>(ctx, 32);
   ScanTiles st[6];
   for (auto &x : st) x = take_scan_tiles(ctx, n > n_c ? n : n_c);
-  if (!mcount || !vw64 || !member_ptr || !members || !mpre || !Sw || !blk_ptr || !big_list || !big_idx ||
+  if (!mcount || !vw64 || !member_ptr || !members || !mstart || !mpre || !Sw || !blk_ptr || !big_list || !big_idx ||
       !unit_ptr || !bkt_ptr || !counts || !scal || !st[5].desc) {
     set_error("workspace under-reserved (construct)");
     return HEC_EINVAL;
@@ -569,7 +636,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
   HEC_TRY(chained_scan(ctx, n_c, CountIn{mcount}, PtrOut{member_ptr}, st[0], member_ptr + n_c));
   if (n > 0) {
-    k_member_fill<<<nblk(n, 256), 256, 0, s>>>(n, n_c, M, member_ptr, mcount, members);
+    k_member_fill<<<nblk(n, 256), 256, 0, s>>>(n, n_c, M, member_ptr, mcount, members, g->row_ptr, mstart);
     HEC_LAUNCH_CHECK();
   }
   HEC_TRY(chained_scan(ctx, n, DegIn{members, g->row_ptr, member_ptr + n_c}, PtrOut{mpre}, st[1], mpre + n));
@@ -628,10 +695,23 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   int32_t *need_wide = arena_take<int32_t>(W2, nblocks + 1);
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
-  // SMALL staging is indexed by member-edge position (the space of all rows)
+  // expanded (b, w) of every active member-edge position; SMALL blocks stage
+  // their sorted rows in place over their own entries
   int32_t *sc_col = arena_take<int32_t>(W2, (size_t)(small_vol + big_vol) + 1);
   int32_t *sc_wgt = arena_take<int32_t>(W2, (size_t)(small_vol + big_vol) + 1);
   if (!sc_wgt) { set_error("workspace under-reserved (blocks)"); return HEC_EINVAL; }
+  {
+    const int phx = phase_begin(ctx, "expand", 12.0 * (double)(small_vol + big_vol) + 16.0 * dn);
+    const int64_t warps = (small_vol + big_vol + kXChunk - 1) / kXChunk;
+    int64_t grid = (warps + kXT / 32 - 1) / (kXT / 32);
+    const int64_t cap = (int64_t)ctx->num_sms * 8;
+    if (grid > cap) grid = cap;
+    if (grid > 0) {
+      k_expand<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
+      HEC_LAUNCH_CHECK();
+    }
+    phase_end(ctx, phx);
+  }
   HEC_CUDA_TRY(cudaMemsetAsync(need_wide, 0, sizeof(int32_t) * (nblocks + 1), s));
   k_block_desc<<<nblk(n_c, 256), 256, 0, s>>>(L, blk_ptr, big_idx, dense, blk);
   HEC_LAUNCH_CHECK();
@@ -662,7 +742,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_bucket_fallback, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(FbSmem)));
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_dense_accum, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)(sizeof(MemberTab) + 4 * kDenseMax)));
+                                      (int)(4 * kDenseMax)));
     attr = true;
   }
 
@@ -671,8 +751,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (nbig > 0 && dense) {
     unsigned long long *dn_arr = arena_take<unsigned long long>(W2, (size_t)nbig * n_c);
     HEC_CUDA_TRY(cudaMemsetAsync(dn_arr, 0, sizeof(unsigned long long) * nbig * n_c, s));
-    DenseArgs D{L, big_list, nbig, unit_ptr, nunits, counts + 2, dn_arr};
-    k_dense_accum<<<ctx->num_sms, kT, sizeof(MemberTab) + 4 * (size_t)n_c, s>>>(D);
+    DenseArgs D{L, big_list, nbig, unit_ptr, nunits, counts + 2, dn_arr, sc_col, sc_wgt};
+    int occ = 1;
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum, kT, 4 * (size_t)n_c));
+    if (occ < 1) occ = 1;
+    k_dense_accum<<<ctx->num_sms * occ, kT, 4 * (size_t)n_c, s>>>(D);
     HEC_LAUNCH_CHECK();
     A.dense = dn_arr;
   } else if (nbig > 0) {
@@ -691,11 +774,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     if (!fb_w) { set_error("workspace under-reserved (buckets)"); return HEC_EINVAL; }
     HEC_CUDA_TRY(cudaMemsetAsync(bkt_cnt, 0, sizeof(unsigned) * (nbkt + 1), s));
     HEC_CUDA_TRY(cudaMemsetAsync(bkt_cur, 0, sizeof(unsigned) * (nbkt + 1), s));
-    k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(L, big_list, nbig, unit_ptr, bkt_ptr, bkt_cnt);
+    PartArgs PA{L, big_list, nbig, unit_ptr, bkt_ptr, sc_col, sc_wgt,
+                (uint64_t)(~0ull / (uint64_t)n_c) + 1};  // ceil(2^64 / n_c), n_c > 32768 here
+    k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt);
     HEC_LAUNCH_CHECK();
     HEC_TRY(chained_scan(ctx, nbkt, CountIn{bkt_cnt}, PtrOut{bkt_off}, stb, bkt_off + nbkt));
-    k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(L, big_list, nbig, unit_ptr, bkt_ptr, bkt_off,
-                                                                bkt_cur, pb, pw);
+    k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, bkt_cur, pb, pw);
     HEC_LAUNCH_CHECK();
     k_fb_jobs<<<nblk(nbig, 256), 256, 0, s>>>(nbig, bkt_ptr, bkt_off, jobs, job_rn, counts + 4, fb_cnt, fb_off,
                                              reinterpret_cast<unsigned long long *>(scal + 10));

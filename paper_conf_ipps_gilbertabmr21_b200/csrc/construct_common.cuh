@@ -157,6 +157,78 @@ __device__ __forceinline__ void expand_window(const Layout &L, MemberTab &T, int
   }
 }
 
+// ------------------------------------------------------- warp expansion
+// Warp-private member window in shared memory.
+struct WarpExpTab {
+  int64_t mp[129];  // member-edge start of members i0 .. i0+128 (mpre)
+  int64_t ms[128];  // row_ptr[members[i]] (mstart)
+};
+
+// One warp expands the member-edge positions [P, limit) with limit <=
+// min(P + 128, Pend, start of member i0 + 128) into registers: slot t of lane l
+// is position P + l + 32 t; b = -1 marks empty slots.  Members are [i0, mend)
+// with i0 the member containing P; on return i0 is the member containing limit.
+// mem[t] receives the member index of the slot.  Only __syncwarp is used, so
+// warps of a CTA proceed independently.  Returns limit - P.
+__device__ __forceinline__ int warp_expand(const Layout &L, const int64_t *__restrict__ mstart, int64_t mend,
+                                           int64_t P, int64_t Pend, int64_t &i0, WarpExpTab &W,
+                                           int32_t (&b)[4], int32_t (&w)[4], int64_t (&mem)[4]) {
+  const int lane = threadIdx.x & 31;
+  const int64_t pend_m = L.mpre[mend];
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    const int64_t j = i0 + lane + 32 * t;
+    W.mp[lane + 32 * t] = j < mend ? L.mpre[j] : pend_m;
+    W.ms[lane + 32 * t] = j < mend ? mstart[j] : 0;
+  }
+  if (lane == 0) W.mp[128] = (i0 + 128 < mend) ? L.mpre[i0 + 128] : pend_m;
+  __syncwarp();
+  int64_t limit = P + 128;
+  if (Pend < limit) limit = Pend;
+  if (W.mp[128] < limit) limit = W.mp[128];
+  int64_t e[4];
+  unsigned valid = 0;
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    const int64_t q = P + lane + 32 * t;
+    b[t] = -1;
+    w[t] = 0;
+    if (q < limit) {
+      const int k = (int)last_le(W.mp, 0, 128, q);
+      e[t] = W.ms[k] + (q - W.mp[k]);
+      mem[t] = i0 + k;
+      valid |= 1u << t;
+    }
+  }
+#pragma unroll
+  for (int t = 0; t < 4; ++t)
+    if (valid & (1u << t)) { b[t] = __ldg(L.col + e[t]); w[t] = __ldg(L.wgt + e[t]); }
+#pragma unroll
+  for (int t = 0; t < 4; ++t)
+    if (valid & (1u << t)) b[t] = __ldg(L.M + b[t]);
+  i0 += last_le(W.mp, 0, 129, limit);
+  __syncwarp();
+  return (int)(limit - P);
+}
+
+// Largest member i in [lo, hi) with mpre[i] <= P (mpre[lo] <= P), by a warp:
+// 32-ary search, one coalesced probe per round.
+__device__ __forceinline__ int64_t warp_find_member(const Layout &L, int64_t lo, int64_t hi, int64_t P) {
+  const int lane = threadIdx.x & 31;
+  while (hi - lo > 32) {
+    const int64_t step = (hi - lo + 31) / 32;
+    const int64_t idx = lo + lane * step;
+    const bool le = idx < hi && L.mpre[idx] <= P;
+    const int k = __popc(__ballot_sync(0xffffffffu, le)) - 1;
+    const int64_t nlo = lo + k * step;
+    hi = nlo + step < hi ? nlo + step : hi;
+    lo = nlo;
+  }
+  const int64_t idx = lo + lane;
+  const bool le = idx < hi && L.mpre[idx] <= P;
+  return lo + __popc(__ballot_sync(0xffffffffu, le)) - 1;
+}
+
 // Members of big row a covering the window [P0, P0+nP): [m0, m1).
 __device__ __forceinline__ void window_members(const Layout &L, int32_t a, int64_t P0, int nP, int64_t *m0,
                                                int64_t *m1) {

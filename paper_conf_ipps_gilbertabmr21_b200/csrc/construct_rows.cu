@@ -26,7 +26,6 @@ template <bool WIDE>
 struct RowsSmemT {
   // phase-aliased areas: [expansion: member table] -> [hash keys] -> [bucket histogram]
   union {
-    MemberTab T;
     int32_t hkey[kHash];
     int32_t hist[kCap + 1];
   } a;
@@ -147,23 +146,36 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
       int32_t kb[kIt], kw[kIt], kr[kIt];
       if (d.kind == B_SMALL) {
         R = d.row1 - d.row0;
-        for (int r = t; r <= R; r += kT) S.mptr[r] = L.member_ptr[d.row0 + r];
+        for (int r = t; r <= R; r += kT) S.mptr[r] = L.upos(d.row0 + r);  // member-edge start of each row
         if (t == 0) S.wtot = 0;
         __syncthreads();
         for (int r = t; r < R; r += kT) {
           S.kmin[r] = INT32_MAX;
           S.kmax[r] = -1;
           S.ucnt[r] = 0;
-          const int32_t U = (int32_t)(L.mpre[S.mptr[r + 1]] - L.mpre[S.mptr[r]]);
+          const int32_t U = (int32_t)(S.mptr[r + 1] - S.mptr[r]);
           S.hbase[r] = U + (U >> 1) + 1;
         }
-        const int64_t m0 = S.mptr[0], m1 = S.mptr[R];
-        const int64_t P0 = L.mpre[m0];
-        const int nP = (int)(L.mpre[m1] - P0);
-        expand_window(L, S.a.T, P0, nP, m0, m1, S.mptr, R, kb, kw, kr);  // ends with a barrier
+        // entries of the block's rows, expanded by k_expand (coalesced)
+        const int64_t P0 = S.mptr[0];
+        const int nP = (int)(S.mptr[R] - P0);
+        const int64_t P_lo = L.upos(L.a_lo);
 #pragma unroll
-        for (int k = 0; k < kIt; ++k)
-          if (kb[k] >= 0 && kb[k] == d.row0 + kr[k]) kb[k] = -1;  // self entries are dropped (L280)
+        for (int k = 0; k < kIt; ++k) {
+          const int s = t + kT * k;
+          kb[k] = -1;
+          kw[k] = 0;
+          kr[k] = 0;
+          if (s < nP) {
+            const int32_t b = A.sc_col[P0 + s - P_lo];
+            const int r = (int)last_le(S.mptr, 0, R, P0 + s);
+            kr[k] = r;
+            if (b != d.row0 + r) {  // self entries are dropped (L280)
+              kb[k] = b;
+              kw[k] = A.sc_wgt[P0 + s - P_lo];
+            }
+          }
+        }
       } else {  // B_BUCKET: partitioned pairs of one skewed row (self entries already dropped)
         const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
         const int64_t q0 = A.bkt_off[bk], cnt = A.bkt_off[bk + 1] - q0;
@@ -294,7 +306,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
     // ---- 4. stage the block's sorted distinct entries; k_place moves them
     const long long c1 = A.trace ? clock64() : 0;
     if (d.kind == B_SMALL) {
-      const int64_t P0 = L.mpre[S.mptr[0]] - L.upos(L.a_lo);  // staging covers the active rows only
+      const int64_t P0 = S.mptr[0] - L.upos(L.a_lo);  // staging covers the active rows only
       for (int q = t; q < T; q += kT) {
         A.sc_col[P0 + q] = pb[q];
         A.sc_wgt[P0 + q] = pw[q];
