@@ -88,24 +88,32 @@ struct DegIn {
   }
 };
 
-// window weight of small rows (U + kRowW), 0 for big rows
+// Row classes by member-edge volume U (bound on the row's length):
+//   U <= kPieceMax                  warp pieces (windows of kPieceWin, weight U + kPieceRowW)
+//   kPieceMax < U <= big_thr        CTA work blocks (windows of kWin, weight U + kRowW)
+//   U > big_thr                     skewed: key-range buckets (BUCKET mode, big_thr =
+//                                   kPieceMax) or dense accumulation (DENSE mode)
+__host__ __device__ __forceinline__ int64_t big_threshold(bool dense) { return dense ? kSmallMax : kPieceMax; }
+
 struct RowWeightIn {
   Layout L;
+  bool dense;
   __device__ __forceinline__ int64_t operator()(int64_t a) const {
     if (!L.active(a)) return 0;
     int64_t U = L.U(a);
-    return U <= kSmallMax ? U + kRowW : 0;
+    if (U <= kPieceMax) return U + kPieceRowW;
+    return U <= big_threshold(dense) ? U + kRowW : 0;
   }
 };
 
 // big rows: list (unordered) + row -> list index; member-edge volume per class
-__global__ void k_big_rows(Layout L, int32_t *__restrict__ big_list, int32_t *__restrict__ big_idx,
+__global__ void k_big_rows(Layout L, int64_t big_thr, int32_t *__restrict__ big_list, int32_t *__restrict__ big_idx,
                            unsigned *__restrict__ nbig, unsigned long long *__restrict__ vol) {
   int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   bool in = a < L.n_c;
   const bool act = in && L.active(a);
   int64_t U = act ? L.U(a) : 0;
-  bool big = act && U > kSmallMax;
+  bool big = act && U > big_thr;
   unsigned m = __ballot_sync(0xffffffffu, big);
   int lane = threadIdx.x & 31;
   unsigned base = 0;
@@ -145,16 +153,21 @@ struct BlockCountIn {
   Layout L;
   const int64_t *S;  // exclusive scan of RowWeightIn
   bool dense;
+  __device__ __forceinline__ int cls(int64_t U) const {
+    return U <= kPieceMax ? 0 : (U <= big_threshold(dense) ? 1 : 2);
+  }
   __device__ __forceinline__ int64_t operator()(int64_t a) const {
     if (!L.active(a)) return 0;
-    int64_t U = L.U(a);
-    if (U > kSmallMax) return dense ? dense_chunks(L.n_c) : row_buckets(U, L.n_c);
-    if (a == L.a_lo) return 1;
-    if (L.U(a - 1) > kSmallMax) return 1;
-    return (S[a] / kWin) != (S[a - 1] / kWin) ? 1 : 0;
+    const int64_t U = L.U(a);
+    const int c = cls(U);
+    if (c == 2) return dense ? dense_chunks(L.n_c) : row_buckets(U, L.n_c);
+    if (a == L.a_lo || cls(L.U(a - 1)) != c) return 1;
+    const int64_t win = c == 0 ? kPieceWin : kWin;  // rows of one class are contiguous in S
+    return (S[a] / win) != (S[a - 1] / win) ? 1 : 0;
   }
 };
 
+// descriptors of PIECE / SMALL blocks and DENSE chunks (BUCKET blocks: k_bucket_blocks)
 __global__ void k_block_desc(Layout L, const int64_t *__restrict__ blk_ptr, const int32_t *__restrict__ big_idx,
                              bool dense, BlockDesc *__restrict__ blk) {
   int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -162,17 +175,17 @@ __global__ void k_block_desc(Layout L, const int64_t *__restrict__ blk_ptr, cons
   int64_t b0 = blk_ptr[a], b1 = blk_ptr[a + 1];
   if (b1 == b0) return;
   if (big_idx[a] >= 0) {
-    for (int64_t k = b0; k < b1; ++k)
-      blk[k] = BlockDesc{dense ? B_DENSE : B_BUCKET, (int32_t)a, (int32_t)a + 1, (int32_t)(k - b0)};
+    if (dense)
+      for (int64_t k = b0; k < b1; ++k) blk[k] = BlockDesc{B_DENSE, (int32_t)a, (int32_t)a + 1, (int32_t)(k - b0)};
   } else {
-    blk[b0] = BlockDesc{B_SMALL, (int32_t)a, -1, 0};
+    blk[b0] = BlockDesc{L.U(a) <= kPieceMax ? B_PIECE : B_SMALL, (int32_t)a, -1, 0};
   }
 }
-// row1 of SMALL blocks = first row of the next block (or the end of the range)
+// row1 of PIECE / SMALL blocks = first row of the next block (or the end of the range)
 __global__ void k_block_ends(int64_t nblocks, int64_t a_hi, BlockDesc *__restrict__ blk) {
   int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= nblocks) return;
-  if (blk[k].kind == B_SMALL) blk[k].row1 = (k + 1 < nblocks) ? blk[k + 1].row0 : (int32_t)a_hi;
+  if (rows_kind(blk[k].kind)) blk[k].row1 = (k + 1 < nblocks) ? blk[k + 1].row0 : (int32_t)a_hi;
 }
 
 // ------------------------------------------------------- a9 BUCKET partition
@@ -219,9 +232,9 @@ __global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restr
 #pragma unroll
       for (int t = 0; t < 4; ++t) {
         const int off = lane + 32 * t;
-        if (off < got) {
-          Sb[q + off - P_lo] = b4[t];
-          Sw[q + off - P_lo] = w4[t];
+        if (off < got) {  // streaming stores: keep M (gathered) resident in L2
+          __stcs(Sb + q + off - P_lo, b4[t]);
+          __stcs(Sw + q + off - P_lo, w4[t]);
         }
       }
       q += got;
@@ -466,27 +479,73 @@ __global__ void __launch_bounds__(kT) k_bucket_fallback(int64_t n_c, const int64
   }
 }
 
-// fallback jobs: buckets with more than kCap entries
-__global__ void k_fb_jobs(int64_t nbig, const int64_t *__restrict__ bkt_ptr, const int64_t *__restrict__ bkt_off,
-                          int64_t *__restrict__ jobs, int32_t *__restrict__ job_rn, unsigned *__restrict__ njobs,
-                          int32_t *__restrict__ fb_cnt, int64_t *__restrict__ fb_off,
-                          unsigned long long *__restrict__ fb_total) {
-  int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (h >= nbig) return;
+// Per bucket k (of big row h): its block descriptor, and a fallback job when it
+// holds more than kCap entries.
+__global__ void k_bucket_blocks(int64_t nbig, int64_t nbkt, const int32_t *__restrict__ big_list,
+                                const int64_t *__restrict__ bkt_ptr, const int64_t *__restrict__ bkt_off,
+                                const int64_t *__restrict__ blk_ptr, BlockDesc *__restrict__ blk,
+                                int64_t *__restrict__ jobs, int32_t *__restrict__ job_rn, unsigned *__restrict__ njobs,
+                                int32_t *__restrict__ fb_cnt, int64_t *__restrict__ fb_off,
+                                unsigned long long *__restrict__ fb_total) {
+  int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (k >= nbkt) return;
+  const int64_t h = last_le(bkt_ptr, 0, nbig, k);
   const int64_t b0 = bkt_ptr[h], b1 = bkt_ptr[h + 1];
-  for (int64_t k = b0; k < b1; ++k) {
-    int64_t c = bkt_off[k + 1] - bkt_off[k];
-    if (c > kCap) {
-      unsigned j = atomicAdd(njobs, 1u);
-      jobs[j] = k;
-      job_rn[2 * j] = (int32_t)(k - b0);
-      job_rn[2 * j + 1] = (int32_t)(b1 - b0);
-      fb_off[k] = (int64_t)atomicAdd(fb_total, (unsigned long long)c);
-      fb_cnt[k] = 0;
-    } else {
-      fb_cnt[k] = -1;
+  const int32_t a = big_list[h];
+  blk[blk_ptr[a] + (k - b0)] = BlockDesc{B_BUCKET, a, a + 1, (int32_t)(k - b0)};
+  const int64_t c = bkt_off[k + 1] - bkt_off[k];
+  if (c > kCap) {
+    unsigned j = atomicAdd(njobs, 1u);
+    jobs[j] = k;
+    job_rn[2 * j] = (int32_t)(k - b0);
+    job_rn[2 * j + 1] = (int32_t)(b1 - b0);
+    fb_off[k] = (int64_t)atomicAdd(fb_total, (unsigned long long)c);
+    fb_cnt[k] = 0;
+  } else {
+    fb_cnt[k] = -1;
+  }
+}
+
+// Tier lists: warp pieces (PIECE blocks, buckets of <= kPieceCap entries) and
+// CTA blocks (SMALL, DENSE, larger buckets).  Fallback buckets are complete:
+// their count is final here.  list_n: [0] warp list, [1] CTA list.
+__global__ void k_tiers(int64_t nblocks, const BlockDesc *__restrict__ blk, const int32_t *__restrict__ big_idx,
+                        const int64_t *__restrict__ bkt_ptr, const int64_t *__restrict__ bkt_off,
+                        const int32_t *__restrict__ fb_cnt, int32_t *__restrict__ blk_cnt,
+                        int32_t *__restrict__ list_w, int32_t *__restrict__ list_c, unsigned *__restrict__ list_n,
+                        const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
+  const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  int tier = -1;  // 0 warp, 1 CTA
+  if (bi < nblocks) {
+    const BlockDesc d = blk[bi];
+    // vertex weight of a skewed row (written by k_place): int32 bound
+    if (!rows_kind(d.kind) && d.sub == 0 && vw64[d.row0] > 0x7fffffffull) atomicOr(err, ERR_OVERFLOW);
+    if (d.kind == B_PIECE) tier = 0;
+    else if (d.kind != B_BUCKET) tier = 1;
+    else {
+      const int64_t bk = bkt_ptr[big_idx[d.row0]] + d.sub;
+      if (fb_cnt[bk] >= 0) blk_cnt[bi] = fb_cnt[bk];
+      else tier = (bkt_off[bk + 1] - bkt_off[bk] <= kPieceCap) ? 0 : 1;
     }
   }
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int q = 0; q < 2; ++q) {
+    const unsigned m = __ballot_sync(0xffffffffu, tier == q);
+    if (!m) continue;
+    const int leader = __ffs(m) - 1;
+    unsigned base = 0;
+    if (lane == leader) base = atomicAdd(list_n + q, (unsigned)__popc(m));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (tier == q) (q ? list_c : list_w)[base + __popc(m & ((1u << lane) - 1))] = (int32_t)bi;
+  }
+}
+
+// blocks flagged for the 64-bit pass
+__global__ void k_wide_list(int64_t nblocks, const int32_t *__restrict__ need_wide, int32_t *__restrict__ list,
+                            unsigned *__restrict__ n) {
+  const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (bi < nblocks && need_wide[bi]) list[atomicAdd(n, 1u)] = (int32_t)bi;
 }
 
 // ------------------------------------------------------------ a9 DENSE path
@@ -646,11 +705,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
   const int64_t n_out = a_hi - a_lo;  // rows produced by this call
   Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi};
-  k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_list, big_idx, counts + 0,
+  const bool dense = n_c <= kDenseMax;
+  k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_threshold(dense), big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));
   HEC_LAUNCH_CHECK();
-  HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L}, PtrOut{Sw}, st[2], Sw + n_c));
-  const bool dense = n_c <= kDenseMax;
+  HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, dense}, PtrOut{Sw}, st[2], Sw + n_c));
   HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 4, counts + 0, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
   phase_end(ctx, ph);
@@ -677,7 +736,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
 
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
-    size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 2 * ws_bytes(nblocks + 1, 4) +
+    size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 5 * ws_bytes(nblocks + 1, 4) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
     if (nbig > 0 && dense) b2 += ws_bytes((size_t)nbig * n_c, 8);
@@ -693,6 +752,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   BlockDesc *blk = arena_take<BlockDesc>(W2, nblocks + 1);
   int32_t *blk_cnt = arena_take<int32_t>(W2, nblocks + 1);
   int32_t *need_wide = arena_take<int32_t>(W2, nblocks + 1);
+  int32_t *list_w = arena_take<int32_t>(W2, nblocks + 1);     // warp-tier blocks
+  int32_t *list_c = arena_take<int32_t>(W2, nblocks + 1);     // CTA-tier blocks
+  int32_t *list_wide = arena_take<int32_t>(W2, nblocks + 1);  // blocks flagged for 64-bit sums
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
   // expanded (b, w) of every active member-edge position; SMALL blocks stage
@@ -714,8 +776,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
   HEC_CUDA_TRY(cudaMemsetAsync(need_wide, 0, sizeof(int32_t) * (nblocks + 1), s));
   k_block_desc<<<nblk(n_c, 256), 256, 0, s>>>(L, blk_ptr, big_idx, dense, blk);
-  HEC_LAUNCH_CHECK();
-  k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
   HEC_LAUNCH_CHECK();
 
   RowsArgs A{};
@@ -781,8 +841,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_TRY(chained_scan(ctx, nbkt, CountIn{bkt_cnt}, PtrOut{bkt_off}, stb, bkt_off + nbkt));
     k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, bkt_cur, pb, pw);
     HEC_LAUNCH_CHECK();
-    k_fb_jobs<<<nblk(nbig, 256), 256, 0, s>>>(nbig, bkt_ptr, bkt_off, jobs, job_rn, counts + 4, fb_cnt, fb_off,
-                                             reinterpret_cast<unsigned long long *>(scal + 10));
+    k_bucket_blocks<<<nblk(nbkt, 256), 256, 0, s>>>(nbig, nbkt, big_list, bkt_ptr, bkt_off, blk_ptr, blk, jobs,
+                                                   job_rn, counts + 4, fb_cnt, fb_off,
+                                                   reinterpret_cast<unsigned long long *>(scal + 10));
     HEC_LAUNCH_CHECK();
     HEC_CUDA_TRY(cudaMemcpyAsync(scal + 9, counts + 4, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
     int64_t rj[1];
@@ -802,6 +863,14 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.fb_w = fb_w;
   }
   phase_end(ctx, ph_skew);
+  // counts: [5] pieces ticket [6] warp list [7] CTA list [8] wide list
+  if (nblocks > 0) {
+    k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
+    HEC_LAUNCH_CHECK();
+    k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.fb_cnt, blk_cnt, list_w,
+                                              list_c, counts + 6, vw64, err);
+    HEC_LAUNCH_CHECK();
+  }
 
   // ---- work blocks (a8/a9 output), then placement (a10)
   HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
@@ -815,6 +884,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.trace = trace;
   }
   const int ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
+  A.list = list_w;
+  A.nlist = counts + 6;
+  HEC_TRY(launch_pieces(ctx, A, counts + 5));
+  A.list = list_c;
+  A.nlist = counts + 7;
   HEC_TRY(launch_rows(ctx, A, false));
   phase_end(ctx, ph_rows);
   if (trace) {
@@ -836,6 +910,10 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     // untouched) are redone with int64 sums
     HEC_CUDA_TRY(cudaMemsetAsync(counts + 1, 0, sizeof(unsigned), s));
     HEC_CUDA_TRY(cudaMemsetAsync(err, 0, sizeof(int), s));
+    k_wide_list<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, need_wide, list_wide, counts + 8);
+    HEC_LAUNCH_CHECK();
+    A.list = list_wide;
+    A.nlist = counts + 8;
     HEC_TRY(launch_rows(ctx, A, true));
     HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks));
     HEC_CUDA_TRY(cudaMemcpyAsync(scal + 12, blk_off + nblocks, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));

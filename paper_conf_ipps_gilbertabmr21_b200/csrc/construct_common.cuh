@@ -1,6 +1,6 @@
 // construct_common.cuh — shared pieces of CONSTRUCTCOARSEGRAPH (construct*.cu):
-// sizes, the member-edge layout, shared-memory member tables and the
-// edge-balanced expansion of fine entries into (b = M[v], w) register tuples.
+// sizes, the member-edge layout, the warp-level expansion of fine entries into
+// (b = M[v], w) register tuples, block descriptors and kernel arguments.
 #pragma once
 #include "hec_internal.cuh"
 
@@ -15,11 +15,17 @@ constexpr int kRowW = 8;           // per-row weight: bounds rows per block
 constexpr int kMaxRows = 2 * kWin / kRowW;  // 512
 constexpr int kSmallMax = kWin - kRowW;     // rows with U <= 2040 are small
 constexpr int kMC = 1024;          // member-table chunk
-constexpr int kBucketAvg = 1024;   // target entries per BUCKET
+constexpr int kBucketAvg = 128;    // target entries per BUCKET (one warp piece)
+constexpr int kPieceMax = 124;     // rows with U <= kPieceMax go to warp pieces
+constexpr int kPieceWin = 128;     // piece window weight (piece weight < 2*kPieceWin)
+constexpr int kPieceRowW = 4;      // per-row piece weight
+constexpr int kPieceRows = kPieceWin / kPieceRowW;  // rows per piece (all start in one window)
+constexpr int kPieceCap = 256;     // entries per warp piece
 constexpr int kDenseMax = 32768;   // n_c bound of the DENSE skew path
 constexpr int32_t kEmpty = -1;
 
-enum : int32_t { B_SMALL = 0, B_BUCKET = 1, B_DENSE = 2 };
+enum : int32_t { B_SMALL = 0, B_BUCKET = 1, B_DENSE = 2, B_PIECE = 3 };
+__host__ __device__ __forceinline__ bool rows_kind(int32_t k) { return k == B_SMALL || k == B_PIECE; }
 enum : int { ERR_LABEL = 1, ERR_OVERFLOW = 2, ERR_WIDE = 4 };
 
 inline unsigned nblk(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
@@ -103,60 +109,6 @@ struct Layout {
   __device__ __forceinline__ int64_t U(int64_t a) const { return upos(a + 1) - upos(a); }
 };
 
-struct MemberTab {
-  int64_t mstart[kMC];    // row_ptr[u] of the member
-  int32_t moff[kMC + 1];  // member's first position relative to the window start
-  int32_t mrow[kMC];      // local row of the member
-};
-
-// Expand the member-edge window [P0, P0+nP) (nP <= kCap), whose members are
-// [m0, m1), into registers: slot s = tid + kT*k holds (b = M[v], w, local row).
-// Slots without an entry keep kb = -1.  s_mptr[0..R]: member_ptr slice of the
-// rows (nullptr => one row, index 0).
-__device__ __forceinline__ void expand_window(const Layout &L, MemberTab &T, int64_t P0, int nP, int64_t m0,
-                                              int64_t m1, const int64_t *s_mptr, int R, int32_t (&kb)[kIt],
-                                              int32_t (&kw)[kIt], int32_t (&kr)[kIt]) {
-  const int t = threadIdx.x;
-#pragma unroll
-  for (int k = 0; k < kIt; ++k) { kb[k] = -1; kw[k] = 0; kr[k] = 0; }
-  for (int64_t cm = m0; cm < m1; cm += kMC) {
-    const int nm = (int)((m1 - cm) < kMC ? (m1 - cm) : kMC);
-    for (int i = t; i < nm; i += kT) {
-      int32_t u = L.members[cm + i];
-      T.mstart[i] = L.row_ptr[u];
-      T.moff[i] = (int32_t)(L.mpre[cm + i] - P0);
-      T.mrow[i] = s_mptr ? (int32_t)last_le(s_mptr, 0, R, cm + i) : 0;
-    }
-    if (t == 0) {
-      int64_t e = L.mpre[cm + nm] - P0;
-      T.moff[nm] = (int32_t)(e > (int64_t)kCap + 1 ? kCap + 1 : e);
-    }
-    __syncthreads();
-    const int lo = T.moff[0] > 0 ? T.moff[0] : 0;
-    const int hi = T.moff[nm] < nP ? T.moff[nm] : nP;
-    unsigned fresh = 0;
-    int64_t ev[kIt];
-#pragma unroll
-    for (int k = 0; k < kIt; ++k) {
-      const int s = t + kT * k;
-      ev[k] = 0;
-      if (s >= lo && s < hi) {
-        int i = (int)last_le(T.moff, 0, nm, s);
-        ev[k] = T.mstart[i] + (s - T.moff[i]);
-        kr[k] = T.mrow[i];
-        fresh |= 1u << k;
-      }
-    }
-#pragma unroll
-    for (int k = 0; k < kIt; ++k)
-      if (fresh & (1u << k)) { kb[k] = __ldg(L.col + ev[k]); kw[k] = __ldg(L.wgt + ev[k]); }
-#pragma unroll
-    for (int k = 0; k < kIt; ++k)
-      if (fresh & (1u << k)) kb[k] = __ldg(L.M + kb[k]);
-    __syncthreads();
-  }
-}
-
 // ------------------------------------------------------- warp expansion
 // Warp-private member window in shared memory.
 struct WarpExpTab {
@@ -202,7 +154,7 @@ __device__ __forceinline__ int warp_expand(const Layout &L, const int64_t *__res
   }
 #pragma unroll
   for (int t = 0; t < 4; ++t)
-    if (valid & (1u << t)) { b[t] = __ldg(L.col + e[t]); w[t] = __ldg(L.wgt + e[t]); }
+    if (valid & (1u << t)) { b[t] = __ldcs(L.col + e[t]); w[t] = __ldcs(L.wgt + e[t]); }  // streamed once
 #pragma unroll
   for (int t = 0; t < 4; ++t)
     if (valid & (1u << t)) b[t] = __ldg(L.M + b[t]);
@@ -227,20 +179,6 @@ __device__ __forceinline__ int64_t warp_find_member(const Layout &L, int64_t lo,
   const int64_t idx = lo + lane;
   const bool le = idx < hi && L.mpre[idx] <= P;
   return lo + __popc(__ballot_sync(0xffffffffu, le)) - 1;
-}
-
-// Members of big row a covering the window [P0, P0+nP): [m0, m1).
-__device__ __forceinline__ void window_members(const Layout &L, int32_t a, int64_t P0, int nP, int64_t *m0,
-                                               int64_t *m1) {
-  const int64_t m0r = L.member_ptr[a], m1r = L.member_ptr[a + 1];
-  *m0 = last_le(L.mpre, m0r, m1r, P0);
-  int64_t lo = *m0, hi = m1r - 1;  // last member i with mpre[i] < P0 + nP
-  while (lo < hi) {
-    int64_t mid = (lo + hi + 1) >> 1;
-    if (L.mpre[mid] < P0 + nP) lo = mid;
-    else hi = mid - 1;
-  }
-  *m1 = lo + 1;
 }
 
 struct BlockDesc {
@@ -284,6 +222,8 @@ struct RowsArgs {
   int32_t *col_c, *wgt_c, *vwgt_c;
   int *err;
   long long *trace;  // debug: per block (compute cycles, 0, kind, T); nullable
+  const int32_t *list;    // blocks of this launch (a tier list)
+  const unsigned *nlist;  // device count of `list`
 };
 
 // keys b with floor(b * nb / n_c) == k: [ceil(k n_c / nb), ceil((k+1) n_c / nb))
@@ -295,7 +235,9 @@ __host__ __device__ __forceinline__ void bucket_range(int64_t k, int64_t nb, int
 }
 
 // Work-block kernel and placement launchers (construct_rows.cu).
+// Work-block kernels take their blocks from A.list / *A.nlist (device count).
 int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide);
+int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket);  // construct_pieces.cu
 int launch_place(hec_ctx *ctx, const RowsArgs &A);
 
 }  // namespace hec

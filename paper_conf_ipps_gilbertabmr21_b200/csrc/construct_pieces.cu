@@ -1,0 +1,293 @@
+// construct_pieces.cu — warp-level work pieces of CONSTRUCTCOARSEGRAPH
+// (SURVEY §8 rows a8, a9).  A piece is either a window of consecutive small
+// coarse rows (member-edge volume U <= kPieceMax each, < 256 entries in total)
+// or one key-range bucket of a partitioned row with <= 256 entries.  One warp
+// owns a piece and never waits for other warps:
+//
+//  1. entries (b, w) — expanded by k_expand / partitioned by k_part_write —
+//     are loaded into registers (striped, coalesced); self entries are dropped;
+//  2. the packed keys (local row, b) are sorted with a register bitonic network
+//     over 64, 128 or 256 slots (shuffles across lanes, register swaps inside a
+//     lane) — the sort-based DEDUPWITHWTS that PAPER.md:L324 and Table II find
+//     fastest on GPUs, at warp scale and oblivious to the key distribution;
+//  3. equal adjacent keys are merged: inclusive prefix sums of w give each run's
+//     total (exact: the piece's total weight is checked to fit int32 first);
+//  4. the sorted distinct entries are staged in place over the piece's input and
+//     its count goes to blk_cnt (k_place moves them to the final CSR later).
+// A piece whose total weight exceeds int32 is flagged for the 64-bit CTA pass.
+#include <stdlib.h>
+
+#include "construct_common.cuh"
+
+namespace hec {
+
+constexpr int kPW = 8;  // warps per CTA
+
+struct PieceTab {
+  uint64_t ukey[kPieceCap];        // key of distinct entry u
+  int32_t upre[kPieceCap];         // inclusive weight prefix at the end of run u
+  int32_t rstart[kPieceRows + 1];  // row start positions, then first distinct index per row
+};
+
+template <typename K>
+struct KeyTraits;
+template <>
+struct KeyTraits<uint32_t> {  // row pieces: (row << 26) | b with b < 2^26; buckets: b
+  static constexpr int kShift = 26;
+  static constexpr uint32_t kPad = 0xffffffffu;
+};
+template <>
+struct KeyTraits<uint64_t> {  // row pieces: (row << 32) | b
+  static constexpr int kShift = 32;
+  static constexpr uint64_t kPad = ~0ull;
+};
+
+__device__ __forceinline__ uint32_t shfl_xor_k(uint32_t v, int m) { return __shfl_xor_sync(0xffffffffu, v, m); }
+__device__ __forceinline__ uint64_t shfl_xor_k(uint64_t v, int m) { return __shfl_xor_sync(0xffffffffu, v, m); }
+__device__ __forceinline__ uint32_t shfl_up_k(uint32_t v, int d) { return __shfl_up_sync(0xffffffffu, v, d); }
+__device__ __forceinline__ uint64_t shfl_up_k(uint64_t v, int d) { return __shfl_up_sync(0xffffffffu, v, d); }
+__device__ __forceinline__ uint32_t shfl_down_k(uint32_t v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
+__device__ __forceinline__ uint64_t shfl_down_k(uint64_t v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
+
+// Ascending bitonic sort of the 32*J (key, val) pairs of a warp; element
+// i = lane*J + k on return (blocked).  Input order is arbitrary.
+template <int J, typename K>
+__device__ __forceinline__ void warp_bitonic(K (&key)[J], int32_t (&val)[J]) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int size = 2; size <= 32 * J; size <<= 1) {
+#pragma unroll
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      if (stride >= J) {  // partner in lane ^ (stride / J), same register
+        const int lm = stride / J;
+        const bool upper = (lane & lm) != 0;
+        const bool asc = (lane & (size / J)) == 0;  // bit `size` of i = lane*J + k
+        // keep the min (f = 0) or the max (f = ~0: compare complemented keys)
+        const K f = (upper != asc) ? (K)0 : ~(K)0;
+#pragma unroll
+        for (int k = 0; k < J; ++k) {
+          const K pk = shfl_xor_k(key[k], lm);
+          const int32_t pv = __shfl_xor_sync(0xffffffffu, val[k], lm);
+          const bool take = (pk ^ f) < (key[k] ^ f);
+          // branch-free exchange (a select here compiles to a divergent branch)
+          const K tm = (K)0 - (K)take;
+          key[k] ^= (key[k] ^ pk) & tm;
+          val[k] ^= (val[k] ^ pv) & (int32_t)(0u - (uint32_t)take);
+        }
+      } else {  // partner in the same lane: registers k, k | stride
+#pragma unroll
+        for (int k = 0; k < J; ++k) {
+          if (k & stride) continue;
+          const int k2 = k | stride;
+          const bool asc = size < J ? (k & size) == 0 : (lane & (size / J)) == 0;
+          const K f = asc ? (K)0 : ~(K)0;
+          const bool sw = (key[k2] ^ f) < (key[k] ^ f);
+          const K dk = (key[k] ^ key[k2]) & ((K)0 - (K)sw);
+          const int32_t dv = (val[k] ^ val[k2]) & (int32_t)(0u - (uint32_t)sw);
+          key[k] ^= dk;
+          key[k2] ^= dk;
+          val[k] ^= dv;
+          val[k2] ^= dv;
+        }
+      }
+    }
+  }
+}
+
+// Sort, merge and stage one piece held in registers (padding slots carry kPad).
+// R > 0: row piece of R rows (keys carry the local row); R == 0: one bucket.
+// Returns the distinct count; row_ptr_rel[r] = first distinct index of row r.
+template <int J, typename K>
+__device__ __forceinline__ int piece_sort_merge(K (&key)[J], int32_t (&val)[J], PieceTab &S,
+                                                int32_t *__restrict__ dst_b, int32_t *__restrict__ dst_w,
+                                                int64_t base, int R, int64_t *__restrict__ row_ptr_rel) {
+  using KT = KeyTraits<K>;
+  const int lane = threadIdx.x & 31;
+  warp_bitonic<J, K>(key, val);
+  // key before slot 0 (previous lane's last; none for lane 0), key after slot J-1
+  K prevk = shfl_up_k(key[J - 1], 1);
+  if (lane == 0) prevk = KT::kPad;
+  K nextk = shfl_down_k(key[0], 1);
+  if (lane == 31) nextk = KT::kPad;
+  // inclusive weight prefix and run heads (padding has weight 0 and sorts last)
+  int32_t pre[J];
+  int run = 0, nh = 0;
+#pragma unroll
+  for (int k = 0; k < J; ++k) {
+    run += val[k];
+    pre[k] = run;
+    const K pk = k ? key[k - 1] : prevk;
+    nh += (key[k] != KT::kPad && pk != key[k]) ? 1 : 0;
+  }
+  int xs = run, xh = nh;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int ys = __shfl_up_sync(0xffffffffu, xs, o), yh = __shfl_up_sync(0xffffffffu, xh, o);
+    if (lane >= o) { xs += ys; xh += yh; }
+  }
+  const int T = __shfl_sync(0xffffffffu, xh, 31);
+  int u = xh - nh;              // distinct entries before this lane's first slot
+  const int woff = xs - run;    // weight before this lane's first slot
+  if (lane < R) S.rstart[lane] = T;  // rows without distinct entries: fixed below
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < J; ++k) {
+    if (key[k] == KT::kPad) break;
+    const K pk = k ? key[k - 1] : prevk;
+    if (pk != key[k]) {  // head of run u
+      if (R > 0 && (pk >> KT::kShift) != (key[k] >> KT::kShift)) S.rstart[(int)(key[k] >> KT::kShift)] = u;
+      ++u;
+    }
+    const K nk = k + 1 < J ? key[k + 1] : nextk;
+    if (nk != key[k]) {  // tail of run u - 1
+      S.ukey[u - 1] = (uint64_t)key[k];
+      S.upre[u - 1] = woff + pre[k];
+    }
+  }
+  __syncwarp();
+  const uint64_t mask = R > 0 ? (1ull << KT::kShift) - 1 : 0xffffffffull;
+  for (int q = lane; q < T; q += 32) {
+    dst_b[base + q] = (int32_t)(S.ukey[q] & mask);
+    dst_w[base + q] = S.upre[q] - (q ? S.upre[q - 1] : 0);
+  }
+  if (R > 0) {  // rows without entries start where the next non-empty row starts
+    int v = lane < R ? S.rstart[lane] : T;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_down_sync(0xffffffffu, v, o);
+      if (lane + o < 32) v = min(v, y);
+    }
+    if (lane < R) row_ptr_rel[lane] = v;
+  }
+  __syncwarp();
+  return T;
+}
+
+// Load a piece (striped) into J slots per lane, check the int32 bound, sort/merge.
+// Returns the distinct count, or -1 when the piece needs 64-bit sums.
+template <int J, typename K>
+__device__ __forceinline__ int piece_run(int32_t row0, PieceTab &S, int R, int n, int32_t *__restrict__ src_b,
+                                         int32_t *__restrict__ src_w, int64_t base, int64_t *row_ptr_rel) {
+  using KT = KeyTraits<K>;
+  const int lane = threadIdx.x & 31;
+  K key[J];
+  int32_t val[J];
+#pragma unroll
+  for (int k = 0; k < J; ++k) {
+    const int s = lane + 32 * k;
+    key[k] = KT::kPad;
+    val[k] = 0;
+    if (s < n) {
+      const int32_t b = __ldcs(src_b + base + s);
+      const int32_t w = __ldcs(src_w + base + s);
+      if (R > 0) {
+        const int r = (int)last_le(S.rstart, 0, R, s);
+        if (b != row0 + r) {  // self entries are dropped (L280)
+          key[k] = ((K)r << KT::kShift) | (K)(uint32_t)b;
+          val[k] = w;
+        }
+      } else {
+        key[k] = (K)(uint32_t)b;
+        val[k] = w;
+      }
+    }
+  }
+  __syncwarp();  // rstart is rewritten by piece_sort_merge
+  long long wsum = 0;
+#pragma unroll
+  for (int k = 0; k < J; ++k) wsum += val[k];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) wsum += __shfl_xor_sync(0xffffffffu, wsum, o);
+  if (wsum > 0x7fffffffLL) return -1;
+  return piece_sort_merge<J, K>(key, val, S, src_b, src_w, base, R, row_ptr_rel);
+}
+
+template <int J>
+__device__ __forceinline__ int piece_dispatch(bool wide_keys, int32_t row0, PieceTab &S, int R, int n,
+                                              int32_t *src_b, int32_t *src_w, int64_t base, int64_t *rp) {
+  if (R > 0 && wide_keys) return piece_run<J, uint64_t>(row0, S, R, n, src_b, src_w, base, rp);
+  return piece_run<J, uint32_t>(row0, S, R, n, src_b, src_w, base, rp);
+}
+
+template <bool WIDE_KEYS>
+__global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__restrict__ ticket) {
+  __shared__ PieceTab tabs[kPW];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  PieceTab &S = tabs[wid];
+  const Layout &L = A.L;
+  const int64_t P_lo = L.upos(L.a_lo);
+  const int64_t nlist = *A.nlist;
+  while (true) {
+    int64_t item = 0;
+    if (lane == 0) item = (int64_t)atomicAdd(ticket, 1u);
+    item = __shfl_sync(0xffffffffu, item, 0);
+    if (item >= nlist) return;
+    const int64_t bi = A.list[item];
+    const BlockDesc d = A.blk[bi];
+    int R, n;
+    int64_t base;  // where the piece's entries are read and its result is staged
+    int32_t *src_b, *src_w;
+    int64_t *rp = nullptr;
+    if (d.kind == B_PIECE) {
+      R = d.row1 - d.row0;
+      const int64_t P0 = L.upos(d.row0);
+      for (int r = lane; r <= R; r += 32) S.rstart[r] = (int32_t)(L.upos(d.row0 + r) - P0);
+      __syncwarp();
+      n = S.rstart[R];
+      base = P0 - P_lo;
+      src_b = A.sc_col;
+      src_w = A.sc_wgt;
+      rp = A.row_ptr_c + (d.row0 - L.a_lo);
+    } else {  // B_BUCKET with <= kPieceCap entries (self entries already dropped)
+      R = 0;
+      const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
+      base = A.bkt_off[bk];
+      n = (int)(A.bkt_off[bk + 1] - base);
+      src_b = A.pb_g;
+      src_w = A.pw_g;
+    }
+    int T;
+    if (n <= 64) T = piece_dispatch<2>(WIDE_KEYS, d.row0, S, R, n, src_b, src_w, base, rp);
+    else if (n <= 128) T = piece_dispatch<4>(WIDE_KEYS, d.row0, S, R, n, src_b, src_w, base, rp);
+    else T = piece_dispatch<8>(WIDE_KEYS, d.row0, S, R, n, src_b, src_w, base, rp);
+    if (T < 0) {
+      if (lane == 0) {
+        A.need_wide[bi] = 1;
+        atomicOr(A.err, ERR_WIDE);
+      }
+      continue;
+    }
+    if (d.kind == B_PIECE) {
+      for (int r = lane; r < R; r += 32) {
+        const int32_t a = d.row0 + r;
+        const unsigned long long s = A.vw64[a];
+        if (s > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
+        A.vwgt_c[a - L.a_lo] = (int32_t)s;
+      }
+    }  // (vertex weights of skewed rows: k_place)
+    if (lane == 0) A.blk_cnt[bi] = T;
+  }
+}
+
+// Persistent: one grid of resident CTAs; the list length is read on the device.
+// Keys of row pieces pack (row, b) into 32 bits while n_c <= 2^26.
+int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket) {
+  static int occ[2] = {0, 0};
+  if (!occ[0]) {
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_pieces<false>, kPW * 32, 0));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_pieces<true>, kPW * 32, 0));
+    if (occ[0] < 1) occ[0] = 1;
+    if (occ[1] < 1) occ[1] = 1;
+  }
+  // (HEC_FORCE_WIDE_KEYS: test hook that exercises the 64-bit key path on small graphs)
+  const bool wide_keys = A.L.n_c > (1ll << KeyTraits<uint32_t>::kShift) || getenv("HEC_FORCE_WIDE_KEYS") != nullptr;
+  int64_t grid = (int64_t)ctx->num_sms * occ[wide_keys ? 1 : 0];
+  if (A.nblocks < grid * kPW) grid = (A.nblocks + kPW - 1) / kPW;
+  if (grid < 1) return HEC_OK;
+  if (wide_keys) k_pieces<true><<<(unsigned)grid, kPW * 32, 0, ctx->stream>>>(A, ticket);
+  else k_pieces<false><<<(unsigned)grid, kPW * 32, 0, ctx->stream>>>(A, ticket);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
+}  // namespace hec

@@ -97,19 +97,16 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
   const int t = threadIdx.x;
   const Layout &L = A.L;
   while (true) {
-    if (t == 0) S.blk = (int32_t)atomicAdd(A.ticket, 1u);
+    if (t == 0) {
+      const unsigned it = atomicAdd(A.ticket, 1u);
+      S.blk = it < *A.nlist ? A.list[it] : -1;
+    }
     __syncthreads();
     const int64_t bi = S.blk;
-    if (bi >= A.nblocks) return;
-    if (WIDE && !A.need_wide[bi]) {  // the 64-bit pass redoes only flagged blocks
-      __syncthreads();
-      continue;
-    }
+    if (bi < 0) return;
     const BlockDesc d = A.blk[bi];
     const long long c0 = A.trace ? clock64() : 0;
     int T = 0, R = 1;
-    bool from_fallback = false;
-    int64_t fb0 = 0;
     if (d.kind == B_DENSE) {
       // key chunk [k0, k0 + kCap) of a dense row, already in key order
       const int32_t h = A.big_idx[d.row0];
@@ -136,15 +133,10 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
           ++pos;
         }
       }
-    } else if (d.kind == B_BUCKET && A.fb_cnt[A.bkt_ptr[A.big_idx[d.row0]] + d.sub] >= 0) {
-      const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
-      T = A.fb_cnt[bk];
-      fb0 = A.fb_off[bk];
-      from_fallback = true;
-    } else {
+    } else {  // (fallback buckets are in no list: their counts come from k_tiers)
       // ---- 1. entries into registers
       int32_t kb[kIt], kw[kIt], kr[kIt];
-      if (d.kind == B_SMALL) {
+      if (rows_kind(d.kind)) {
         R = d.row1 - d.row0;
         for (int r = t; r <= R; r += kT) S.mptr[r] = L.upos(d.row0 + r);  // member-edge start of each row
         if (t == 0) S.wtot = 0;
@@ -305,7 +297,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
     __syncthreads();
     // ---- 4. stage the block's sorted distinct entries; k_place moves them
     const long long c1 = A.trace ? clock64() : 0;
-    if (d.kind == B_SMALL) {
+    if (rows_kind(d.kind)) {
       const int64_t P0 = S.mptr[0] - L.upos(L.a_lo);  // staging covers the active rows only
       for (int q = t; q < T; q += kT) {
         A.sc_col[P0 + q] = pb[q];
@@ -319,7 +311,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
         A.vwgt_c[a - L.a_lo] = (int32_t)s;
       }
     } else {
-      if (d.kind == B_BUCKET && !from_fallback) {
+      if (d.kind == B_BUCKET) {
         const int64_t q0 = A.bkt_off[A.bkt_ptr[A.big_idx[d.row0]] + d.sub];
         for (int q = t; q < T; q += kT) {  // in place over the bucket's own pairs
           A.pb_g[q0 + q] = pb[q];
@@ -333,19 +325,14 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
           st[2 * q + 1] = pw[q];
         }
       }
-      if (d.sub == 0 && t == 0) {
-        const unsigned long long s = A.vw64[d.row0];
-        if (s > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
-        A.vwgt_c[d.row0 - L.a_lo] = (int32_t)s;
-      }
     }
     if (t == 0) {
       A.blk_cnt[bi] = T;
       if (A.trace) {
         A.trace[4 * bi] = c1 - c0;
         // expansion cycles << 32 | hashing cycles (0 for DENSE / fallback blocks)
-        A.trace[4 * bi + 1] = (d.kind == B_DENSE || from_fallback) ? 0 : (S.tx[0] << 32) | (S.tx[1] & 0xffffffff);
-        A.trace[4 * bi + 2] = d.kind * 100000 + (d.kind == B_SMALL ? R : d.sub);
+        A.trace[4 * bi + 1] = d.kind == B_DENSE ? 0 : (S.tx[0] << 32) | (S.tx[1] & 0xffffffff);
+        A.trace[4 * bi + 2] = d.kind * 100000 + (rows_kind(d.kind) ? R : d.sub);
         A.trace[4 * bi + 3] = T;
       }
     }
@@ -353,52 +340,58 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
   }
 }
 
-// One CTA per work block: copy its staged entries to the final CSR position.
+// One warp per work block: copy its staged entries to the final CSR position
+// (blocks hold ~100 - 4096 entries; a CTA per block would be launch-bound).
 constexpr int kPlaceT = 256;
+__device__ __forceinline__ void warp_copy(int32_t *__restrict__ dc, int32_t *__restrict__ dw,
+                                          const int32_t *__restrict__ sc, const int32_t *__restrict__ sw, int T,
+                                          int lane) {
+  for (int q = lane; q < T; q += 32) {
+    dc[q] = __ldcs(sc + q);
+    dw[q] = __ldcs(sw + q);
+  }
+}
 __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
-  const int64_t bi = blockIdx.x;
+  const int lane = threadIdx.x & 31;
+  const int64_t bi = (int64_t)blockIdx.x * (kPlaceT / 32) + (threadIdx.x >> 5);
+  if (bi >= A.nblocks) return;
   const BlockDesc d = A.blk[bi];
   const Layout &L = A.L;
   const int64_t O = A.blk_off[bi];
   const int T = A.blk_cnt[bi];
-  const int t = threadIdx.x;
-  if (d.kind == B_SMALL) {
-    const int64_t P0 = L.mpre[L.member_ptr[d.row0]] - L.upos(L.a_lo);
-    for (int q = t; q < T; q += kPlaceT) {
-      A.col_c[O + q] = A.sc_col[P0 + q];
-      A.wgt_c[O + q] = A.sc_wgt[P0 + q];
-    }
-    for (int a = d.row0 + t; a < d.row1; a += kPlaceT) A.row_ptr_c[a - L.a_lo] += O;
+  if (rows_kind(d.kind)) {
+    const int64_t P0 = L.upos(d.row0) - L.upos(L.a_lo);
+    warp_copy(A.col_c + O, A.wgt_c + O, A.sc_col + P0, A.sc_wgt + P0, T, lane);
+    for (int a = d.row0 + lane; a < d.row1; a += 32) A.row_ptr_c[a - L.a_lo] += O;
   } else {
-    const int64_t bk = d.kind == B_BUCKET ? A.bkt_ptr[A.big_idx[d.row0]] + d.sub : 0;
     if (d.kind == B_DENSE) {
       const int32_t *st = reinterpret_cast<const int32_t *>(A.dense + (int64_t)A.big_idx[d.row0] * L.n_c +
                                                             (int64_t)d.sub * kCap);
-      for (int q = t; q < T; q += kPlaceT) {
+      for (int q = lane; q < T; q += 32) {
         A.col_c[O + q] = st[2 * q];
         A.wgt_c[O + q] = st[2 * q + 1];
       }
-    } else if (A.fb_cnt[bk] >= 0) {
-      const int64_t f0 = A.fb_off[bk];
-      for (int q = t; q < T; q += kPlaceT) {
-        A.col_c[O + q] = A.fb_b[f0 + q];
-        A.wgt_c[O + q] = A.fb_w[f0 + q];
-      }
     } else {
-      const int64_t q0 = A.bkt_off[bk];
-      for (int q = t; q < T; q += kPlaceT) {
-        A.col_c[O + q] = A.pb_g[q0 + q];
-        A.wgt_c[O + q] = A.pw_g[q0 + q];
+      const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
+      if (A.fb_cnt[bk] >= 0) {
+        const int64_t f0 = A.fb_off[bk];
+        warp_copy(A.col_c + O, A.wgt_c + O, A.fb_b + f0, A.fb_w + f0, T, lane);
+      } else {
+        const int64_t q0 = A.bkt_off[bk];
+        warp_copy(A.col_c + O, A.wgt_c + O, A.pb_g + q0, A.pw_g + q0, T, lane);
       }
     }
-    if (d.sub == 0 && t == 0) A.row_ptr_c[d.row0 - L.a_lo] = O;
+    if (d.sub == 0 && lane == 0) {  // the row's first block: row start and vertex weight
+      A.row_ptr_c[d.row0 - L.a_lo] = O;
+      A.vwgt_c[d.row0 - L.a_lo] = (int32_t)A.vw64[d.row0];  // bound checked by k_tiers
+    }
   }
-  if (bi == A.nblocks - 1 && t == 0) A.row_ptr_c[L.a_hi - L.a_lo] = O + T;
+  if (bi == A.nblocks - 1 && lane == 0) A.row_ptr_c[L.a_hi - L.a_lo] = O + T;
 }
 
 int launch_place(hec_ctx *ctx, const RowsArgs &A) {
   if (A.nblocks <= 0) return HEC_OK;
-  k_place<<<(unsigned)A.nblocks, kPlaceT, 0, ctx->stream>>>(A);
+  k_place<<<nblk(A.nblocks, kPlaceT / 32), kPlaceT, 0, ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }
@@ -417,9 +410,10 @@ int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide) {
     if (occ[0] < 1) occ[0] = 1;
     if (occ[1] < 1) occ[1] = 1;
   }
-  // persistent: every CTA holding a ticket must be resident (look-back progress)
+  // persistent; the list length is read on the device
   int64_t grid = (int64_t)ctx->num_sms * occ[wide ? 1 : 0];
-  if (A.nblocks < grid) grid = A.nblocks > 0 ? A.nblocks : 1;
+  if (A.nblocks < grid) grid = A.nblocks;
+  if (grid < 1) return HEC_OK;
   if (wide) k_rows<true><<<(unsigned)grid, kT, sizeof(RowsSmemT<true>), ctx->stream>>>(A);
   else k_rows<false><<<(unsigned)grid, kT, sizeof(RowsSmemT<false>), ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();

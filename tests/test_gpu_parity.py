@@ -182,8 +182,9 @@ def test_construct_random_labels(P, ctx):
 
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
 def test_construct_size_classes(P, ctx, nc):
-    """R-MAT s14 with random labels into nc aggregates: few labels give huge rows
-    (DENSE when nc <= 16384, BIN otherwise), many labels give SMALL/MID rows."""
+    """R-MAT with random labels into nc aggregates: few labels give huge rows
+    (DENSE when nc <= 32768, key-range buckets otherwise), many labels give
+    warp-piece and CTA-window rows."""
     rng = np.random.default_rng(15 + nc)
     g = gg.rmat(14 if nc < 20000 else 17, 16)
     g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
@@ -194,6 +195,46 @@ def test_construct_size_classes(P, ctx, nc):
     nc = min(nc, g.n)
     M = rng.integers(0, nc, g.n).astype(np.int32)
     M[rng.permutation(g.n)[:nc]] = np.arange(nc)
+    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+    assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
+
+
+def test_construct_wide_piece_keys(P, ctx, monkeypatch):
+    """The 64-bit (row, b) key path of the warp pieces (used when n_c > 2^26),
+    forced on small graphs through the library's test hook."""
+    monkeypatch.setenv("HEC_FORCE_WIDE_KEYS", "1")
+    rng = np.random.default_rng(21)
+    for t in range(10):
+        g = random_graph(int(rng.integers(2, 300)), rng, p=0.1, wmax=50)
+        nc = int(rng.integers(1, g.n + 1))
+        M = rng.integers(0, nc, g.n).astype(np.int32)
+        M[:nc] = np.arange(nc)
+        cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+        assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
+    check_hierarchy(P, ctx, gg.config(2), 1000)
+
+
+def test_construct_duplicate_heavy_rows(P, ctx):
+    """Skewed rows whose entries repeat few keys: key-range buckets far above a
+    warp piece (CTA tier) and above a CTA block (fallback), next to ordinary rows."""
+    rng = np.random.default_rng(22)
+    n = 60000
+    hub_targets = rng.integers(0, n, 4000)
+    edges = {}
+    for h in range(8):  # 8 hubs, each adjacent to the same 4000 targets
+        for v in hub_targets:
+            if v != h:
+                edges[(min(h, v), max(h, v))] = 1 + (h + int(v)) % 7
+    for _ in range(3 * n):
+        u, v = rng.integers(0, n, 2)
+        if u != v:
+            edges[(min(u, v), max(u, v))] = int(rng.integers(1, 9))
+    g = gg.from_edges(n, [(u, v, w) for (u, v), w in edges.items()])
+    nc = 40000  # > kDenseMax: BUCKET mode
+    M = rng.integers(0, nc, n).astype(np.int32)
+    M[:8] = 0  # all hubs in one coarse row
+    M[hub_targets] = rng.integers(1, 40, hub_targets.size)  # targets collapse onto few keys
+    M[rng.permutation(np.setdiff1d(np.arange(8, n), hub_targets))[:nc]] = np.arange(nc)
     cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
