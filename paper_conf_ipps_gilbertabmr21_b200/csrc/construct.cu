@@ -141,8 +141,12 @@ __global__ void k_big_rows(Layout L, int64_t big_thr, int32_t *__restrict__ big_
   }
 }
 
+constexpr int kPartHist = 8192;  // buckets per skewed row (bounds the partition's smem tables)
+constexpr int kUnit = 65536;     // member-edge positions per partition CTA
+
 __host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c) {
   int64_t nb = (U + kBucketAvg - 1) / kBucketAvg;
+  if (nb > kPartHist) nb = kPartHist;
   if (nb > n_c) nb = n_c;
   return nb < 1 ? 1 : nb;
 }
@@ -189,13 +193,15 @@ __global__ void k_block_ends(int64_t nblocks, int64_t a_hi, BlockDesc *__restric
 }
 
 // ------------------------------------------------------- a9 BUCKET partition
-// Work units: big row h (list index) split into ceil(U/kCap) windows of kCap
-// member-edge positions; unit_ptr = exclusive scan over big rows.
+// Work units: big row h (list index) split into ceil(U/unit) windows of `unit`
+// member-edge positions (kUnit: partition, kCap: dense accumulation);
+// unit_ptr = exclusive scan over big rows.
 struct UnitsIn {
   Layout L;
   const int32_t *big_list;
+  int64_t unit;
   __device__ __forceinline__ int64_t operator()(int64_t h) const {
-    return (L.U(big_list[h]) + kCap - 1) / kCap;
+    return (L.U(big_list[h]) + unit - 1) / unit;
   }
 };
 struct BucketsIn {
@@ -243,83 +249,81 @@ __global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restr
 }
 
 // ------------------------------------------------------- a9 BUCKET partition
-// Work units: big row h (list index) split into ceil(U/kCap) windows of kCap
-// member-edge positions; unit_ptr = exclusive scan over big rows.
-constexpr int kPartHist = 4096;  // buckets of a row counted in smem (more: global atomics)
-
+// One CTA per unit (<= kUnit positions of one skewed row): a shared-memory
+// histogram over the row's key-range buckets (bucket = floor(b * nb / n_c)),
+// flushed once per unit; the write pass reserves each bucket's slice of the unit
+// with one global atomic and scatters with shared-memory cursors, so a bucket
+// receives a contiguous run from every unit.  Offsets inside a row fit int32.
 struct PartSmem {
   int32_t hist[kPartHist];
-  int64_t base[kPartHist];
+  int32_t base[kPartHist];  // slot cursor relative to the row's first bucket
 };
-
-// floor(x / d) for x < 2^62 with a precomputed 64-bit reciprocal rcp = ceil(2^64 / d)
-__device__ __forceinline__ int64_t div_rcp(uint64_t x, uint64_t d, uint64_t rcp) {
-  uint64_t q = __umul64hi(x, rcp);
-  if (q * d > x) --q;
-  else if ((q + 1) * d <= x) ++q;
-  return (int64_t)q;
-}
 
 struct PartArgs {
   Layout L;
   const int32_t *big_list;
   int64_t nbig;
-  const int64_t *unit_ptr;
+  const int64_t *unit_ptr;  // units of kUnit positions
   const int64_t *bkt_ptr;
   const int32_t *Sb, *Sw;   // expanded entries, indexed from upos(a_lo)
-  uint64_t nc_rcp;          // ceil(2^64 / n_c)
 };
 
-// Registers of a unit: bucket (kr) of each entry of big row h, self entries dropped.
-__device__ __forceinline__ void unit_load(const PartArgs &A, int64_t unit, int64_t *h_out, int64_t *nb_out,
-                                          int32_t (&kb)[kIt], int32_t (&kw)[kIt], int32_t (&kr)[kIt]) {
+struct UnitInfo {
+  int64_t p0, p1;  // staging index range of the unit
+  int64_t b0;      // first bucket of the row
+  int32_t a;       // the row
+  int32_t nb;      // buckets of the row
+  float scale;     // nb / n_c
+};
+
+__device__ __forceinline__ UnitInfo unit_info(const PartArgs &A, int64_t unit) {
   const Layout &L = A.L;
   const int64_t h = last_le(A.unit_ptr, 0, A.nbig, unit);
-  const int32_t a = A.big_list[h];
-  const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kCap;
-  const int64_t Pend = L.upos(a + 1);
-  const int64_t nb = A.bkt_ptr[h + 1] - A.bkt_ptr[h];
+  UnitInfo u;
+  u.a = A.big_list[h];
   const int64_t P_lo = L.upos(L.a_lo);
+  const int64_t P0 = L.upos(u.a) + (unit - A.unit_ptr[h]) * kUnit;
+  const int64_t Pe = L.upos(u.a + 1);
+  u.p0 = P0 - P_lo;
+  u.p1 = (P0 + kUnit < Pe ? P0 + kUnit : Pe) - P_lo;
+  u.b0 = A.bkt_ptr[h];
+  u.nb = (int32_t)(A.bkt_ptr[h + 1] - u.b0);
+  u.scale = (float)u.nb / (float)L.n_c;
+  return u;
+}
+
+// bucket of key b: floor(b * nb / n_c) in float arithmetic, clamped.  Any
+// function works as long as it is monotone in b (buckets are key ranges, so the
+// concatenation of sorted buckets is the sorted row) and identical in both passes.
+__device__ __forceinline__ int part_bucket(const UnitInfo &u, int32_t b) {
+  const int k = (int)__fmul_rz((float)b, u.scale);
+  return k < u.nb - 1 ? k : u.nb - 1;
+}
+
+constexpr int kPartU = 8;  // loads in flight per thread in the partition passes
+
+// histogram of the unit's entries (self entries dropped) into S.hist
+__device__ __forceinline__ void unit_hist(const PartArgs &A, const UnitInfo &u, PartSmem &S) {
+  for (int i = threadIdx.x; i < u.nb; i += kT) S.hist[i] = 0;
+  __syncthreads();
+  for (int64_t p = u.p0 + threadIdx.x; p < u.p1; p += kPartU * kT) {
+    int32_t b[kPartU];
 #pragma unroll
-  for (int k = 0; k < kIt; ++k) {
-    const int64_t p = P0 + threadIdx.x + (int64_t)kT * k;
-    kb[k] = -1;
-    kw[k] = 0;
-    kr[k] = 0;
-    if (p < Pend) {
-      const int32_t b = A.Sb[p - P_lo];
-      if (b != a) {
-        kb[k] = b;
-        kw[k] = A.Sw[p - P_lo];
-        kr[k] = (int32_t)div_rcp((uint64_t)b * (uint64_t)nb, (uint64_t)L.n_c, A.nc_rcp);
-      }
-    }
+    for (int j = 0; j < kPartU; ++j) b[j] = p + j * kT < u.p1 ? __ldcs(A.Sb + p + j * kT) : u.a;
+#pragma unroll
+    for (int j = 0; j < kPartU; ++j)
+      if (b[j] != u.a) atomicAdd(&S.hist[part_bucket(u, b[j])], 1);
   }
-  *h_out = h;
-  *nb_out = nb;
+  __syncthreads();
 }
 
 __global__ void __launch_bounds__(kT) k_part_count(PartArgs A, unsigned *__restrict__ bkt_cnt) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
-  int32_t kb[kIt], kw[kIt], kr[kIt];
-  int64_t h, nb;
-  unit_load(A, blockIdx.x, &h, &nb, kb, kw, kr);
-  const bool sh = nb <= kPartHist;
-  if (sh)
-    for (int i = threadIdx.x; i < nb; i += kT) S.hist[i] = 0;
-  __syncthreads();
-  const int64_t b0 = A.bkt_ptr[h];
-#pragma unroll
-  for (int k = 0; k < kIt; ++k)
-    if (kb[k] >= 0) {
-      if (sh) atomicAdd(&S.hist[kr[k]], 1);
-      else atomicAdd(bkt_cnt + b0 + kr[k], 1u);
-    }
-  __syncthreads();
-  if (sh)
-    for (int i = threadIdx.x; i < nb; i += kT)
-      if (S.hist[i]) atomicAdd(bkt_cnt + b0 + i, (unsigned)S.hist[i]);
+  const UnitInfo u = unit_info(A, blockIdx.x);
+  unit_hist(A, u, S);
+  for (int i = threadIdx.x; i < u.nb; i += kT)
+    if (S.hist[i]) atomicAdd(bkt_cnt + u.b0 + i, (unsigned)S.hist[i]);
 }
 
 __global__ void __launch_bounds__(kT) k_part_write(PartArgs A, const int64_t *__restrict__ bkt_off,
@@ -327,36 +331,28 @@ __global__ void __launch_bounds__(kT) k_part_write(PartArgs A, const int64_t *__
                                                    int32_t *__restrict__ pw) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
-  int32_t kb[kIt], kw[kIt], kr[kIt];
-  int64_t h, nb;
-  unit_load(A, blockIdx.x, &h, &nb, kb, kw, kr);
-  const int64_t b0 = A.bkt_ptr[h];
-  if (nb <= kPartHist) {
-    for (int i = threadIdx.x; i < nb; i += kT) S.hist[i] = 0;
-    __syncthreads();
-    int rank[kIt];
+  const UnitInfo u = unit_info(A, blockIdx.x);
+  unit_hist(A, u, S);
+  const int64_t off0 = bkt_off[u.b0];
+  for (int i = threadIdx.x; i < u.nb; i += kT) {
+    const int c = S.hist[i];
+    if (c) S.base[i] = (int32_t)(bkt_off[u.b0 + i] - off0) + (int32_t)atomicAdd(bkt_cur + u.b0 + i, (unsigned)c);
+  }
+  __syncthreads();
+  for (int64_t p = u.p0 + threadIdx.x; p < u.p1; p += kPartU * kT) {
+    int32_t b[kPartU], w[kPartU];
 #pragma unroll
-    for (int k = 0; k < kIt; ++k) rank[k] = kb[k] >= 0 ? atomicAdd(&S.hist[kr[k]], 1) : 0;
-    __syncthreads();
-    for (int i = threadIdx.x; i < nb; i += kT) {
-      int c = S.hist[i];
-      S.base[i] = c ? bkt_off[b0 + i] + atomicAdd(bkt_cur + b0 + i, (unsigned)c) : 0;
+    for (int j = 0; j < kPartU; ++j) {
+      const bool in = p + j * kT < u.p1;
+      b[j] = in ? __ldcs(A.Sb + p + j * kT) : u.a;
+      w[j] = in ? __ldcs(A.Sw + p + j * kT) : 0;
     }
-    __syncthreads();
 #pragma unroll
-    for (int k = 0; k < kIt; ++k)
-      if (kb[k] >= 0) {
-        int64_t q = S.base[kr[k]] + rank[k];
-        pb[q] = kb[k];
-        pw[q] = kw[k];
-      }
-  } else {
-#pragma unroll
-    for (int k = 0; k < kIt; ++k)
-      if (kb[k] >= 0) {
-        int64_t q = bkt_off[b0 + kr[k]] + atomicAdd(bkt_cur + b0 + kr[k], 1u);
-        pb[q] = kb[k];
-        pw[q] = kw[k];
+    for (int j = 0; j < kPartU; ++j)
+      if (b[j] != u.a) {
+        const int64_t q = off0 + atomicAdd(&S.base[part_bucket(u, b[j])], 1);
+        pb[q] = b[j];
+        pw[q] = w[j];
       }
   }
 }
@@ -367,6 +363,7 @@ struct FbSmem {
   int32_t key[kFbTab];
   unsigned long long val[kFbTab];
   unsigned nkeys, nout;
+  int32_t kmin, kmax;
   int64_t job;
 };
 
@@ -392,8 +389,7 @@ __device__ void block_bitonic(int32_t *key, V *val, int N) {
   }
 }
 
-__global__ void __launch_bounds__(kT) k_bucket_fallback(int64_t n_c, const int64_t *__restrict__ jobs, int64_t njobs,
-                                                        const int32_t *__restrict__ job_rn,  // (sub, nb) per job
+__global__ void __launch_bounds__(kT) k_bucket_fallback(const int64_t *__restrict__ jobs, int64_t njobs,
                                                         const int64_t *__restrict__ bkt_off,
                                                         const int32_t *__restrict__ pb, const int32_t *__restrict__ pw,
                                                         const int64_t *__restrict__ fb_off, int32_t *__restrict__ fb_cnt,
@@ -408,8 +404,21 @@ __global__ void __launch_bounds__(kT) k_bucket_fallback(int64_t n_c, const int64
     if (j >= njobs) return;
     const int64_t bk = jobs[j];
     const int64_t q0 = bkt_off[bk], q1 = bkt_off[bk + 1];
-    int32_t lo, hi;
-    bucket_range(job_rn[2 * j], job_rn[2 * j + 1], n_c, &lo, &hi);
+    // key range of the bucket's entries (sub-ranges split it when a pass overflows)
+    if (threadIdx.x == 0) { S.kmin = INT32_MAX; S.kmax = -1; }
+    __syncthreads();
+    {
+      int32_t mn = INT32_MAX, mx = -1;
+      for (int64_t q = q0 + threadIdx.x; q < q1; q += kT) {
+        const int32_t b = pb[q];
+        mn = min(mn, b);
+        mx = max(mx, b);
+      }
+      atomicMin(&S.kmin, mn);
+      atomicMax(&S.kmax, mx);
+    }
+    __syncthreads();
+    const int32_t lo = S.kmin, hi = S.kmax + 1;
     const int64_t out = fb_off[bk];
     int64_t written = 0;
     int nsub = 1, sub = 0;
@@ -484,21 +493,19 @@ __global__ void __launch_bounds__(kT) k_bucket_fallback(int64_t n_c, const int64
 __global__ void k_bucket_blocks(int64_t nbig, int64_t nbkt, const int32_t *__restrict__ big_list,
                                 const int64_t *__restrict__ bkt_ptr, const int64_t *__restrict__ bkt_off,
                                 const int64_t *__restrict__ blk_ptr, BlockDesc *__restrict__ blk,
-                                int64_t *__restrict__ jobs, int32_t *__restrict__ job_rn, unsigned *__restrict__ njobs,
+                                int64_t *__restrict__ jobs, unsigned *__restrict__ njobs,
                                 int32_t *__restrict__ fb_cnt, int64_t *__restrict__ fb_off,
                                 unsigned long long *__restrict__ fb_total) {
   int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= nbkt) return;
   const int64_t h = last_le(bkt_ptr, 0, nbig, k);
-  const int64_t b0 = bkt_ptr[h], b1 = bkt_ptr[h + 1];
+  const int64_t b0 = bkt_ptr[h];
   const int32_t a = big_list[h];
   blk[blk_ptr[a] + (k - b0)] = BlockDesc{B_BUCKET, a, a + 1, (int32_t)(k - b0)};
   const int64_t c = bkt_off[k + 1] - bkt_off[k];
   if (c > kCap) {
     unsigned j = atomicAdd(njobs, 1u);
     jobs[j] = k;
-    job_rn[2 * j] = (int32_t)(k - b0);
-    job_rn[2 * j + 1] = (int32_t)(b1 - b0);
     fb_off[k] = (int64_t)atomicAdd(fb_total, (unsigned long long)c);
     fb_cnt[k] = 0;
   } else {
@@ -722,7 +729,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t small_vol = r0[1], big_vol = r0[2];
   const int64_t nbig = r0[4] & 0xffffffffLL;
   if (nbig > 0) {
-    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list}, PtrOut{unit_ptr}, st[4], unit_ptr + nbig));
+    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)kCap : (int64_t)kUnit}, PtrOut{unit_ptr},
+                         st[4], unit_ptr + nbig));
     if (!dense) HEC_TRY(chained_scan(ctx, nbig, BucketsIn{L, big_list}, PtrOut{bkt_ptr}, st[5], bkt_ptr + nbig));
     HEC_CUDA_TRY(cudaMemcpyAsync(scal + 5, unit_ptr + nbig, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
     if (!dense) HEC_CUDA_TRY(cudaMemcpyAsync(scal + 6, bkt_ptr + nbig, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
@@ -828,21 +836,19 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     int32_t *pw = arena_take<int32_t>(W2, (size_t)big_vol + 1);
     ScanTiles stb = take_scan_tiles(W2, nbkt);
     int64_t *jobs = arena_take<int64_t>(W2, nbkt + 1);
-    int32_t *job_rn = arena_take<int32_t>(W2, 2 * nbkt + 2);
     int32_t *fb_b = arena_take<int32_t>(W2, (size_t)big_vol + 1);
     int32_t *fb_w = arena_take<int32_t>(W2, (size_t)big_vol + 1);
     if (!fb_w) { set_error("workspace under-reserved (buckets)"); return HEC_EINVAL; }
     HEC_CUDA_TRY(cudaMemsetAsync(bkt_cnt, 0, sizeof(unsigned) * (nbkt + 1), s));
     HEC_CUDA_TRY(cudaMemsetAsync(bkt_cur, 0, sizeof(unsigned) * (nbkt + 1), s));
-    PartArgs PA{L, big_list, nbig, unit_ptr, bkt_ptr, sc_col, sc_wgt,
-                (uint64_t)(~0ull / (uint64_t)n_c) + 1};  // ceil(2^64 / n_c), n_c > 32768 here
+    PartArgs PA{L, big_list, nbig, unit_ptr, bkt_ptr, sc_col, sc_wgt};
     k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt);
     HEC_LAUNCH_CHECK();
     HEC_TRY(chained_scan(ctx, nbkt, CountIn{bkt_cnt}, PtrOut{bkt_off}, stb, bkt_off + nbkt));
     k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, bkt_cur, pb, pw);
     HEC_LAUNCH_CHECK();
     k_bucket_blocks<<<nblk(nbkt, 256), 256, 0, s>>>(nbig, nbkt, big_list, bkt_ptr, bkt_off, blk_ptr, blk, jobs,
-                                                   job_rn, counts + 4, fb_cnt, fb_off,
+                                                   counts + 4, fb_cnt, fb_off,
                                                    reinterpret_cast<unsigned long long *>(scal + 10));
     HEC_LAUNCH_CHECK();
     HEC_CUDA_TRY(cudaMemcpyAsync(scal + 9, counts + 4, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
@@ -850,7 +856,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_TRY(read_scalars(ctx, scal + 9, 1, rj));
     const int64_t njobs = rj[0] & 0xffffffffLL;
     if (njobs > 0) {
-      k_bucket_fallback<<<ctx->num_sms, kT, sizeof(FbSmem), s>>>(n_c, jobs, njobs, job_rn, bkt_off, pb, pw, fb_off,
+      k_bucket_fallback<<<ctx->num_sms, kT, sizeof(FbSmem), s>>>(jobs, njobs, bkt_off, pb, pw, fb_off,
                                                                 fb_cnt, fb_b, fb_w, counts + 3, err);
       HEC_LAUNCH_CHECK();
     }

@@ -114,14 +114,17 @@ struct Layout {
 struct WarpExpTab {
   int64_t mp[129];  // member-edge start of members i0 .. i0+128 (mpre)
   int64_t ms[128];  // row_ptr[members[i]] (mstart)
+  int32_t mk[128];  // position -> member (relative to i0)
 };
 
 // One warp expands the member-edge positions [P, limit) with limit <=
 // min(P + 128, Pend, start of member i0 + 128) into registers: slot t of lane l
 // is position P + l + 32 t; b = -1 marks empty slots.  Members are [i0, mend)
 // with i0 the member containing P; on return i0 is the member containing limit.
-// mem[t] receives the member index of the slot.  Only __syncwarp is used, so
-// warps of a CTA proceed independently.  Returns limit - P.
+// mem[t] receives the member index of the slot.  Positions find their member by
+// a mark + warp max-scan (each non-empty member marks its first position).
+// Only __syncwarp is used, so warps of a CTA proceed independently.
+// Returns limit - P.
 __device__ __forceinline__ int warp_expand(const Layout &L, const int64_t *__restrict__ mstart, int64_t mend,
                                            int64_t P, int64_t Pend, int64_t &i0, WarpExpTab &W,
                                            int32_t (&b)[4], int32_t (&w)[4], int64_t (&mem)[4]) {
@@ -132,22 +135,50 @@ __device__ __forceinline__ int warp_expand(const Layout &L, const int64_t *__res
     const int64_t j = i0 + lane + 32 * t;
     W.mp[lane + 32 * t] = j < mend ? L.mpre[j] : pend_m;
     W.ms[lane + 32 * t] = j < mend ? mstart[j] : 0;
+    W.mk[lane + 32 * t] = -1;
   }
   if (lane == 0) W.mp[128] = (i0 + 128 < mend) ? L.mpre[i0 + 128] : pend_m;
   __syncwarp();
   int64_t limit = P + 128;
   if (Pend < limit) limit = Pend;
   if (W.mp[128] < limit) limit = W.mp[128];
+  const int n = (int)(limit - P);
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {  // member k starts inside the window and is non-empty
+    const int k = lane + 32 * t;
+    const int64_t rs = W.mp[k] - P;
+    if (rs >= 0 && rs < n && W.mp[k + 1] > W.mp[k]) W.mk[rs] = k;
+  }
+  __syncwarp();
+  // inclusive max-scan over positions (blocked: lane owns 4 consecutive ones)
+  int m[4], run = 0;  // position 0 lies in member 0 (i0 contains P)
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    run = max(run, W.mk[4 * lane + t]);
+    m[t] = run;
+  }
+  int x = run;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x = max(x, y);
+  }
+  int before = __shfl_up_sync(0xffffffffu, x, 1);
+  if (lane == 0) before = 0;
+  __syncwarp();
+#pragma unroll
+  for (int t = 0; t < 4; ++t) W.mk[4 * lane + t] = max(before, m[t]);
+  __syncwarp();
   int64_t e[4];
   unsigned valid = 0;
 #pragma unroll
   for (int t = 0; t < 4; ++t) {
-    const int64_t q = P + lane + 32 * t;
+    const int r = lane + 32 * t;
     b[t] = -1;
     w[t] = 0;
-    if (q < limit) {
-      const int k = (int)last_le(W.mp, 0, 128, q);
-      e[t] = W.ms[k] + (q - W.mp[k]);
+    if (r < n) {
+      const int k = W.mk[r];
+      e[t] = W.ms[k] + (P + r - W.mp[k]);
       mem[t] = i0 + k;
       valid |= 1u << t;
     }
@@ -160,7 +191,7 @@ __device__ __forceinline__ int warp_expand(const Layout &L, const int64_t *__res
     if (valid & (1u << t)) b[t] = __ldg(L.M + b[t]);
   i0 += last_le(W.mp, 0, 129, limit);
   __syncwarp();
-  return (int)(limit - P);
+  return n;
 }
 
 // Largest member i in [lo, hi) with mpre[i] <= P (mpre[lo] <= P), by a warp:
@@ -225,14 +256,6 @@ struct RowsArgs {
   const int32_t *list;    // blocks of this launch (a tier list)
   const unsigned *nlist;  // device count of `list`
 };
-
-// keys b with floor(b * nb / n_c) == k: [ceil(k n_c / nb), ceil((k+1) n_c / nb))
-__host__ __device__ __forceinline__ void bucket_range(int64_t k, int64_t nb, int64_t n_c, int32_t *lo,
-                                                      int32_t *hi) {
-  *lo = (int32_t)((k * n_c + nb - 1) / nb);
-  int64_t h = ((k + 1) * n_c + nb - 1) / nb;
-  *hi = (int32_t)(h < n_c ? h : n_c);
-}
 
 // Work-block kernel and placement launchers (construct_rows.cu).
 // Work-block kernels take their blocks from A.list / *A.nlist (device count).

@@ -49,48 +49,75 @@ __device__ __forceinline__ uint64_t shfl_up_k(uint64_t v, int d) { return __shfl
 __device__ __forceinline__ uint32_t shfl_down_k(uint32_t v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
 __device__ __forceinline__ uint64_t shfl_down_k(uint64_t v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
 
+// Exchange step between lanes (partner lane ^ lm, same register): keep the min
+// (f = 0) or the max (f = ~0, comparing complemented keys).  Branch-free: a
+// select here compiles to a divergent branch.
+template <int J, typename K>
+__device__ __forceinline__ void bitonic_lanes(K (&key)[J], int32_t (&val)[J], int lm, bool keep_min) {
+  const K f = keep_min ? (K)0 : ~(K)0;
+#pragma unroll
+  for (int k = 0; k < J; ++k) {
+    const K pk = shfl_xor_k(key[k], lm);
+    const int32_t pv = __shfl_xor_sync(0xffffffffu, val[k], lm);
+    const bool take = (pk ^ f) < (key[k] ^ f);
+    key[k] ^= (key[k] ^ pk) & ((K)0 - (K)take);
+    val[k] ^= (val[k] ^ pv) & (int32_t)(0u - (uint32_t)take);
+  }
+}
+
+// Exchange step inside a lane: registers k, k | STRIDE; `asc_of(k)` gives the direction.
+template <int J, int STRIDE, typename K, typename AscFn>
+__device__ __forceinline__ void bitonic_regs(K (&key)[J], int32_t (&val)[J], AscFn asc_of) {
+#pragma unroll
+  for (int k = 0; k < J; ++k) {
+    if (k & STRIDE) continue;
+    const int k2 = k | STRIDE;
+    const K f = asc_of(k) ? (K)0 : ~(K)0;
+    const bool sw = (key[k2] ^ f) < (key[k] ^ f);
+    const K dk = (key[k] ^ key[k2]) & ((K)0 - (K)sw);
+    const int32_t dv = (val[k] ^ val[k2]) & (int32_t)(0u - (uint32_t)sw);
+    key[k] ^= dk;
+    key[k2] ^= dk;
+    val[k] ^= dv;
+    val[k2] ^= dv;
+  }
+}
+
+// All in-lane strides J/2 .. 1 of a merge step whose direction is uniform per lane.
+template <int J, typename K>
+__device__ __forceinline__ void bitonic_regs_all(K (&key)[J], int32_t (&val)[J], bool asc) {
+  auto f = [asc](int) { return asc; };
+  if (J >= 16) bitonic_regs<J, (J >= 16 ? 8 : 1)>(key, val, f);
+  if (J >= 8) bitonic_regs<J, (J >= 8 ? 4 : 1)>(key, val, f);
+  if (J >= 4) bitonic_regs<J, (J >= 4 ? 2 : 1)>(key, val, f);
+  bitonic_regs<J, 1>(key, val, f);
+}
+
 // Ascending bitonic sort of the 32*J (key, val) pairs of a warp; element
-// i = lane*J + k on return (blocked).  Input order is arbitrary.
+// i = lane*J + k on return (blocked).  Input order is arbitrary.  Sizes up to J
+// are unrolled (in-lane); larger sizes run as a compact runtime loop so the
+// three piece sizes share little code (the unrolled network overflowed the
+// instruction cache).
 template <int J, typename K>
 __device__ __forceinline__ void warp_bitonic(K (&key)[J], int32_t (&val)[J]) {
   const int lane = threadIdx.x & 31;
+  // sizes 2 .. J/2: inside each lane; direction from bit `size` of k
 #pragma unroll
-  for (int size = 2; size <= 32 * J; size <<= 1) {
-#pragma unroll
-    for (int stride = size >> 1; stride > 0; stride >>= 1) {
-      if (stride >= J) {  // partner in lane ^ (stride / J), same register
-        const int lm = stride / J;
-        const bool upper = (lane & lm) != 0;
-        const bool asc = (lane & (size / J)) == 0;  // bit `size` of i = lane*J + k
-        // keep the min (f = 0) or the max (f = ~0: compare complemented keys)
-        const K f = (upper != asc) ? (K)0 : ~(K)0;
-#pragma unroll
-        for (int k = 0; k < J; ++k) {
-          const K pk = shfl_xor_k(key[k], lm);
-          const int32_t pv = __shfl_xor_sync(0xffffffffu, val[k], lm);
-          const bool take = (pk ^ f) < (key[k] ^ f);
-          // branch-free exchange (a select here compiles to a divergent branch)
-          const K tm = (K)0 - (K)take;
-          key[k] ^= (key[k] ^ pk) & tm;
-          val[k] ^= (val[k] ^ pv) & (int32_t)(0u - (uint32_t)take);
-        }
-      } else {  // partner in the same lane: registers k, k | stride
-#pragma unroll
-        for (int k = 0; k < J; ++k) {
-          if (k & stride) continue;
-          const int k2 = k | stride;
-          const bool asc = size < J ? (k & size) == 0 : (lane & (size / J)) == 0;
-          const K f = asc ? (K)0 : ~(K)0;
-          const bool sw = (key[k2] ^ f) < (key[k] ^ f);
-          const K dk = (key[k] ^ key[k2]) & ((K)0 - (K)sw);
-          const int32_t dv = (val[k] ^ val[k2]) & (int32_t)(0u - (uint32_t)sw);
-          key[k] ^= dk;
-          key[k2] ^= dk;
-          val[k] ^= dv;
-          val[k2] ^= dv;
-        }
-      }
-    }
+  for (int size = 2; size < J; size <<= 1) {
+    auto asc_of = [size](int k) { return (k & size) == 0; };
+    if (size >= 16) bitonic_regs<J, (J >= 16 ? 8 : 1)>(key, val, asc_of);
+    if (size >= 8) bitonic_regs<J, (J >= 8 ? 4 : 1)>(key, val, asc_of);
+    if (size >= 4) bitonic_regs<J, (J >= 4 ? 2 : 1)>(key, val, asc_of);
+    bitonic_regs<J, 1>(key, val, asc_of);
+  }
+  // sizes J .. 32J: strides >= J across lanes, then the in-lane strides; the
+  // direction (bit `size` of i = lane*J + k) comes from the lane
+#pragma unroll 1
+  for (int sz = 1; sz <= 32; sz <<= 1) {  // size = sz * J
+    const bool asc = (lane & sz) == 0;
+#pragma unroll 1
+    for (int lm = sz >> 1; lm > 0; lm >>= 1) bitonic_lanes<J, K>(key, val, lm, ((lane & lm) != 0) != asc);
+    bitonic_regs_all<J, K>(key, val, asc);
   }
 }
 
@@ -202,10 +229,10 @@ __device__ __forceinline__ int piece_run(int32_t row0, PieceTab &S, int R, int n
   return piece_sort_merge<J, K>(key, val, S, src_b, src_w, base, R, row_ptr_rel);
 }
 
-template <int J>
-__device__ __forceinline__ int piece_dispatch(bool wide_keys, int32_t row0, PieceTab &S, int R, int n,
-                                              int32_t *src_b, int32_t *src_w, int64_t base, int64_t *rp) {
-  if (R > 0 && wide_keys) return piece_run<J, uint64_t>(row0, S, R, n, src_b, src_w, base, rp);
+template <int J, bool WIDE_KEYS>
+__device__ __forceinline__ int piece_dispatch(int32_t row0, PieceTab &S, int R, int n, int32_t *src_b,
+                                              int32_t *src_w, int64_t base, int64_t *rp) {
+  if (WIDE_KEYS && R > 0) return piece_run<J, uint64_t>(row0, S, R, n, src_b, src_w, base, rp);
   return piece_run<J, uint32_t>(row0, S, R, n, src_b, src_w, base, rp);
 }
 
@@ -247,9 +274,9 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
       src_w = A.pw_g;
     }
     int T;
-    if (n <= 64) T = piece_dispatch<2>(WIDE_KEYS, d.row0, S, R, n, src_b, src_w, base, rp);
-    else if (n <= 128) T = piece_dispatch<4>(WIDE_KEYS, d.row0, S, R, n, src_b, src_w, base, rp);
-    else T = piece_dispatch<8>(WIDE_KEYS, d.row0, S, R, n, src_b, src_w, base, rp);
+    if (n <= 64) T = piece_dispatch<2, WIDE_KEYS>(d.row0, S, R, n, src_b, src_w, base, rp);
+    else if (n <= 128) T = piece_dispatch<4, WIDE_KEYS>(d.row0, S, R, n, src_b, src_w, base, rp);
+    else T = piece_dispatch<8, WIDE_KEYS>(d.row0, S, R, n, src_b, src_w, base, rp);
     if (T < 0) {
       if (lane == 0) {
         A.need_wide[bi] = 1;
