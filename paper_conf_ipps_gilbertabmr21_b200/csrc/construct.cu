@@ -513,26 +513,57 @@ __global__ void k_bucket_blocks(int64_t nbig, int64_t nbkt, const int32_t *__res
   }
 }
 
-// Tier lists: warp pieces (PIECE blocks, buckets of <= kPieceCap entries) and
-// CTA blocks (SMALL, DENSE, larger buckets).  Fallback buckets are complete:
-// their count is final here.  list_n: [0] warp list, [1] CTA list.
-__global__ void k_tiers(int64_t nblocks, const BlockDesc *__restrict__ blk, const int32_t *__restrict__ big_idx,
+// Bin groups: consecutive bins of a skewed row form one piece while they start
+// inside one window of kGroupWin entries (so a group of bins <= kGroupWin each
+// holds < 2 kGroupWin entries); a bin above kGroupWin stands alone.  The group's
+// first bin carries its block (count, staging at its first pair); the other
+// bins' blocks are empty.
+__device__ __forceinline__ bool group_start(const int64_t *__restrict__ bkt_off, int64_t b0, int64_t k) {
+  if (k == b0) return true;
+  const int64_t ck = bkt_off[k + 1] - bkt_off[k], cp = bkt_off[k] - bkt_off[k - 1];
+  if (ck > kGroupWin || cp > kGroupWin) return true;
+  return (bkt_off[k] - bkt_off[b0]) / kGroupWin != (bkt_off[k - 1] - bkt_off[b0]) / kGroupWin;
+}
+
+// Tier lists: warp pieces (PIECE blocks, bin groups of <= kPieceCap entries) and
+// CTA blocks (SMALL, DENSE, larger bins).  Fallback bins are complete: their
+// count is final here.  list_n: [0] warp list, [1] CTA list.
+__global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__ blk, const int32_t *__restrict__ big_idx,
                         const int64_t *__restrict__ bkt_ptr, const int64_t *__restrict__ bkt_off,
                         const int32_t *__restrict__ fb_cnt, int32_t *__restrict__ blk_cnt,
-                        int32_t *__restrict__ list_w, int32_t *__restrict__ list_c, unsigned *__restrict__ list_n,
+                        int64_t *__restrict__ grp_end,
+                        WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, unsigned *__restrict__ list_n,
                         const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
   const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   int tier = -1;  // 0 warp, 1 CTA
+  WorkItem it{0, (int32_t)bi, 0, 0, 0};
   if (bi < nblocks) {
     const BlockDesc d = blk[bi];
+    it.row0 = d.row0;
     // vertex weight of a skewed row (written by k_place): int32 bound
     if (!rows_kind(d.kind) && d.sub == 0 && vw64[d.row0] > 0x7fffffffull) atomicOr(err, ERR_OVERFLOW);
-    if (d.kind == B_PIECE) tier = 0;
-    else if (d.kind != B_BUCKET) tier = 1;
+    if (d.kind == B_PIECE) {
+      tier = 0;
+      const int64_t p0 = L.upos(d.row0);
+      it.base = p0 - L.upos(L.a_lo);
+      it.n = (int32_t)(L.upos(d.row1) - p0);
+      it.R = d.row1 - d.row0;
+    } else if (d.kind != B_BUCKET) tier = 1;
     else {
-      const int64_t bk = bkt_ptr[big_idx[d.row0]] + d.sub;
-      if (fb_cnt[bk] >= 0) blk_cnt[bi] = fb_cnt[bk];
-      else tier = (bkt_off[bk + 1] - bkt_off[bk] <= kPieceCap) ? 0 : 1;
+      const int64_t h = big_idx[d.row0];
+      const int64_t b0 = bkt_ptr[h], b1 = bkt_ptr[h + 1], bk = b0 + d.sub;
+      if (fb_cnt[bk] >= 0) {
+        blk_cnt[bi] = fb_cnt[bk];
+      } else if (!group_start(bkt_off, b0, bk)) {
+        blk_cnt[bi] = 0;
+      } else {
+        int64_t e = bk + 1;
+        while (e < b1 && !group_start(bkt_off, b0, e)) ++e;
+        grp_end[bi] = e;
+        it.base = bkt_off[bk];
+        it.n = (int32_t)(bkt_off[e] - bkt_off[bk]);
+        tier = it.n <= kPieceCap ? 0 : 1;
+      }
     }
   }
   const int lane = threadIdx.x & 31;
@@ -544,7 +575,11 @@ __global__ void k_tiers(int64_t nblocks, const BlockDesc *__restrict__ blk, cons
     unsigned base = 0;
     if (lane == leader) base = atomicAdd(list_n + q, (unsigned)__popc(m));
     base = __shfl_sync(0xffffffffu, base, leader);
-    if (tier == q) (q ? list_c : list_w)[base + __popc(m & ((1u << lane) - 1))] = (int32_t)bi;
+    if (tier == q) {
+      const unsigned pos = base + __popc(m & ((1u << lane) - 1));
+      if (q) list_c[pos] = (int32_t)bi;
+      else list_w[pos] = it;
+    }
   }
 }
 
@@ -744,7 +779,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
 
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
-    size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 5 * ws_bytes(nblocks + 1, 4) +
+    size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
+                ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
     if (nbig > 0 && dense) b2 += ws_bytes((size_t)nbig * n_c, 8);
@@ -760,9 +796,10 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   BlockDesc *blk = arena_take<BlockDesc>(W2, nblocks + 1);
   int32_t *blk_cnt = arena_take<int32_t>(W2, nblocks + 1);
   int32_t *need_wide = arena_take<int32_t>(W2, nblocks + 1);
-  int32_t *list_w = arena_take<int32_t>(W2, nblocks + 1);     // warp-tier blocks
+  WorkItem *list_w = arena_take<WorkItem>(W2, nblocks + 1);   // warp-tier work items
   int32_t *list_c = arena_take<int32_t>(W2, nblocks + 1);     // CTA-tier blocks
   int32_t *list_wide = arena_take<int32_t>(W2, nblocks + 1);  // blocks flagged for 64-bit sums
+  int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
   // expanded (b, w) of every active member-edge position; SMALL blocks stage
@@ -799,6 +836,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   A.vw64 = vw64;
   A.big_idx = big_idx;
   A.bkt_ptr = bkt_ptr;
+  A.grp_end = grp_end;
   A.err = err;
 
   static bool attr = false;
@@ -873,7 +911,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (nblocks > 0) {
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
-    k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.fb_cnt, blk_cnt, list_w,
+    k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.fb_cnt, blk_cnt, grp_end, list_w,
                                               list_c, counts + 6, vw64, err);
     HEC_LAUNCH_CHECK();
   }
@@ -890,7 +928,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.trace = trace;
   }
   const int ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
-  A.list = list_w;
+  A.items = list_w;
   A.nlist = counts + 6;
   HEC_TRY(launch_pieces(ctx, A, counts + 5));
   A.list = list_c;

@@ -15,7 +15,8 @@ constexpr int kRowW = 8;           // per-row weight: bounds rows per block
 constexpr int kMaxRows = 2 * kWin / kRowW;  // 512
 constexpr int kSmallMax = kWin - kRowW;     // rows with U <= 2040 are small
 constexpr int kMC = 1024;          // member-table chunk
-constexpr int kBucketAvg = 128;    // target entries per BUCKET (one warp piece)
+constexpr int kBucketAvg = 32;     // target entries per key-range bin of a skewed row
+constexpr int kGroupWin = 128;     // bins are grouped into pieces by windows of this weight
 constexpr int kPieceMax = 124;     // rows with U <= kPieceMax go to warp pieces
 constexpr int kPieceWin = 128;     // piece window weight (piece weight < 2*kPieceWin)
 constexpr int kPieceRowW = 4;      // per-row piece weight
@@ -212,6 +213,17 @@ __device__ __forceinline__ int64_t warp_find_member(const Layout &L, int64_t lo,
   return lo + __popc(__ballot_sync(0xffffffffu, le)) - 1;
 }
 
+// A warp-tier work item, self-contained so a warp goes straight to its data:
+// entries [base, base + n) of the staging (PIECE: sc_col/sc_wgt) or of the
+// partitioned pairs (bin group: pb_g/pw_g); R > 0 rows starting at row0.
+struct WorkItem {
+  int64_t base;
+  int32_t bi;  // block index (count, flags)
+  int32_t n;
+  int32_t row0;
+  int32_t R;
+};
+
 struct BlockDesc {
   int32_t kind;
   int32_t row0;  // first row (SMALL) / the row (BUCKET, DENSE)
@@ -242,6 +254,7 @@ struct RowsArgs {
   // BUCKET mode
   const int64_t *bkt_ptr;           // [nbig+1] first bucket of big row h
   const int64_t *bkt_off;           // [nbkt+1] pair offsets
+  const int64_t *grp_end;           // [nblocks] BUCKET group: one past its last bin (k_tiers)
   int32_t *pb_g, *pw_g;             // partitioned pairs (sorted uniques written back in place)
   const int32_t *fb_cnt;            // fallback unique count per bucket (-1: not overflowed)
   const int64_t *fb_off;            // fallback scratch offset per bucket
@@ -254,7 +267,8 @@ struct RowsArgs {
   int *err;
   long long *trace;  // debug: per block (compute cycles, 0, kind, T); nullable
   const int32_t *list;    // blocks of this launch (a tier list)
-  const unsigned *nlist;  // device count of `list`
+  const WorkItem *items;  // warp tier: the same, as work items
+  const unsigned *nlist;  // device count of `list` / `items`
 };
 
 // Work-block kernel and placement launchers (construct_rows.cu).

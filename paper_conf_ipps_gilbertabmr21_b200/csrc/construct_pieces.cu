@@ -244,39 +244,37 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
   const Layout &L = A.L;
   const int64_t P_lo = L.upos(L.a_lo);
   const int64_t nlist = *A.nlist;
+  constexpr int kBatch = 4;  // items per ticket (one global atomic per 4 pieces)
+  int64_t item = 0, item_end = 0;
   while (true) {
-    int64_t item = 0;
-    if (lane == 0) item = (int64_t)atomicAdd(ticket, 1u);
-    item = __shfl_sync(0xffffffffu, item, 0);
-    if (item >= nlist) return;
-    const int64_t bi = A.list[item];
-    const BlockDesc d = A.blk[bi];
-    int R, n;
-    int64_t base;  // where the piece's entries are read and its result is staged
+    if (item == item_end) {
+      int64_t t = 0;
+      if (lane == 0) t = (int64_t)atomicAdd(ticket, (unsigned)kBatch);
+      item = __shfl_sync(0xffffffffu, t, 0) ;
+      item_end = item + kBatch < nlist ? item + kBatch : nlist;
+      if (item >= nlist) return;
+    }
+    const WorkItem wi = A.items[item++];
+    const int64_t bi = wi.bi;
+    const int R = wi.R, n = wi.n;
+    const int64_t base = wi.base;  // where the piece's entries are read and its result is staged
     int32_t *src_b, *src_w;
     int64_t *rp = nullptr;
-    if (d.kind == B_PIECE) {
-      R = d.row1 - d.row0;
-      const int64_t P0 = L.upos(d.row0);
-      for (int r = lane; r <= R; r += 32) S.rstart[r] = (int32_t)(L.upos(d.row0 + r) - P0);
+    if (R > 0) {  // PIECE: rows row0 .. row0 + R
+      const int64_t P0 = L.upos(wi.row0);
+      for (int r = lane; r <= R; r += 32) S.rstart[r] = (int32_t)(L.upos(wi.row0 + r) - P0);
       __syncwarp();
-      n = S.rstart[R];
-      base = P0 - P_lo;
       src_b = A.sc_col;
       src_w = A.sc_wgt;
-      rp = A.row_ptr_c + (d.row0 - L.a_lo);
-    } else {  // B_BUCKET with <= kPieceCap entries (self entries already dropped)
-      R = 0;
-      const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
-      base = A.bkt_off[bk];
-      n = (int)(A.bkt_off[bk + 1] - base);
+      rp = A.row_ptr_c + (wi.row0 - L.a_lo);
+    } else {  // bin group with <= kPieceCap entries (self entries already dropped)
       src_b = A.pb_g;
       src_w = A.pw_g;
     }
     int T;
-    if (n <= 64) T = piece_dispatch<2, WIDE_KEYS>(d.row0, S, R, n, src_b, src_w, base, rp);
-    else if (n <= 128) T = piece_dispatch<4, WIDE_KEYS>(d.row0, S, R, n, src_b, src_w, base, rp);
-    else T = piece_dispatch<8, WIDE_KEYS>(d.row0, S, R, n, src_b, src_w, base, rp);
+    if (n <= 64) T = piece_dispatch<2, WIDE_KEYS>(wi.row0, S, R, n, src_b, src_w, base, rp);
+    else if (n <= 128) T = piece_dispatch<4, WIDE_KEYS>(wi.row0, S, R, n, src_b, src_w, base, rp);
+    else T = piece_dispatch<8, WIDE_KEYS>(wi.row0, S, R, n, src_b, src_w, base, rp);
     if (T < 0) {
       if (lane == 0) {
         A.need_wide[bi] = 1;
@@ -284,9 +282,9 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
       }
       continue;
     }
-    if (d.kind == B_PIECE) {
+    if (R > 0) {
       for (int r = lane; r < R; r += 32) {
-        const int32_t a = d.row0 + r;
+        const int32_t a = wi.row0 + r;
         const unsigned long long s = A.vw64[a];
         if (s > 0x7fffffffull) atomicOr(A.err, ERR_OVERFLOW);
         A.vwgt_c[a - L.a_lo] = (int32_t)s;

@@ -170,7 +170,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
         }
       } else {  // B_BUCKET: partitioned pairs of one skewed row (self entries already dropped)
         const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
-        const int64_t q0 = A.bkt_off[bk], cnt = A.bkt_off[bk + 1] - q0;
+        const int64_t q0 = A.bkt_off[bk], cnt = A.bkt_off[A.grp_end[bi]] - q0;  // the bin group
 #pragma unroll
         for (int k = 0; k < kIt; ++k) {
           const int s = t + kT * k;
@@ -340,8 +340,10 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
   }
 }
 
-// One warp per work block: copy its staged entries to the final CSR position
-// (blocks hold ~100 - 4096 entries; a CTA per block would be launch-bound).
+// Placement: each warp sweeps 32 consecutive blocks (one per lane for the
+// metadata) and copies the non-empty ones cooperatively to their final CSR
+// position (bin blocks inside a group are empty; a CTA or warp per block
+// would be launch- and latency-bound).
 constexpr int kPlaceT = 256;
 __device__ __forceinline__ void warp_copy(int32_t *__restrict__ dc, int32_t *__restrict__ dw,
                                           const int32_t *__restrict__ sc, const int32_t *__restrict__ sw, int T,
@@ -353,45 +355,65 @@ __device__ __forceinline__ void warp_copy(int32_t *__restrict__ dc, int32_t *__r
 }
 __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   const int lane = threadIdx.x & 31;
-  const int64_t bi = (int64_t)blockIdx.x * (kPlaceT / 32) + (threadIdx.x >> 5);
-  if (bi >= A.nblocks) return;
-  const BlockDesc d = A.blk[bi];
+  const int64_t b0 = ((int64_t)blockIdx.x * (kPlaceT / 32) + (threadIdx.x >> 5)) * 32;
+  if (b0 >= A.nblocks) return;
   const Layout &L = A.L;
-  const int64_t O = A.blk_off[bi];
-  const int T = A.blk_cnt[bi];
-  if (rows_kind(d.kind)) {
-    const int64_t P0 = L.upos(d.row0) - L.upos(L.a_lo);
-    warp_copy(A.col_c + O, A.wgt_c + O, A.sc_col + P0, A.sc_wgt + P0, T, lane);
-    for (int a = d.row0 + lane; a < d.row1; a += 32) A.row_ptr_c[a - L.a_lo] += O;
-  } else {
-    if (d.kind == B_DENSE) {
-      const int32_t *st = reinterpret_cast<const int32_t *>(A.dense + (int64_t)A.big_idx[d.row0] * L.n_c +
-                                                            (int64_t)d.sub * kCap);
-      for (int q = lane; q < T; q += 32) {
-        A.col_c[O + q] = st[2 * q];
-        A.wgt_c[O + q] = st[2 * q + 1];
-      }
+  const int64_t mine = b0 + lane;
+  BlockDesc dm{-1, 0, 0, 0};
+  int64_t Om = 0;
+  int Tm = 0;
+  bool need = false;
+  if (mine < A.nblocks) {
+    dm = A.blk[mine];
+    Om = A.blk_off[mine];
+    Tm = A.blk_cnt[mine];
+    need = Tm > 0 || rows_kind(dm.kind) || dm.sub == 0;
+  }
+  if (mine == A.nblocks - 1) A.row_ptr_c[L.a_hi - L.a_lo] = Om + Tm;
+  unsigned m = __ballot_sync(0xffffffffu, need);
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    BlockDesc d;
+    d.kind = __shfl_sync(0xffffffffu, dm.kind, j);
+    d.row0 = __shfl_sync(0xffffffffu, dm.row0, j);
+    d.row1 = __shfl_sync(0xffffffffu, dm.row1, j);
+    d.sub = __shfl_sync(0xffffffffu, dm.sub, j);
+    const int64_t O = __shfl_sync(0xffffffffu, Om, j);
+    const int T = __shfl_sync(0xffffffffu, Tm, j);
+    if (rows_kind(d.kind)) {
+      const int64_t P0 = L.upos(d.row0) - L.upos(L.a_lo);
+      warp_copy(A.col_c + O, A.wgt_c + O, A.sc_col + P0, A.sc_wgt + P0, T, lane);
+      for (int a = d.row0 + lane; a < d.row1; a += 32) A.row_ptr_c[a - L.a_lo] += O;
     } else {
-      const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
-      if (A.fb_cnt[bk] >= 0) {
-        const int64_t f0 = A.fb_off[bk];
-        warp_copy(A.col_c + O, A.wgt_c + O, A.fb_b + f0, A.fb_w + f0, T, lane);
-      } else {
-        const int64_t q0 = A.bkt_off[bk];
-        warp_copy(A.col_c + O, A.wgt_c + O, A.pb_g + q0, A.pw_g + q0, T, lane);
+      if (d.kind == B_DENSE) {
+        const int32_t *st = reinterpret_cast<const int32_t *>(A.dense + (int64_t)A.big_idx[d.row0] * L.n_c +
+                                                              (int64_t)d.sub * kCap);
+        for (int q = lane; q < T; q += 32) {
+          A.col_c[O + q] = st[2 * q];
+          A.wgt_c[O + q] = st[2 * q + 1];
+        }
+      } else if (T > 0) {
+        const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
+        if (A.fb_cnt[bk] >= 0) {
+          const int64_t f0 = A.fb_off[bk];
+          warp_copy(A.col_c + O, A.wgt_c + O, A.fb_b + f0, A.fb_w + f0, T, lane);
+        } else {
+          const int64_t q0 = A.bkt_off[bk];
+          warp_copy(A.col_c + O, A.wgt_c + O, A.pb_g + q0, A.pw_g + q0, T, lane);
+        }
       }
-    }
-    if (d.sub == 0 && lane == 0) {  // the row's first block: row start and vertex weight
-      A.row_ptr_c[d.row0 - L.a_lo] = O;
-      A.vwgt_c[d.row0 - L.a_lo] = (int32_t)A.vw64[d.row0];  // bound checked by k_tiers
+      if (d.sub == 0 && lane == 0) {  // the row's first block: row start and vertex weight
+        A.row_ptr_c[d.row0 - L.a_lo] = O;
+        A.vwgt_c[d.row0 - L.a_lo] = (int32_t)A.vw64[d.row0];  // bound checked by k_tiers
+      }
     }
   }
-  if (bi == A.nblocks - 1 && lane == 0) A.row_ptr_c[L.a_hi - L.a_lo] = O + T;
 }
 
 int launch_place(hec_ctx *ctx, const RowsArgs &A) {
   if (A.nblocks <= 0) return HEC_OK;
-  k_place<<<nblk(A.nblocks, kPlaceT / 32), kPlaceT, 0, ctx->stream>>>(A);
+  k_place<<<nblk((A.nblocks + 31) / 32, kPlaceT / 32), kPlaceT, 0, ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }
