@@ -93,16 +93,23 @@ struct DegIn {
 //   kPieceMax < U <= big_thr        CTA work blocks (windows of kWin, weight U + kRowW)
 //   U > big_thr                     skewed: key-range buckets (BUCKET mode, big_thr =
 //                                   kPieceMax) or dense accumulation (DENSE mode)
-__host__ __device__ __forceinline__ int64_t big_threshold(bool dense) { return dense ? kSmallMax : kPieceMax; }
+// (HEC_BUCKET_BIG_THR: tuning hook for the skewed-row threshold in BUCKET mode,
+//  clamped to [kPieceMax, kSmallMax])
+static int64_t big_threshold_host(bool dense) {
+  if (dense) return kSmallMax;
+  const char *e = getenv("HEC_BUCKET_BIG_THR");
+  int64_t t = e ? atoll(e) : kPieceMax;
+  return t < kPieceMax ? kPieceMax : (t > kSmallMax ? kSmallMax : t);
+}
 
 struct RowWeightIn {
   Layout L;
-  bool dense;
+  int64_t big_thr;
   __device__ __forceinline__ int64_t operator()(int64_t a) const {
     if (!L.active(a)) return 0;
     int64_t U = L.U(a);
     if (U <= kPieceMax) return U + kPieceRowW;
-    return U <= big_threshold(dense) ? U + kRowW : 0;
+    return U <= big_thr ? U + kRowW : 0;
   }
 };
 
@@ -157,8 +164,9 @@ struct BlockCountIn {
   Layout L;
   const int64_t *S;  // exclusive scan of RowWeightIn
   bool dense;
+  int64_t big_thr;
   __device__ __forceinline__ int cls(int64_t U) const {
-    return U <= kPieceMax ? 0 : (U <= big_threshold(dense) ? 1 : 2);
+    return U <= kPieceMax ? 0 : (U <= big_thr ? 1 : 2);
   }
   __device__ __forceinline__ int64_t operator()(int64_t a) const {
     if (!L.active(a)) return 0;
@@ -196,19 +204,41 @@ __global__ void k_block_ends(int64_t nblocks, int64_t a_hi, BlockDesc *__restric
 // Work units: big row h (list index) split into ceil(U/unit) windows of `unit`
 // member-edge positions (kUnit: partition, kCap: dense accumulation);
 // unit_ptr = exclusive scan over big rows.
+// Rows with U <= min_u get no units (BUCKET mode: partitioned by one warp).
 struct UnitsIn {
   Layout L;
   const int32_t *big_list;
   int64_t unit;
+  int64_t min_u;
   __device__ __forceinline__ int64_t operator()(int64_t h) const {
-    return (L.U(big_list[h]) + unit - 1) / unit;
+    const int64_t U = L.U(big_list[h]);
+    return U <= min_u ? 0 : (U + unit - 1) / unit;
   }
 };
+// Member-edge volume of big row h: prow = its exclusive scan places every
+// skewed row's partitioned pairs at [prow[h], prow[h] + U) (self entries leave
+// a gap at the end), so a row's bin offsets need no global scan.
+struct RowUIn {
+  Layout L;
+  const int32_t *big_list;
+  __device__ __forceinline__ int64_t operator()(int64_t h) const { return L.U(big_list[h]); }
+};
+constexpr int64_t kWarpRowMax = 4096;  // skewed rows up to this volume: one warp partitions the row
+constexpr int kWarpBins = (int)((kWarpRowMax + 31) / 32);  // row_buckets(kWarpRowMax) with kBucketAvg 32
 struct BucketsIn {
   Layout L;
   const int32_t *big_list;
   __device__ __forceinline__ int64_t operator()(int64_t h) const { return row_buckets(L.U(big_list[h]), L.n_c); }
 };
+
+// Segment -> owner table: out[k] = h for k in [ptr[h], ptr[h+1]) (a warp per
+// segment), replacing per-thread binary searches over the segment offsets.
+__global__ void k_seg_fill(int64_t nseg, const int64_t *__restrict__ ptr, int32_t *__restrict__ out) {
+  const int64_t h = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (h >= nseg) return;
+  const int lane = threadIdx.x & 31;
+  for (int64_t k = ptr[h] + lane; k < ptr[h + 1]; k += 32) out[k] = (int32_t)h;
+}
 
 // ------------------------------------------------------------ expansion
 // Every member-edge position p in [P_lo, P_hi) (the active rows) gets its
@@ -217,8 +247,89 @@ struct BucketsIn {
 // arrays with coalesced loads.  Self entries are kept (b == own row): the
 // consumers know their row and drop them.
 constexpr int kXT = 256;       // threads per CTA
-constexpr int kXChunk = 2048;  // positions per warp task
+constexpr int kXChunk = 4096;  // positions per warp task
 
+// Member table [tb, tb + 128) of the warp: member-edge starts (mpre) and source
+// row starts (mstart).  Reloaded only when the walk leaves it, so a window of
+// 128 positions inside a long member row costs no metadata traffic.
+__device__ __forceinline__ void exp_table_load(const Layout &L, const int64_t *__restrict__ mstart, int64_t mend,
+                                               int64_t tb, WarpExpTab &W) {
+  const int lane = threadIdx.x & 31;
+  const int64_t pend_m = L.mpre[mend];
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    const int64_t j = tb + lane + 32 * t;
+    W.mp[lane + 32 * t] = j < mend ? L.mpre[j] : pend_m;
+    W.ms[lane + 32 * t] = j < mend ? mstart[j] : 0;
+  }
+  if (lane == 0) W.mp[128] = tb + 128 < mend ? L.mpre[tb + 128] : pend_m;
+  __syncwarp();
+}
+
+// Plan the window of positions [q, q + n) (n <= 128) whose first position lies
+// in member i0: e[t] = source entry of position q + lane + 32 t (or -1).
+// Advances i0 to the member containing q + n; may reload the table.
+__device__ __forceinline__ int exp_plan(const Layout &L, const int64_t *__restrict__ mstart, int64_t mend, int64_t q,
+                                        int64_t Pend, int64_t &i0, int64_t &tb, WarpExpTab &W, int64_t (&e)[4]) {
+  const int lane = threadIdx.x & 31;
+  const int64_t want = q + 128 < Pend ? q + 128 : Pend;
+  if (i0 >= tb + 128 || (W.mp[128] < want && i0 != tb)) {
+    __syncwarp();
+    tb = i0;
+    exp_table_load(L, mstart, mend, tb, W);
+  }
+  const int64_t limit = W.mp[128] < want ? W.mp[128] : want;
+  const int n = (int)(limit - q);
+#pragma unroll
+  for (int t = 0; t < 4; ++t) W.mk[lane + 32 * t] = -1;
+  __syncwarp();
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {  // member k starts inside the window and is non-empty
+    const int k = lane + 32 * t;
+    const int64_t rs = W.mp[k] - q;
+    if (rs >= 0 && rs < n && W.mp[k + 1] > W.mp[k]) W.mk[rs] = k;
+  }
+  __syncwarp();
+  // inclusive max-scan over positions (blocked: lane owns 4 consecutive ones)
+  const int base = (int)(i0 - tb);  // member containing q, relative to the table
+  int m[4], run = base;
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    run = max(run, W.mk[4 * lane + t]);
+    m[t] = run;
+  }
+  int x = run;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x = max(x, y);
+  }
+  int before = __shfl_up_sync(0xffffffffu, x, 1);
+  if (lane == 0) before = base;
+  __syncwarp();
+#pragma unroll
+  for (int t = 0; t < 4; ++t) W.mk[4 * lane + t] = max(before, m[t]);
+  __syncwarp();
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    const int r = lane + 32 * t;
+    e[t] = -1;
+    if (r < n) {
+      const int k = W.mk[r];
+      e[t] = W.ms[k] + (q + r - W.mp[k]);
+    }
+  }
+  i0 = tb + last_le(W.mp, 0, 129, limit);
+  __syncwarp();
+  return n;
+}
+
+// Every member-edge position p in [P_lo, P_hi) (the active rows) gets its
+// fine entry's (b = M[v], w): Sb/Sw[p - P_lo].  One streaming pass with warp-level
+// member walks (no CTA barriers); all later construction kernels read these
+// arrays with coalesced loads.  Self entries are kept (b == own row): the
+// consumers know their row and drop them.  Two windows are in flight per warp:
+// the next window's col/wgt loads are issued before this window's M gathers.
 __global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restrict__ mstart,
                                               int32_t *__restrict__ Sb, int32_t *__restrict__ Sw) {
   __shared__ WarpExpTab W[kXT / 32];
@@ -228,22 +339,44 @@ __global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restr
   const int64_t gw = (int64_t)blockIdx.x * (kXT / 32) + wid;
   const int64_t nw = (int64_t)gridDim.x * (kXT / 32);
   for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
-    int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
+    const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
     int64_t i0 = warp_find_member(L, m_lo, m_hi, P);
-    int64_t q = P;
-    while (q < Pend) {
-      int32_t b4[4], w4[4];
-      int64_t m4[4];
-      const int got = warp_expand(L, mstart, m_hi, q, Pend, i0, W[wid], b4, w4, m4);
+    int64_t tb = i0;
+    exp_table_load(L, mstart, m_hi, tb, W[wid]);
+    int64_t q = P, e[4];
+    int32_t b0[4], w0[4];
+    int n0 = exp_plan(L, mstart, m_hi, q, Pend, i0, tb, W[wid], e);
+    int64_t q0 = q;
+    q += n0;
+#pragma unroll
+    for (int t = 0; t < 4; ++t)
+      if (e[t] >= 0) { b0[t] = __ldcs(L.col + e[t]); w0[t] = __ldcs(L.wgt + e[t]); }
+    while (n0 > 0) {
+      int32_t b1[4], w1[4];
+      int n1 = 0;
+      const int64_t q1 = q;
+      if (q < Pend) {
+        n1 = exp_plan(L, mstart, m_hi, q, Pend, i0, tb, W[wid], e);
+        q += n1;
+#pragma unroll
+        for (int t = 0; t < 4; ++t)
+          if (e[t] >= 0) { b1[t] = __ldcs(L.col + e[t]); w1[t] = __ldcs(L.wgt + e[t]); }
+      }
+#pragma unroll
+      for (int t = 0; t < 4; ++t)
+        if (lane + 32 * t < n0) b0[t] = __ldg(L.M + b0[t]);
 #pragma unroll
       for (int t = 0; t < 4; ++t) {
         const int off = lane + 32 * t;
-        if (off < got) {  // streaming stores: keep M (gathered) resident in L2
-          __stcs(Sb + q + off - P_lo, b4[t]);
-          __stcs(Sw + q + off - P_lo, w4[t]);
+        if (off < n0) {  // streaming stores: keep M (gathered) resident in L2
+          __stcs(Sb + q0 + off - P_lo, b0[t]);
+          __stcs(Sw + q0 + off - P_lo, w0[t]);
         }
       }
-      q += got;
+#pragma unroll
+      for (int t = 0; t < 4; ++t) { b0[t] = b1[t]; w0[t] = w1[t]; }
+      n0 = n1;
+      q0 = q1;
     }
   }
 }
@@ -264,6 +397,7 @@ struct PartArgs {
   const int32_t *big_list;
   int64_t nbig;
   const int64_t *unit_ptr;  // units of kUnit positions
+  const int32_t *unit_row;  // unit -> big row index
   const int64_t *bkt_ptr;
   const int32_t *Sb, *Sw;   // expanded entries, indexed from upos(a_lo)
 };
@@ -278,7 +412,7 @@ struct UnitInfo {
 
 __device__ __forceinline__ UnitInfo unit_info(const PartArgs &A, int64_t unit) {
   const Layout &L = A.L;
-  const int64_t h = last_le(A.unit_ptr, 0, A.nbig, unit);
+  const int64_t h = A.unit_row[unit];
   UnitInfo u;
   u.a = A.big_list[h];
   const int64_t P_lo = L.upos(L.a_lo);
@@ -302,17 +436,29 @@ __device__ __forceinline__ int part_bucket(const UnitInfo &u, int32_t b) {
 
 constexpr int kPartU = 8;  // loads in flight per thread in the partition passes
 
+// Bucket of the entry, or -1 for a self entry (dropped, L280) / past the unit.
+__device__ __forceinline__ int entry_bucket(const UnitInfo &u, int32_t b) {
+  return b == u.a ? -1 : part_bucket(u, b);
+}
+
+// Slot of the entry in its bucket (shared-memory cursor), or -1.  (A
+// __match_any_sync warp aggregation of equal buckets was measured slower: the
+// passes are bound by per-unit latency, not by same-address replays.)
+__device__ __forceinline__ int agg_add(int32_t *ctr, int bk) { return bk < 0 ? -1 : atomicAdd(ctr + bk, 1); }
+
 // histogram of the unit's entries (self entries dropped) into S.hist
 __device__ __forceinline__ void unit_hist(const PartArgs &A, const UnitInfo &u, PartSmem &S) {
   for (int i = threadIdx.x; i < u.nb; i += kT) S.hist[i] = 0;
   __syncthreads();
-  for (int64_t p = u.p0 + threadIdx.x; p < u.p1; p += kPartU * kT) {
+  const int32_t *Sb = A.Sb + u.p0;
+  const int cnt = (int)(u.p1 - u.p0);  // <= kUnit
+  // warp-uniform trip count: agg_add's __match_any_sync needs every lane
+  for (int p = threadIdx.x; p - (int)(threadIdx.x & 31) < cnt; p += kPartU * kT) {
     int32_t b[kPartU];
 #pragma unroll
-    for (int j = 0; j < kPartU; ++j) b[j] = p + j * kT < u.p1 ? __ldcs(A.Sb + p + j * kT) : u.a;
+    for (int j = 0; j < kPartU; ++j) b[j] = p + j * kT < cnt ? __ldcs(Sb + p + j * kT) : u.a;
 #pragma unroll
-    for (int j = 0; j < kPartU; ++j)
-      if (b[j] != u.a) atomicAdd(&S.hist[part_bucket(u, b[j])], 1);
+    for (int j = 0; j < kPartU; ++j) agg_add(S.hist, entry_bucket(u, b[j]));
   }
   __syncthreads();
 }
@@ -339,21 +485,120 @@ __global__ void __launch_bounds__(kT) k_part_write(PartArgs A, const int64_t *__
     if (c) S.base[i] = (int32_t)(bkt_off[u.b0 + i] - off0) + (int32_t)atomicAdd(bkt_cur + u.b0 + i, (unsigned)c);
   }
   __syncthreads();
-  for (int64_t p = u.p0 + threadIdx.x; p < u.p1; p += kPartU * kT) {
+  const int32_t *Sb = A.Sb + u.p0, *Sw = A.Sw + u.p0;
+  int32_t *pbr = pb + off0, *pwr = pw + off0;
+  const int cnt = (int)(u.p1 - u.p0);
+  for (int p = threadIdx.x; p - (int)(threadIdx.x & 31) < cnt; p += kPartU * kT) {
     int32_t b[kPartU], w[kPartU];
 #pragma unroll
     for (int j = 0; j < kPartU; ++j) {
-      const bool in = p + j * kT < u.p1;
-      b[j] = in ? __ldcs(A.Sb + p + j * kT) : u.a;
-      w[j] = in ? __ldcs(A.Sw + p + j * kT) : 0;
+      const bool in = p + j * kT < cnt;
+      b[j] = in ? __ldcs(Sb + p + j * kT) : u.a;
+      w[j] = in ? __ldcs(Sw + p + j * kT) : 0;
     }
 #pragma unroll
-    for (int j = 0; j < kPartU; ++j)
-      if (b[j] != u.a) {
-        const int64_t q = off0 + atomicAdd(&S.base[part_bucket(u, b[j])], 1);
-        pb[q] = b[j];
-        pw[q] = w[j];
+    for (int j = 0; j < kPartU; ++j) {
+      const int q = agg_add(S.base, entry_bucket(u, b[j]));
+      if (q >= 0) {
+        pbr[q] = b[j];
+        pwr[q] = w[j];
       }
+    }
+  }
+}
+
+// Skewed rows with U <= kWarpRowMax (<= kWarpBins bins): one warp counts the
+// row's entries per bin in shared memory, scans the counts into the row's bin
+// offsets (bkt_off = prow[h] + prefix, bkt_n = count) and scatters the pairs --
+// count, offsets and scatter without a CTA barrier or a global scan.
+constexpr int kPWT = 256;
+__global__ void __launch_bounds__(kPWT) k_part_warp(PartArgs A, const int64_t *__restrict__ prow,
+                                                    int64_t *__restrict__ bkt_off, unsigned *__restrict__ bkt_n,
+                                                    int32_t *__restrict__ pb, int32_t *__restrict__ pw) {
+  __shared__ int32_t hist[kPWT / 32][kWarpBins];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t h = (blockIdx.x * (int64_t)kPWT + threadIdx.x) >> 5;
+  if (h >= A.nbig) return;
+  const Layout &L = A.L;
+  UnitInfo u;
+  u.a = A.big_list[h];
+  const int64_t P_lo = L.upos(L.a_lo);
+  const int64_t P0 = L.upos(u.a), U = L.upos(u.a + 1) - P0;
+  if (U > kWarpRowMax) return;
+  u.b0 = A.bkt_ptr[h];
+  u.nb = (int32_t)(A.bkt_ptr[h + 1] - u.b0);
+  u.scale = (float)u.nb / (float)L.n_c;
+  int32_t *H = hist[wid];
+  for (int i = lane; i < u.nb; i += 32) H[i] = 0;
+  __syncwarp();
+  const int32_t *Sb = A.Sb + (P0 - P_lo), *Sw = A.Sw + (P0 - P_lo);
+  const int n = (int)U;
+  for (int p = lane; p < n; p += 32) {
+    const int32_t b = __ldg(Sb + p);
+    if (b != u.a) atomicAdd(&H[part_bucket(u, b)], 1);
+  }
+  __syncwarp();
+  // exclusive scan of the <= 128 bin counts (4 consecutive per lane)
+  int c[4], tot = 0;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int i = 4 * lane + j;
+    c[j] = i < u.nb ? H[i] : 0;
+    tot += c[j];
+  }
+  int x = tot;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  int run = x - tot;
+  const int64_t base = prow[h];
+  __syncwarp();
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int i = 4 * lane + j;
+    if (i < u.nb) {
+      H[i] = run;
+      bkt_off[u.b0 + i] = base + run;
+      bkt_n[u.b0 + i] = (unsigned)c[j];
+    }
+    run += c[j];
+  }
+  __syncwarp();
+  for (int p = lane; p < n; p += 32) {
+    const int32_t b = __ldg(Sb + p);
+    if (b != u.a) {
+      const int64_t q = base + atomicAdd(&H[part_bucket(u, b)], 1);
+      pb[q] = b;
+      pw[q] = __ldg(Sw + p);
+    }
+  }
+}
+
+// Bin offsets of the CTA-partitioned rows (U > kWarpRowMax): a warp scans the
+// row's bin counts (from k_part_count) into bkt_off = prow[h] + prefix.
+__global__ void k_row_bins(PartArgs A, const int64_t *__restrict__ prow, const unsigned *__restrict__ bkt_n,
+                           int64_t *__restrict__ bkt_off) {
+  const int lane = threadIdx.x & 31;
+  const int64_t h = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (h >= A.nbig) return;
+  const Layout &L = A.L;
+  const int32_t a = A.big_list[h];
+  if (L.U(a) <= kWarpRowMax) return;
+  const int64_t b0 = A.bkt_ptr[h], b1 = A.bkt_ptr[h + 1];
+  int64_t run = prow[h];
+  for (int64_t k0 = b0; k0 < b1; k0 += 32) {
+    const int64_t k = k0 + lane;
+    const int64_t c = k < b1 ? (int64_t)bkt_n[k] : 0;
+    int64_t x = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (k < b1) bkt_off[k] = run + x - c;
+    run += __shfl_sync(0xffffffffu, x, 31);
   }
 }
 
@@ -391,6 +636,7 @@ __device__ void block_bitonic(int32_t *key, V *val, int N) {
 
 __global__ void __launch_bounds__(kT) k_bucket_fallback(const int64_t *__restrict__ jobs, int64_t njobs,
                                                         const int64_t *__restrict__ bkt_off,
+                                                        const unsigned *__restrict__ bkt_n,
                                                         const int32_t *__restrict__ pb, const int32_t *__restrict__ pw,
                                                         const int64_t *__restrict__ fb_off, int32_t *__restrict__ fb_cnt,
                                                         int32_t *__restrict__ fb_b, int32_t *__restrict__ fb_w,
@@ -403,7 +649,7 @@ __global__ void __launch_bounds__(kT) k_bucket_fallback(const int64_t *__restric
     const int64_t j = S.job;
     if (j >= njobs) return;
     const int64_t bk = jobs[j];
-    const int64_t q0 = bkt_off[bk], q1 = bkt_off[bk + 1];
+    const int64_t q0 = bkt_off[bk], q1 = q0 + bkt_n[bk];
     // key range of the bucket's entries (sub-ranges split it when a pass overflows)
     if (threadIdx.x == 0) { S.kmin = INT32_MAX; S.kmax = -1; }
     __syncthreads();
@@ -491,18 +737,19 @@ __global__ void __launch_bounds__(kT) k_bucket_fallback(const int64_t *__restric
 // Per bucket k (of big row h): its block descriptor, and a fallback job when it
 // holds more than kCap entries.
 __global__ void k_bucket_blocks(int64_t nbig, int64_t nbkt, const int32_t *__restrict__ big_list,
-                                const int64_t *__restrict__ bkt_ptr, const int64_t *__restrict__ bkt_off,
+                                const int64_t *__restrict__ bkt_ptr, const int32_t *__restrict__ bin_row,
+                                const unsigned *__restrict__ bkt_n,
                                 const int64_t *__restrict__ blk_ptr, BlockDesc *__restrict__ blk,
                                 int64_t *__restrict__ jobs, unsigned *__restrict__ njobs,
                                 int32_t *__restrict__ fb_cnt, int64_t *__restrict__ fb_off,
                                 unsigned long long *__restrict__ fb_total) {
   int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= nbkt) return;
-  const int64_t h = last_le(bkt_ptr, 0, nbig, k);
+  const int64_t h = bin_row[k];
   const int64_t b0 = bkt_ptr[h];
   const int32_t a = big_list[h];
   blk[blk_ptr[a] + (k - b0)] = BlockDesc{B_BUCKET, a, a + 1, (int32_t)(k - b0)};
-  const int64_t c = bkt_off[k + 1] - bkt_off[k];
+  const int64_t c = bkt_n[k];
   if (c > kCap) {
     unsigned j = atomicAdd(njobs, 1u);
     jobs[j] = k;
@@ -518,10 +765,17 @@ __global__ void k_bucket_blocks(int64_t nbig, int64_t nbkt, const int32_t *__res
 // holds < 2 kGroupWin entries); a bin above kGroupWin stands alone.  The group's
 // first bin carries its block (count, staging at its first pair); the other
 // bins' blocks are empty.
-__device__ __forceinline__ bool group_start(const int64_t *__restrict__ bkt_off, int64_t b0, int64_t k) {
+// Groups also break where the bins' key ranges cross a kGroupRange window, so a
+// group of a dense enough row spans < 2 kGroupRange keys and takes the
+// bitmap-rank path of k_pieces (bin k covers keys ~[k n_c / nb, (k+1) n_c / nb)).
+constexpr int64_t kGroupRange = 16384;
+__device__ __forceinline__ bool group_start(const int64_t *__restrict__ bkt_off, const unsigned *__restrict__ bkt_n,
+                                            int64_t b0, int64_t b1, int64_t n_c, int64_t k) {
   if (k == b0) return true;
-  const int64_t ck = bkt_off[k + 1] - bkt_off[k], cp = bkt_off[k] - bkt_off[k - 1];
+  const int64_t ck = bkt_n[k], cp = bkt_n[k - 1];
   if (ck > kGroupWin || cp > kGroupWin) return true;
+  const int64_t nb = b1 - b0;
+  if (((k - b0) * n_c / nb) / kGroupRange != ((k - 1 - b0) * n_c / nb) / kGroupRange) return true;
   return (bkt_off[k] - bkt_off[b0]) / kGroupWin != (bkt_off[k - 1] - bkt_off[b0]) / kGroupWin;
 }
 
@@ -530,6 +784,7 @@ __device__ __forceinline__ bool group_start(const int64_t *__restrict__ bkt_off,
 // count is final here.  list_n: [0] warp list, [1] CTA list.
 __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__ blk, const int32_t *__restrict__ big_idx,
                         const int64_t *__restrict__ bkt_ptr, const int64_t *__restrict__ bkt_off,
+                        const unsigned *__restrict__ bkt_n,
                         const int32_t *__restrict__ fb_cnt, int32_t *__restrict__ blk_cnt,
                         int64_t *__restrict__ grp_end,
                         WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, unsigned *__restrict__ list_n,
@@ -554,14 +809,14 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
       const int64_t b0 = bkt_ptr[h], b1 = bkt_ptr[h + 1], bk = b0 + d.sub;
       if (fb_cnt[bk] >= 0) {
         blk_cnt[bi] = fb_cnt[bk];
-      } else if (!group_start(bkt_off, b0, bk)) {
+      } else if (!group_start(bkt_off, bkt_n, b0, b1, L.n_c, bk)) {
         blk_cnt[bi] = 0;
       } else {
         int64_t e = bk + 1;
-        while (e < b1 && !group_start(bkt_off, b0, e)) ++e;
+        while (e < b1 && !group_start(bkt_off, bkt_n, b0, b1, L.n_c, e)) ++e;
         grp_end[bi] = e;
         it.base = bkt_off[bk];
-        it.n = (int32_t)(bkt_off[e] - bkt_off[bk]);
+        it.n = (int32_t)(bkt_off[e - 1] + bkt_n[e - 1] - bkt_off[bk]);
         tier = it.n <= kPieceCap ? 0 : 1;
       }
     }
@@ -599,11 +854,18 @@ struct DenseArgs {
   const int32_t *big_list;
   int64_t nbig;
   const int64_t *unit_ptr;
+  const int32_t *unit_row;
   int64_t nunits;
   unsigned *ticket;
   unsigned long long *dense;  // [nbig][n_c] (zeroed)
   const int32_t *Sb, *Sw;     // expanded entries, indexed from upos(a_lo)
 };
+
+// A dense unit is kDenseIt entries per thread: all of a unit's loads are issued
+// before its atomics, so each CTA keeps 16 KB x 2 of staging reads in flight
+// (one 4096-entry unit per round trip left the kernel latency-bound).
+constexpr int kDenseIt = 16;
+constexpr int kDenseUnit = kT * kDenseIt;
 
 __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -621,22 +883,25 @@ __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
     if (threadIdx.x == 0) s_unit = (int64_t)atomicAdd(A.ticket, 1u);
     __syncthreads();
     const int64_t unit = s_unit;
-    const int64_t h = unit < A.nunits ? last_le(A.unit_ptr, 0, A.nbig, unit) : -1;
-    int32_t kb[kIt], kw[kIt];
+    const int64_t h = unit < A.nunits ? A.unit_row[unit] : -1;
+    int32_t kb[kDenseIt], kw[kDenseIt];
     long long usum = 0;  // exact weight of this thread's slots
 #pragma unroll
-    for (int k = 0; k < kIt; ++k) { kb[k] = -1; kw[k] = 0; }
+    for (int k = 0; k < kDenseIt; ++k) { kb[k] = -1; kw[k] = 0; }
     if (h >= 0) {
       const int32_t a = A.big_list[h];
-      const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kCap;
-      const int64_t Pend = L.upos(a + 1);
+      const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kDenseUnit;
+      const int cnt = (int)min((int64_t)kDenseUnit, L.upos(a + 1) - P0);
+      const int32_t *Sb = A.Sb + (P0 - P_lo), *Sw = A.Sw + (P0 - P_lo);
 #pragma unroll
-      for (int k = 0; k < kIt; ++k) {
-        const int64_t p = P0 + threadIdx.x + (int64_t)kT * k;
-        if (p < Pend) {
-          const int32_t b = A.Sb[p - P_lo];
-          if (b != a) { kb[k] = b; kw[k] = A.Sw[p - P_lo]; usum += kw[k]; }
-        }
+      for (int k = 0; k < kDenseIt; ++k) {
+        const int p = threadIdx.x + kT * k;
+        if (p < cnt) { kb[k] = __ldcs(Sb + p); kw[k] = __ldcs(Sw + p); }
+      }
+#pragma unroll
+      for (int k = 0; k < kDenseIt; ++k) {
+        if (kb[k] == a) kb[k] = -1;  // self entry (L280)
+        if (kb[k] >= 0) usum += kw[k];
       }
     }
 #pragma unroll
@@ -656,9 +921,17 @@ __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
     }
     if (h < 0) return;
     cur_h = h;
+    if (unit_w > 0x7fffffffLL) {  // the unit alone could overflow int32: exact 64-bit sums in global
+      unsigned long long *dst = A.dense + h * (int64_t)nc;
+#pragma unroll
+      for (int k = 0; k < kDenseIt; ++k)
+        if (kb[k] >= 0) atomicAdd(dst + kb[k], (unsigned long long)(uint32_t)kw[k]);
+      __syncthreads();
+      continue;
+    }
     running += unit_w;
 #pragma unroll
-    for (int k = 0; k < kIt; ++k)
+    for (int k = 0; k < kDenseIt; ++k)
       if (kb[k] >= 0) atomicAdd(acc + kb[k], kw[k]);
     __syncthreads();
   }
@@ -748,11 +1021,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t n_out = a_hi - a_lo;  // rows produced by this call
   Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi};
   const bool dense = n_c <= kDenseMax;
-  k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_threshold(dense), big_list, big_idx, counts + 0,
+  const int64_t big_thr = big_threshold_host(dense);
+  k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_thr, big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));
   HEC_LAUNCH_CHECK();
-  HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, dense}, PtrOut{Sw}, st[2], Sw + n_c));
-  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c));
+  HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, big_thr}, PtrOut{Sw}, st[2], Sw + n_c));
+  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 4, counts + 0, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
   phase_end(ctx, ph);
   int64_t r0[5];
@@ -764,7 +1038,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t small_vol = r0[1], big_vol = r0[2];
   const int64_t nbig = r0[4] & 0xffffffffLL;
   if (nbig > 0) {
-    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)kCap : (int64_t)kUnit}, PtrOut{unit_ptr},
+    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)kDenseUnit : (int64_t)kUnit,
+                                             dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
                          st[4], unit_ptr + nbig));
     if (!dense) HEC_TRY(chained_scan(ctx, nbig, BucketsIn{L, big_list}, PtrOut{bkt_ptr}, st[5], bkt_ptr + nbig));
     HEC_CUDA_TRY(cudaMemcpyAsync(scal + 5, unit_ptr + nbig, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
@@ -783,11 +1058,14 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
+    if (nbig > 0) b2 += ws_bytes(nunits + 1, 4);  // unit_row
     if (nbig > 0 && dense) b2 += ws_bytes((size_t)nbig * n_c, 8);
     if (nbig > 0 && !dense) {
       b2 += 2 * ws_bytes(nbkt + 1, 4) + 2 * ws_bytes(nbkt + 1, 8) + ws_bytes(nbkt + 1, 4);
       b2 += 4 * ws_bytes((size_t)big_vol + 1, 4) + scan_ws_bytes(nbkt);
       b2 += ws_bytes(nbkt + 1, 8) + ws_bytes(2 * nbkt + 2, 4);
+      b2 += ws_bytes(nbkt + 1, 4);  // bin_row
+      b2 += ws_bytes(nbig + 1, 8);  // prow
     }
     HEC_TRY(arena_reserve(ctx, &ctx->ws2, b2));
     ctx->ws2.used = 0;
@@ -854,10 +1132,17 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
 
   // ---- a9 skewed rows
   const int ph_skew = phase_begin(ctx, "rows_skew", 8.0 * (double)big_vol);
+  int32_t *unit_row = nullptr;
+  if (nbig > 0) {
+    unit_row = arena_take<int32_t>(W2, nunits + 1);
+    if (!unit_row) { set_error("workspace under-reserved (units)"); return HEC_EINVAL; }
+    k_seg_fill<<<nblk(nbig * 32, 256), 256, 0, s>>>(nbig, unit_ptr, unit_row);
+    HEC_LAUNCH_CHECK();
+  }
   if (nbig > 0 && dense) {
     unsigned long long *dn_arr = arena_take<unsigned long long>(W2, (size_t)nbig * n_c);
     HEC_CUDA_TRY(cudaMemsetAsync(dn_arr, 0, sizeof(unsigned long long) * nbig * n_c, s));
-    DenseArgs D{L, big_list, nbig, unit_ptr, nunits, counts + 2, dn_arr, sc_col, sc_wgt};
+    DenseArgs D{L, big_list, nbig, unit_ptr, unit_row, nunits, counts + 2, dn_arr, sc_col, sc_wgt};
     int occ = 1;
     HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum, kT, 4 * (size_t)n_c));
     if (occ < 1) occ = 1;
@@ -879,13 +1164,25 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     if (!fb_w) { set_error("workspace under-reserved (buckets)"); return HEC_EINVAL; }
     HEC_CUDA_TRY(cudaMemsetAsync(bkt_cnt, 0, sizeof(unsigned) * (nbkt + 1), s));
     HEC_CUDA_TRY(cudaMemsetAsync(bkt_cur, 0, sizeof(unsigned) * (nbkt + 1), s));
-    PartArgs PA{L, big_list, nbig, unit_ptr, bkt_ptr, sc_col, sc_wgt};
-    k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt);
+    int64_t *prow = arena_take<int64_t>(W2, nbig + 1);
+    if (!prow) { set_error("workspace under-reserved (prow)"); return HEC_EINVAL; }
+    HEC_TRY(chained_scan(ctx, nbig, RowUIn{L, big_list}, PtrOut{prow}, stb, prow + nbig));
+    PartArgs PA{L, big_list, nbig, unit_ptr, unit_row, bkt_ptr, sc_col, sc_wgt};
+    if (nunits > 0) {  // rows above kWarpRowMax: CTA units count, per-row scan, scatter
+      k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt);
+      HEC_LAUNCH_CHECK();
+      k_row_bins<<<nblk(nbig * 32, 256), 256, 0, s>>>(PA, prow, bkt_cnt, bkt_off);
+      HEC_LAUNCH_CHECK();
+      k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, bkt_cur, pb, pw);
+      HEC_LAUNCH_CHECK();
+    }
+    k_part_warp<<<nblk(nbig * 32, kPWT), kPWT, 0, s>>>(PA, prow, bkt_off, bkt_cnt, pb, pw);
     HEC_LAUNCH_CHECK();
-    HEC_TRY(chained_scan(ctx, nbkt, CountIn{bkt_cnt}, PtrOut{bkt_off}, stb, bkt_off + nbkt));
-    k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, bkt_cur, pb, pw);
+    int32_t *bin_row = arena_take<int32_t>(W2, nbkt + 1);
+    if (!bin_row) { set_error("workspace under-reserved (bins)"); return HEC_EINVAL; }
+    k_seg_fill<<<nblk(nbig * 32, 256), 256, 0, s>>>(nbig, bkt_ptr, bin_row);
     HEC_LAUNCH_CHECK();
-    k_bucket_blocks<<<nblk(nbkt, 256), 256, 0, s>>>(nbig, nbkt, big_list, bkt_ptr, bkt_off, blk_ptr, blk, jobs,
+    k_bucket_blocks<<<nblk(nbkt, 256), 256, 0, s>>>(nbig, nbkt, big_list, bkt_ptr, bin_row, bkt_cnt, blk_ptr, blk, jobs,
                                                    counts + 4, fb_cnt, fb_off,
                                                    reinterpret_cast<unsigned long long *>(scal + 10));
     HEC_LAUNCH_CHECK();
@@ -894,11 +1191,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_TRY(read_scalars(ctx, scal + 9, 1, rj));
     const int64_t njobs = rj[0] & 0xffffffffLL;
     if (njobs > 0) {
-      k_bucket_fallback<<<ctx->num_sms, kT, sizeof(FbSmem), s>>>(jobs, njobs, bkt_off, pb, pw, fb_off,
+      k_bucket_fallback<<<ctx->num_sms, kT, sizeof(FbSmem), s>>>(jobs, njobs, bkt_off, bkt_cnt, pb, pw, fb_off,
                                                                 fb_cnt, fb_b, fb_w, counts + 3, err);
       HEC_LAUNCH_CHECK();
     }
     A.bkt_off = bkt_off;
+    A.bkt_n = bkt_cnt;
     A.pb_g = pb;
     A.pw_g = pw;
     A.fb_cnt = fb_cnt;
@@ -911,7 +1209,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (nblocks > 0) {
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
-    k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.fb_cnt, blk_cnt, grp_end, list_w,
+    k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
                                               list_c, counts + 6, vw64, err);
     HEC_LAUNCH_CHECK();
   }

@@ -253,7 +253,8 @@ struct RowsArgs {
   int32_t *sc_col, *sc_wgt;         // SMALL staging, member-edge space [nnz]
   // BUCKET mode
   const int64_t *bkt_ptr;           // [nbig+1] first bucket of big row h
-  const int64_t *bkt_off;           // [nbkt+1] pair offsets
+  const int64_t *bkt_off;           // [nbkt+1] pair offsets (bin start in pb_g/pw_g)
+  const unsigned *bkt_n;            // [nbkt] pairs per bin (a row's bins are contiguous)
   const int64_t *grp_end;           // [nblocks] BUCKET group: one past its last bin (k_tiers)
   int32_t *pb_g, *pw_g;             // partitioned pairs (sorted uniques written back in place)
   const int32_t *fb_cnt;            // fallback unique count per bucket (-1: not overflowed)

@@ -229,6 +229,204 @@ __device__ __forceinline__ int piece_run(int32_t row0, PieceTab &S, int R, int n
   return piece_sort_merge<J, K>(key, val, S, src_b, src_w, base, R, row_ptr_rel);
 }
 
+// ---------------------------------------------------------------------------
+// Bin groups with a narrow key range: ordered dedup by bitmap rank, no sort.
+// All keys of a group lie in [lo, lo + kGrpBits); a warp-private bitmap marks
+// the distinct keys, so the rank of a key in the sorted output is the number of
+// set bits before it (per-lane 32-word block totals -> warp scan, per-word
+// prefixes inside a block).  Each entry then adds its weight at its rank: the
+// duplicate merge of DEDUPWITHWTS with O(entries) work
+// instead of a sorting network.  Bitmap words are XOR-swizzled inside their
+// 32-word block so the per-lane block walks are bank-conflict free.
+constexpr int kGrpBits = 32768;
+constexpr int kGrpWords = kGrpBits / 32;
+
+struct GroupTab {
+  uint32_t bm[kGrpWords];
+  uint16_t pref[kGrpWords];   // set bits before the word inside its 32-word block
+  int32_t key[kPieceCap];
+  int32_t val[kPieceCap];
+};
+union WarpTab {
+  PieceTab p;
+  GroupTab g;
+};
+
+__device__ __forceinline__ int grp_swz(int wd) { return wd ^ ((wd >> 5) & 31); }
+
+// Entries b[k] >= 0 (padding: -1) with total weight <= INT32_MAX; keys in
+// [lo, lo + 32 * nwords).  Writes the sorted distinct (key, summed weight) to
+// dst_b/dst_w[base ...] and returns their number.
+template <int J>
+__device__ __forceinline__ int group_bitmap(const int32_t (&b)[J], const int32_t (&w)[J], int32_t lo, int nwords,
+                                            GroupTab &G, int32_t *__restrict__ dst_b, int32_t *__restrict__ dst_w,
+                                            int64_t base) {
+  const int lane = threadIdx.x & 31;
+  const int nblk = (nwords + 31) >> 5;
+  for (int i = lane; i < nblk * 32; i += 32) G.bm[i] = 0;
+  for (int i = lane; i < kPieceCap; i += 32) G.val[i] = 0;
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < J; ++k)
+    if (b[k] >= 0) {
+      const int o = b[k] - lo;
+      atomicOr(&G.bm[grp_swz(o >> 5)], 1u << (o & 31));
+    }
+  __syncwarp();
+  int cnt = 0;
+  if (lane < nblk) {
+#pragma unroll 8
+    for (int i = 0; i < 32; ++i) {
+      const int ph = lane * 32 + (i ^ lane);  // grp_swz(lane * 32 + i)
+      G.pref[ph] = (uint16_t)cnt;
+      cnt += __popc(G.bm[ph]);
+    }
+  }
+  int incl = cnt;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += y;
+  }
+  const int excl = incl - cnt;
+  const int T = __shfl_sync(0xffffffffu, incl, 31);
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < J; ++k) {
+    const bool v = b[k] >= 0;
+    const int o = v ? b[k] - lo : 0;
+    const int wd = o >> 5;
+    const int bb = __shfl_sync(0xffffffffu, excl, wd >> 5);
+    if (v) {
+      const int ph = grp_swz(wd);
+      const int r = bb + G.pref[ph] + __popc(G.bm[ph] & ((1u << (o & 31)) - 1u));
+      atomicAdd(&G.val[r], w[k]);
+      G.key[r] = b[k];  // every duplicate stores the same key
+    }
+  }
+  __syncwarp();
+  for (int q = lane; q < T; q += 32) {
+    dst_b[base + q] = G.key[q];
+    dst_w[base + q] = G.val[q];
+  }
+  __syncwarp();
+  return T;
+}
+
+// Small bin groups (n <= 32 J entries, J <= 2): rank by bit-serial ballots.
+// For each own key, eq[s] / less[s] are the lanes whose slot-s key equals /
+// is below it on the bits seen so far (most significant first, only the bits
+// where the group's keys differ).  Duplicates are merged with one
+// __reduce_add_sync per slot over the equal-key partition (labelled-partition
+// reduction); the first copy (lowest slot, then lane) writes (key, sum) at its
+// rank among the distinct keys -- no sorting network, no shared memory.
+template <int J>
+__device__ __forceinline__ int group_ballot(const int32_t (&b)[J], const int32_t (&w)[J], int32_t mn, int32_t mx,
+                                            int32_t *__restrict__ dst_b, int32_t *__restrict__ dst_w, int64_t base) {
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = (1u << lane) - 1u;
+  unsigned vm[J];
+#pragma unroll
+  for (int s = 0; s < J; ++s) vm[s] = __ballot_sync(0xffffffffu, b[s] >= 0);
+  unsigned eq[J][J], less[J][J];
+#pragma unroll
+  for (int t = 0; t < J; ++t)
+#pragma unroll
+    for (int s = 0; s < J; ++s) { eq[t][s] = vm[s]; less[t][s] = 0u; }
+  const int nbits = 32 - __clz((unsigned)(mx ^ mn));
+  for (int i = nbits - 1; i >= 0; --i) {
+    unsigned ones[J];
+#pragma unroll
+    for (int s = 0; s < J; ++s) ones[s] = __ballot_sync(0xffffffffu, (b[s] >> i) & 1);
+#pragma unroll
+    for (int t = 0; t < J; ++t) {
+      const unsigned bt = 0u - (((unsigned)b[t] >> i) & 1u);  // all ones when the bit is set
+#pragma unroll
+      for (int s = 0; s < J; ++s) {
+        less[t][s] |= bt & eq[t][s] & ~ones[s];
+        eq[t][s] &= ~(bt ^ ones[s]);
+      }
+    }
+  }
+  // first copy of each key: no equal key in a lower slot, none on a lower lane of its slot
+  bool lead[J];
+  unsigned lm[J];
+#pragma unroll
+  for (int t = 0; t < J; ++t) {
+    bool l = b[t] >= 0 && (eq[t][t] & lt) == 0u;
+#pragma unroll
+    for (int s = 0; s < t; ++s) l = l && eq[t][s] == 0u;
+    lead[t] = l;
+  }
+#pragma unroll
+  for (int s = 0; s < J; ++s) lm[s] = __ballot_sync(0xffffffffu, lead[s]);
+  int red[J];
+#pragma unroll
+  for (int s = 0; s < J; ++s) red[s] = __reduce_add_sync(b[s] >= 0 ? eq[s][s] : (1u << lane), w[s]);
+  int T = 0;
+#pragma unroll
+  for (int s = 0; s < J; ++s) T += __popc(lm[s]);
+#pragma unroll
+  for (int t = 0; t < J; ++t) {
+    int rank = 0, sum = 0;
+#pragma unroll
+    for (int s = 0; s < J; ++s) {
+      rank += __popc(less[t][s] & lm[s]);
+      const unsigned e = b[t] >= 0 ? eq[t][s] : 0u;
+      const int src = e ? __ffs(e) - 1 : lane;
+      const int v = __shfl_sync(0xffffffffu, red[s], src);
+      sum += e ? v : 0;
+    }
+    if (lead[t]) {
+      dst_b[base + rank] = b[t];
+      dst_w[base + rank] = sum;
+    }
+  }
+  __syncwarp();
+  return T;
+}
+
+// A bin group (R == 0): bitmap rank when its key range is narrow, else the
+// sorting network.  Returns the distinct count or -1 (needs 64-bit sums).
+template <int J>
+__device__ __forceinline__ int group_run(WarpTab &S, int n, int32_t *__restrict__ src_b, int32_t *__restrict__ src_w,
+                                         int64_t base) {
+  const int lane = threadIdx.x & 31;
+  int32_t b[J], w[J];
+  long long wsum = 0;
+  int mn = INT32_MAX, mx = -1;
+#pragma unroll
+  for (int k = 0; k < J; ++k) {
+    const int s = lane + 32 * k;
+    b[k] = -1;
+    w[k] = 0;
+    if (s < n) {
+      b[k] = __ldcs(src_b + base + s);
+      w[k] = __ldcs(src_w + base + s);
+      wsum += w[k];
+      mn = min(mn, b[k]);
+      mx = max(mx, b[k]);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    wsum += __shfl_xor_sync(0xffffffffu, wsum, o);
+    mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+    mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  }
+  if (wsum > 0x7fffffffLL) return -1;
+  if (mx < 0) return 0;
+  if constexpr (J <= 2) {
+    return group_ballot<J>(b, w, mn, mx, src_b, src_w, base);
+  } else if ((int64_t)mx - mn < kGrpBits) {
+    return group_bitmap<J>(b, w, mn, ((mx - mn) >> 5) + 1, S.g, src_b, src_w, base);
+  }
+  uint32_t key[J];
+#pragma unroll
+  for (int k = 0; k < J; ++k) key[k] = (uint32_t)b[k];  // padding -1 == kPad
+  return piece_sort_merge<J, uint32_t>(key, w, S.p, src_b, src_w, base, 0, nullptr);
+}
+
 template <int J, bool WIDE_KEYS>
 __device__ __forceinline__ int piece_dispatch(int32_t row0, PieceTab &S, int R, int n, int32_t *src_b,
                                               int32_t *src_w, int64_t base, int64_t *rp) {
@@ -238,9 +436,10 @@ __device__ __forceinline__ int piece_dispatch(int32_t row0, PieceTab &S, int R, 
 
 template <bool WIDE_KEYS>
 __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__restrict__ ticket) {
-  __shared__ PieceTab tabs[kPW];
+  extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  PieceTab &S = tabs[wid];
+  WarpTab &W = reinterpret_cast<WarpTab *>(smem_raw)[wid];
+  PieceTab &S = W.p;
   const Layout &L = A.L;
   const int64_t P_lo = L.upos(L.a_lo);
   const int64_t nlist = *A.nlist;
@@ -272,7 +471,12 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
       src_w = A.pw_g;
     }
     int T;
-    if (n <= 64) T = piece_dispatch<2, WIDE_KEYS>(wi.row0, S, R, n, src_b, src_w, base, rp);
+    if (R == 0) {
+      if (n <= 32) T = group_run<1>(W, n, src_b, src_w, base);
+      else if (n <= 64) T = group_run<2>(W, n, src_b, src_w, base);
+      else if (n <= 128) T = group_run<4>(W, n, src_b, src_w, base);
+      else T = group_run<8>(W, n, src_b, src_w, base);
+    } else if (n <= 64) T = piece_dispatch<2, WIDE_KEYS>(wi.row0, S, R, n, src_b, src_w, base, rp);
     else if (n <= 128) T = piece_dispatch<4, WIDE_KEYS>(wi.row0, S, R, n, src_b, src_w, base, rp);
     else T = piece_dispatch<8, WIDE_KEYS>(wi.row0, S, R, n, src_b, src_w, base, rp);
     if (T < 0) {
@@ -298,9 +502,12 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
 // Keys of row pieces pack (row, b) into 32 bits while n_c <= 2^26.
 int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket) {
   static int occ[2] = {0, 0};
+  constexpr size_t smem = sizeof(WarpTab) * kPW;
   if (!occ[0]) {
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_pieces<false>, kPW * 32, 0));
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_pieces<true>, kPW * 32, 0));
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_pieces<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_pieces<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_pieces<false>, kPW * 32, smem));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_pieces<true>, kPW * 32, smem));
     if (occ[0] < 1) occ[0] = 1;
     if (occ[1] < 1) occ[1] = 1;
   }
@@ -309,8 +516,8 @@ int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket) {
   int64_t grid = (int64_t)ctx->num_sms * occ[wide_keys ? 1 : 0];
   if (A.nblocks < grid * kPW) grid = (A.nblocks + kPW - 1) / kPW;
   if (grid < 1) return HEC_OK;
-  if (wide_keys) k_pieces<true><<<(unsigned)grid, kPW * 32, 0, ctx->stream>>>(A, ticket);
-  else k_pieces<false><<<(unsigned)grid, kPW * 32, 0, ctx->stream>>>(A, ticket);
+  if (wide_keys) k_pieces<true><<<(unsigned)grid, kPW * 32, smem, ctx->stream>>>(A, ticket);
+  else k_pieces<false><<<(unsigned)grid, kPW * 32, smem, ctx->stream>>>(A, ticket);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }

@@ -170,7 +170,8 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
         }
       } else {  // B_BUCKET: partitioned pairs of one skewed row (self entries already dropped)
         const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
-        const int64_t q0 = A.bkt_off[bk], cnt = A.bkt_off[A.grp_end[bi]] - q0;  // the bin group
+        const int64_t ge = A.grp_end[bi] - 1;
+        const int64_t q0 = A.bkt_off[bk], cnt = A.bkt_off[ge] + A.bkt_n[ge] - q0;  // the bin group
 #pragma unroll
         for (int k = 0; k < kIt; ++k) {
           const int s = t + kT * k;
@@ -348,9 +349,19 @@ constexpr int kPlaceT = 256;
 __device__ __forceinline__ void warp_copy(int32_t *__restrict__ dc, int32_t *__restrict__ dw,
                                           const int32_t *__restrict__ sc, const int32_t *__restrict__ sw, int T,
                                           int lane) {
-  for (int q = lane; q < T; q += 32) {
-    dc[q] = __ldcs(sc + q);
-    dw[q] = __ldcs(sw + q);
+  // four loads per lane in flight before the stores (the copy is latency-bound)
+  for (int q0 = 0; q0 < T; q0 += 128) {
+    int32_t c[4], w[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int q = q0 + lane + 32 * j;
+      if (q < T) { c[j] = __ldcs(sc + q); w[j] = __ldcs(sw + q); }
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int q = q0 + lane + 32 * j;
+      if (q < T) { dc[q] = c[j]; dw[q] = w[j]; }
+    }
   }
 }
 __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {

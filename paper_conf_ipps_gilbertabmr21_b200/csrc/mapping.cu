@@ -20,8 +20,11 @@
 namespace hec {
 
 // ---------------------------------------------------------------- a1 heavy
+// 2048-item tiles keep a CTA's shared memory at ~37 KB, so six CTAs share an SM
+// and one CTA's TMA load overlaps the others' walks (HBM needs ~35 KB in flight
+// per SM); 4096-item tiles (82 KB, two per SM) left the stream latency-bound.
 constexpr int kHvBlock = 256;
-constexpr int kHvItems = 16;
+constexpr int kHvItems = 8;
 constexpr int kHvTile = kHvBlock * kHvItems;  // merge items (row ends + entries) per tile
 
 // Merge-path split of diagonal d between the row-end list row_ptr[1..n] and the
@@ -85,10 +88,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
   }
 }
 
+static_assert(kHvTile + 2 < 32767, "rb[] holds int16 offsets");
 struct HeavySmem {
   alignas(16) int32_t col[kHvTile + 8];
   alignas(16) int32_t wgt[kHvTile + 8];
-  int32_t rb[kHvTile + 2];        // row begin offsets relative to the tile's first entry
+  int16_t rb[kHvTile + 2];        // row begin offsets relative to the tile's first entry
   uint64_t key[kHvTile + 2];      // per-row partial argmax keys (rows split across threads)
   uint64_t bar;
 };
@@ -149,7 +153,7 @@ __global__ void __launch_bounds__(kHvBlock) k_heavy(int64_t n, int64_t nnz,
     int64_t r = x0 + k;
     int64_t b = r <= n ? __ldg(row_ptr + r) - ebase : nnz;
     int64_t rel = b - y0;
-    S.rb[k] = rel < -1 ? -1 : (rel > kHvTile + 1 ? kHvTile + 1 : (int32_t)rel);
+    S.rb[k] = (int16_t)(rel < -1 ? -1 : (rel > kHvTile + 1 ? kHvTile + 1 : rel));
     S.key[k] = 0;
   }
   __syncthreads();

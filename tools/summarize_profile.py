@@ -31,6 +31,8 @@ PHASE = {
     "UnitsIn": "rows_skew", "BucketsIn": "rows_skew", "k_part_count": "rows_skew", "k_part_write": "rows_skew",
     "k_fb_jobs": "rows_skew", "k_bucket_fallback": "rows_skew", "k_dense_accum": "rows_skew",
     "k_block_desc": "rows", "k_block_ends": "rows", "k_rows": "rows", "BlkCntIn": "rows",
+    "k_pieces": "rows", "k_tiers": "rows", "k_wide_list": "rows", "k_expand": "expand",
+    "k_bucket_blocks": "rows_skew",
     "k_place": "place",
 }
 
