@@ -151,8 +151,9 @@ __global__ void k_big_rows(Layout L, int64_t big_thr, int32_t *__restrict__ big_
 constexpr int kPartHist = 8192;  // buckets per skewed row (bounds the partition's smem tables)
 constexpr int kUnit = 65536;     // member-edge positions per partition CTA
 
-__host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c) {
-  int64_t nb = (U + kBucketAvg - 1) / kBucketAvg;
+__host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c, bool rbm = false) {
+  const int64_t avg = rbm ? kRbmBinAvg : kBucketAvg;
+  int64_t nb = (U + avg - 1) / avg;
   if (nb > kPartHist) nb = kPartHist;
   if (nb > n_c) nb = n_c;
   return nb < 1 ? 1 : nb;
@@ -165,6 +166,7 @@ struct BlockCountIn {
   const int64_t *S;  // exclusive scan of RowWeightIn
   bool dense;
   int64_t big_thr;
+  bool rbm;  // class-1 rows are single-row bitmap-rank items
   __device__ __forceinline__ int cls(int64_t U) const {
     return U <= kPieceMax ? 0 : (U <= big_thr ? 1 : 2);
   }
@@ -172,7 +174,8 @@ struct BlockCountIn {
     if (!L.active(a)) return 0;
     const int64_t U = L.U(a);
     const int c = cls(U);
-    if (c == 2) return dense ? dense_chunks(L.n_c) : row_buckets(U, L.n_c);
+    if (c == 2) return dense ? dense_chunks(L.n_c) : row_buckets(U, L.n_c, rbm);
+    if (c == 1 && rbm) return 1;
     if (a == L.a_lo || cls(L.U(a - 1)) != c) return 1;
     const int64_t win = c == 0 ? kPieceWin : kWin;  // rows of one class are contiguous in S
     return (S[a] / win) != (S[a - 1] / win) ? 1 : 0;
@@ -181,7 +184,7 @@ struct BlockCountIn {
 
 // descriptors of PIECE / SMALL blocks and DENSE chunks (BUCKET blocks: k_bucket_blocks)
 __global__ void k_block_desc(Layout L, const int64_t *__restrict__ blk_ptr, const int32_t *__restrict__ big_idx,
-                             bool dense, BlockDesc *__restrict__ blk) {
+                             bool dense, bool rbm, BlockDesc *__restrict__ blk) {
   int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (a >= L.n_c) return;
   int64_t b0 = blk_ptr[a], b1 = blk_ptr[a + 1];
@@ -190,7 +193,10 @@ __global__ void k_block_desc(Layout L, const int64_t *__restrict__ blk_ptr, cons
     if (dense)
       for (int64_t k = b0; k < b1; ++k) blk[k] = BlockDesc{B_DENSE, (int32_t)a, (int32_t)a + 1, (int32_t)(k - b0)};
   } else {
-    blk[b0] = BlockDesc{L.U(a) <= kPieceMax ? B_PIECE : B_SMALL, (int32_t)a, -1, 0};
+    const int64_t U = L.U(a);
+    if (U <= kPieceMax) blk[b0] = BlockDesc{B_PIECE, (int32_t)a, -1, 0};
+    else if (rbm) blk[b0] = BlockDesc{B_RBM, (int32_t)a, (int32_t)a + 1, 0};
+    else blk[b0] = BlockDesc{B_SMALL, (int32_t)a, -1, 0};
   }
 }
 // row1 of PIECE / SMALL blocks = first row of the next block (or the end of the range)
@@ -228,7 +234,8 @@ constexpr int kWarpBins = (int)((kWarpRowMax + 31) / 32);  // row_buckets(kWarpR
 struct BucketsIn {
   Layout L;
   const int32_t *big_list;
-  __device__ __forceinline__ int64_t operator()(int64_t h) const { return row_buckets(L.U(big_list[h]), L.n_c); }
+  bool rbm;
+  __device__ __forceinline__ int64_t operator()(int64_t h) const { return row_buckets(L.U(big_list[h]), L.n_c, rbm); }
 };
 
 // Segment -> owner table: out[k] = h for k in [ptr[h], ptr[h+1]) (a warp per
@@ -742,7 +749,7 @@ __global__ void k_bucket_blocks(int64_t nbig, int64_t nbkt, const int32_t *__res
                                 const int64_t *__restrict__ blk_ptr, BlockDesc *__restrict__ blk,
                                 int64_t *__restrict__ jobs, unsigned *__restrict__ njobs,
                                 int32_t *__restrict__ fb_cnt, int64_t *__restrict__ fb_off,
-                                unsigned long long *__restrict__ fb_total) {
+                                unsigned long long *__restrict__ fb_total, int64_t fb_thr) {
   int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= nbkt) return;
   const int64_t h = bin_row[k];
@@ -750,7 +757,7 @@ __global__ void k_bucket_blocks(int64_t nbig, int64_t nbkt, const int32_t *__res
   const int32_t a = big_list[h];
   blk[blk_ptr[a] + (k - b0)] = BlockDesc{B_BUCKET, a, a + 1, (int32_t)(k - b0)};
   const int64_t c = bkt_n[k];
-  if (c > kCap) {
+  if (c > fb_thr) {
     unsigned j = atomicAdd(njobs, 1u);
     jobs[j] = k;
     fb_off[k] = (int64_t)atomicAdd(fb_total, (unsigned long long)c);
@@ -787,11 +794,13 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
                         const unsigned *__restrict__ bkt_n,
                         const int32_t *__restrict__ fb_cnt, int32_t *__restrict__ blk_cnt,
                         int64_t *__restrict__ grp_end,
-                        WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, unsigned *__restrict__ list_n,
+                        WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, RbmItem *__restrict__ list_r,
+                        unsigned *__restrict__ list_n, bool rbm,
                         const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
   const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  int tier = -1;  // 0 warp, 1 CTA
+  int tier = -1;  // 0 warp, 1 CTA, 2 bitmap-rank CTA
   WorkItem it{0, (int32_t)bi, 0, 0, 0};
+  RbmItem ri{};
   if (bi < nblocks) {
     const BlockDesc d = blk[bi];
     it.row0 = d.row0;
@@ -803,6 +812,26 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
       it.base = p0 - L.upos(L.a_lo);
       it.n = (int32_t)(L.upos(d.row1) - p0);
       it.R = d.row1 - d.row0;
+    } else if (d.kind == B_RBM || (rbm && d.kind == B_BUCKET)) {
+      tier = 2;
+      ri.bi = (int32_t)bi;
+      ri.row = d.row0;
+      if (d.kind == B_RBM) {
+        const int64_t p0 = L.upos(d.row0);
+        ri.src = p0 - L.upos(L.a_lo);
+        ri.n = (int32_t)(L.upos(d.row0 + 1) - p0);
+        ri.lo = 0;
+        ri.hi = (int32_t)L.n_c;
+        ri.bk = -1;
+      } else {
+        const int64_t h = big_idx[d.row0];
+        const int64_t b0 = bkt_ptr[h], nb = bkt_ptr[h + 1] - b0, bk = b0 + d.sub;
+        ri.src = bkt_off[bk];
+        ri.n = (int32_t)bkt_n[bk];
+        ri.lo = (int32_t)bin_lower(d.sub, nb, L.n_c);
+        ri.hi = (int32_t)bin_lower(d.sub + 1, nb, L.n_c);
+        ri.bk = (int32_t)bk;
+      }
     } else if (d.kind != B_BUCKET) tier = 1;
     else {
       const int64_t h = big_idx[d.row0];
@@ -823,7 +852,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
   }
   const int lane = threadIdx.x & 31;
 #pragma unroll
-  for (int q = 0; q < 2; ++q) {
+  for (int q = 0; q < 3; ++q) {
     const unsigned m = __ballot_sync(0xffffffffu, tier == q);
     if (!m) continue;
     const int leader = __ffs(m) - 1;
@@ -832,7 +861,8 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
     base = __shfl_sync(0xffffffffu, base, leader);
     if (tier == q) {
       const unsigned pos = base + __popc(m & ((1u << lane) - 1));
-      if (q) list_c[pos] = (int32_t)bi;
+      if (q == 2) list_r[pos] = ri;
+      else if (q) list_c[pos] = (int32_t)bi;
       else list_w[pos] = it;
     }
   }
@@ -1021,12 +1051,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t n_out = a_hi - a_lo;  // rows produced by this call
   Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi};
   const bool dense = n_c <= kDenseMax;
-  const int64_t big_thr = big_threshold_host(dense);
+  // bitmap-rank items replace the bin pieces when the key range fits the
+  // shared-memory bitmap (HEC_NO_RBM: test / tuning hook for the bin-piece path)
+  const bool rbm = !dense && n_c <= kRbmRange && getenv("HEC_NO_RBM") == nullptr;
+  const int64_t big_thr = rbm ? (int64_t)kRbmRow : big_threshold_host(dense);
   k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_thr, big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));
   HEC_LAUNCH_CHECK();
   HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, big_thr}, PtrOut{Sw}, st[2], Sw + n_c));
-  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c));
+  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr, rbm}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 4, counts + 0, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
   phase_end(ctx, ph);
   int64_t r0[5];
@@ -1041,7 +1074,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)kDenseUnit : (int64_t)kUnit,
                                              dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
                          st[4], unit_ptr + nbig));
-    if (!dense) HEC_TRY(chained_scan(ctx, nbig, BucketsIn{L, big_list}, PtrOut{bkt_ptr}, st[5], bkt_ptr + nbig));
+    if (!dense) HEC_TRY(chained_scan(ctx, nbig, BucketsIn{L, big_list, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + nbig));
     HEC_CUDA_TRY(cudaMemcpyAsync(scal + 5, unit_ptr + nbig, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
     if (!dense) HEC_CUDA_TRY(cudaMemcpyAsync(scal + 6, bkt_ptr + nbig, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
   }
@@ -1055,6 +1088,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
+                ws_bytes(nblocks + 1, sizeof(RbmItem)) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
@@ -1077,6 +1111,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   WorkItem *list_w = arena_take<WorkItem>(W2, nblocks + 1);   // warp-tier work items
   int32_t *list_c = arena_take<int32_t>(W2, nblocks + 1);     // CTA-tier blocks
   int32_t *list_wide = arena_take<int32_t>(W2, nblocks + 1);  // blocks flagged for 64-bit sums
+  RbmItem *list_r = arena_take<RbmItem>(W2, nblocks + 1);     // bitmap-rank items
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1098,7 +1133,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     phase_end(ctx, phx);
   }
   HEC_CUDA_TRY(cudaMemsetAsync(need_wide, 0, sizeof(int32_t) * (nblocks + 1), s));
-  k_block_desc<<<nblk(n_c, 256), 256, 0, s>>>(L, blk_ptr, big_idx, dense, blk);
+  k_block_desc<<<nblk(n_c, 256), 256, 0, s>>>(L, blk_ptr, big_idx, dense, rbm, blk);
   HEC_LAUNCH_CHECK();
 
   RowsArgs A{};
@@ -1184,7 +1219,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_LAUNCH_CHECK();
     k_bucket_blocks<<<nblk(nbkt, 256), 256, 0, s>>>(nbig, nbkt, big_list, bkt_ptr, bin_row, bkt_cnt, blk_ptr, blk, jobs,
                                                    counts + 4, fb_cnt, fb_off,
-                                                   reinterpret_cast<unsigned long long *>(scal + 10));
+                                                   reinterpret_cast<unsigned long long *>(scal + 10),
+                                                   rbm ? INT64_MAX : (int64_t)kCap);
     HEC_LAUNCH_CHECK();
     HEC_CUDA_TRY(cudaMemcpyAsync(scal + 9, counts + 4, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
     int64_t rj[1];
@@ -1203,14 +1239,20 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.fb_off = fb_off;
     A.fb_b = fb_b;
     A.fb_w = fb_w;
+    A.fb_total = reinterpret_cast<unsigned long long *>(scal + 10);
+    A.fb_off_w = fb_off;
+    A.fb_cnt_w = fb_cnt;
+    A.fb_b_w = fb_b;
+    A.fb_w_w = fb_w;
   }
   phase_end(ctx, ph_skew);
-  // counts: [5] pieces ticket [6] warp list [7] CTA list [8] wide list
+  // counts: [5] pieces ticket [8] wide list [10] warp list [11] CTA list [12] bitmap-rank list
+  //         [13] bitmap-rank ticket
   if (nblocks > 0) {
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, counts + 6, vw64, err);
+                                              list_c, list_r, counts + 10, rbm, vw64, err);
     HEC_LAUNCH_CHECK();
   }
 
@@ -1227,11 +1269,34 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
   const int ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
   A.items = list_w;
-  A.nlist = counts + 6;
+  A.nlist = counts + 10;
+  unsigned long long *pstats = nullptr;
+  if (getenv("HEC_PIECE_STATS")) {
+    HEC_TRY(dev_alloc(ctx, (void **)&pstats, 16 * sizeof(unsigned long long)));
+    HEC_CUDA_TRY(cudaMemsetAsync(pstats, 0, 16 * sizeof(unsigned long long), s));
+    A.pstats = pstats;
+  }
   HEC_TRY(launch_pieces(ctx, A, counts + 5));
+  if (pstats) {
+    unsigned long long h[16];
+    HEC_CUDA_TRY(cudaMemcpyAsync(h, pstats, sizeof h, cudaMemcpyDeviceToHost, s));
+    HEC_CUDA_TRY(cudaStreamSynchronize(s));
+    fprintf(stderr, "[pieces n_c=%lld]", (long long)n_c);
+    for (int c = 0; c < 8; ++c) fprintf(stderr, " %s%d:%llu/%llu", c < 4 ? "bin" : "row", 32 << (c & 3), h[2 * c], h[2 * c + 1]);
+    fprintf(stderr, "\n");
+    dev_free(ctx, pstats);
+    A.pstats = nullptr;
+  }
   A.list = list_c;
-  A.nlist = counts + 7;
+  A.nlist = counts + 11;
   HEC_TRY(launch_rows(ctx, A, false));
+  if (rbm) {
+    A.ritems = list_r;
+    A.nlist = counts + 12;
+    A.ticket = counts + 13;
+    HEC_TRY(launch_rbm(ctx, A));
+    A.ticket = counts + 1;
+  }
   phase_end(ctx, ph_rows);
   if (trace) {
     std::vector<long long> h(4 * nblocks);
@@ -1262,6 +1327,10 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_TRY(read_scalars(ctx, scal, 13, r2));
   }
   out->nnz_c = r2[12];
+  if ((int)(r2[0] & 0xffffffff) & ERR_INTERNAL) {
+    set_error("build_coarse_graph: internal error (bitmap-rank key outside its bin)");
+    return HEC_ECUDA;
+  }
   if ((int)(r2[0] & 0xffffffff) & ERR_OVERFLOW) {
     set_error("build_coarse_graph: a coarse weight exceeds INT32_MAX");
     return HEC_EOVERFLOW;

@@ -24,10 +24,17 @@ constexpr int kPieceRows = kPieceWin / kPieceRowW;  // rows per piece (all start
 constexpr int kPieceCap = 256;     // entries per warp piece
 constexpr int kDenseMax = 32768;   // n_c bound of the DENSE skew path
 constexpr int32_t kEmpty = -1;
+// Bitmap-rank items (construct_rbm.cu), used in BUCKET mode when n_c <= kRbmRange:
+// rows with kPieceMax < U <= kRbmRow are single-row items; larger rows are
+// partitioned into bins of ~kRbmBinAvg entries, each bin an item.
+constexpr int64_t kRbmRange = 917504;  // keys covered by the shared-memory bitmap
+constexpr int kRbmRow = 4096;
+constexpr int kRbmBinAvg = 2048;
+constexpr int kRbmCap = 4096;          // distinct keys per rank window
 
-enum : int32_t { B_SMALL = 0, B_BUCKET = 1, B_DENSE = 2, B_PIECE = 3 };
+enum : int32_t { B_SMALL = 0, B_BUCKET = 1, B_DENSE = 2, B_PIECE = 3, B_RBM = 4 };
 __host__ __device__ __forceinline__ bool rows_kind(int32_t k) { return k == B_SMALL || k == B_PIECE; }
-enum : int { ERR_LABEL = 1, ERR_OVERFLOW = 2, ERR_WIDE = 4 };
+enum : int { ERR_LABEL = 1, ERR_OVERFLOW = 2, ERR_WIDE = 4, ERR_INTERNAL = 8 };
 
 inline unsigned nblk(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
 
@@ -224,6 +231,31 @@ struct WorkItem {
   int32_t R;
 };
 
+// A bitmap-rank item (construct_rbm.cu), self-contained so a CTA prefetches it:
+// entries [src, src + n) of sc_col/sc_wgt (B_RBM whole row) or pb_g/pw_g (bin),
+// keys in [lo, hi); row = the coarse row (its self entries are dropped).
+struct RbmItem {
+  int64_t src;
+  int32_t n, row, lo, hi, bi, bk;  // bk: bin index (-1 for a whole row)
+};
+
+// smallest b in [0, n_c] whose partition bin floor(b * nb / n_c) (float, clamped
+// to nb - 1 -- the exact function k_part_* use) is >= k
+__device__ __forceinline__ int64_t bin_lower(int64_t k, int64_t nb, int64_t n_c) {
+  if (k <= 0) return 0;
+  if (k >= nb) return n_c;
+  const float scale = (float)nb / (float)n_c;
+  int64_t lo = 0, hi = n_c;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi) >> 1;
+    int bk = (int)__fmul_rz((float)mid, scale);
+    bk = bk < nb - 1 ? bk : (int)(nb - 1);
+    if (bk >= k) hi = mid;
+    else lo = mid + 1;
+  }
+  return lo;
+}
+
 struct BlockDesc {
   int32_t kind;
   int32_t row0;  // first row (SMALL) / the row (BUCKET, DENSE)
@@ -260,6 +292,10 @@ struct RowsArgs {
   const int32_t *fb_cnt;            // fallback unique count per bucket (-1: not overflowed)
   const int64_t *fb_off;            // fallback scratch offset per bucket
   const int32_t *fb_b, *fb_w;
+  // bitmap-rank items with several rank windows stage to the fallback scratch
+  unsigned long long *fb_total;
+  int64_t *fb_off_w;
+  int32_t *fb_cnt_w, *fb_b_w, *fb_w_w;
   // DENSE mode
   unsigned long long *dense;        // [nbig][n_c] sums, then staged pairs
   // outputs (row-indexed outputs start at row L.a_lo)
@@ -267,8 +303,10 @@ struct RowsArgs {
   int32_t *col_c, *wgt_c, *vwgt_c;
   int *err;
   long long *trace;  // debug: per block (compute cycles, 0, kind, T); nullable
+  unsigned long long *pstats;  // debug (HEC_PIECE_STATS): warp items / entries per kind x size class; nullable
   const int32_t *list;    // blocks of this launch (a tier list)
   const WorkItem *items;  // warp tier: the same, as work items
+  const RbmItem *ritems;  // bitmap-rank tier
   const unsigned *nlist;  // device count of `list` / `items`
 };
 
@@ -277,5 +315,6 @@ struct RowsArgs {
 int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide);
 int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket);  // construct_pieces.cu
 int launch_place(hec_ctx *ctx, const RowsArgs &A);
+int launch_rbm(hec_ctx *ctx, const RowsArgs &A);  // construct_rbm.cu
 
 }  // namespace hec

@@ -316,18 +316,23 @@ __device__ __forceinline__ int group_bitmap(const int32_t (&b)[J], const int32_t
 // Small bin groups (n <= 32 J entries, J <= 2): rank by bit-serial ballots.
 // For each own key, eq[s] / less[s] are the lanes whose slot-s key equals /
 // is below it on the bits seen so far (most significant first, only the bits
-// where the group's keys differ).  Duplicates are merged with one
-// __reduce_add_sync per slot over the equal-key partition (labelled-partition
-// reduction); the first copy (lowest slot, then lane) writes (key, sum) at its
-// rank among the distinct keys -- no sorting network, no shared memory.
+// where the group's keys differ).  Equal keys share a rank among the distinct
+// keys, so duplicates merge with one shared-memory atomicAdd at that rank and
+// the first copy (lowest slot, then lane) writes (key, sum) -- no sorting
+// network.  (A labelled-partition __reduce_add_sync was measured to serialise
+// per distinct mask.)
 template <int J>
 __device__ __forceinline__ int group_ballot(const int32_t (&b)[J], const int32_t (&w)[J], int32_t mn, int32_t mx,
-                                            int32_t *__restrict__ dst_b, int32_t *__restrict__ dst_w, int64_t base) {
+                                            int32_t *__restrict__ val, int32_t *__restrict__ dst_b,
+                                            int32_t *__restrict__ dst_w, int64_t base) {
   const int lane = threadIdx.x & 31;
   const unsigned lt = (1u << lane) - 1u;
   unsigned vm[J];
 #pragma unroll
-  for (int s = 0; s < J; ++s) vm[s] = __ballot_sync(0xffffffffu, b[s] >= 0);
+  for (int s = 0; s < J; ++s) {
+    vm[s] = __ballot_sync(0xffffffffu, b[s] >= 0);
+    val[lane + 32 * s] = 0;
+  }
   unsigned eq[J][J], less[J][J];
 #pragma unroll
   for (int t = 0; t < J; ++t)
@@ -360,28 +365,24 @@ __device__ __forceinline__ int group_ballot(const int32_t (&b)[J], const int32_t
   }
 #pragma unroll
   for (int s = 0; s < J; ++s) lm[s] = __ballot_sync(0xffffffffu, lead[s]);
-  int red[J];
-#pragma unroll
-  for (int s = 0; s < J; ++s) red[s] = __reduce_add_sync(b[s] >= 0 ? eq[s][s] : (1u << lane), w[s]);
-  int T = 0;
+  int T = 0, rank[J];
 #pragma unroll
   for (int s = 0; s < J; ++s) T += __popc(lm[s]);
+  __syncwarp();
 #pragma unroll
   for (int t = 0; t < J; ++t) {
-    int rank = 0, sum = 0;
+    rank[t] = 0;
 #pragma unroll
-    for (int s = 0; s < J; ++s) {
-      rank += __popc(less[t][s] & lm[s]);
-      const unsigned e = b[t] >= 0 ? eq[t][s] : 0u;
-      const int src = e ? __ffs(e) - 1 : lane;
-      const int v = __shfl_sync(0xffffffffu, red[s], src);
-      sum += e ? v : 0;
-    }
-    if (lead[t]) {
-      dst_b[base + rank] = b[t];
-      dst_w[base + rank] = sum;
-    }
+    for (int s = 0; s < J; ++s) rank[t] += __popc(less[t][s] & lm[s]);
+    if (b[t] >= 0) atomicAdd(&val[rank[t]], w[t]);
   }
+  __syncwarp();
+#pragma unroll
+  for (int t = 0; t < J; ++t)
+    if (lead[t]) {
+      dst_b[base + rank[t]] = b[t];
+      dst_w[base + rank[t]] = val[rank[t]];
+    }
   __syncwarp();
   return T;
 }
@@ -417,7 +418,7 @@ __device__ __forceinline__ int group_run(WarpTab &S, int n, int32_t *__restrict_
   if (wsum > 0x7fffffffLL) return -1;
   if (mx < 0) return 0;
   if constexpr (J <= 2) {
-    return group_ballot<J>(b, w, mn, mx, src_b, src_w, base);
+    return group_ballot<J>(b, w, mn, mx, S.g.val, src_b, src_w, base);
   } else if ((int64_t)mx - mn < kGrpBits) {
     return group_bitmap<J>(b, w, mn, ((mx - mn) >> 5) + 1, S.g, src_b, src_w, base);
   }
@@ -469,6 +470,11 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
     } else {  // bin group with <= kPieceCap entries (self entries already dropped)
       src_b = A.pb_g;
       src_w = A.pw_g;
+    }
+    if (A.pstats && lane == 0) {
+      const int c = (R > 0 ? 4 : 0) + (n <= 32 ? 0 : n <= 64 ? 1 : n <= 128 ? 2 : 3);
+      atomicAdd(A.pstats + 2 * c, 1ull);
+      atomicAdd(A.pstats + 2 * c + 1, (unsigned long long)n);
     }
     int T;
     if (R == 0) {

@@ -341,29 +341,15 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
   }
 }
 
-// Placement: each warp sweeps 32 consecutive blocks (one per lane for the
-// metadata) and copies the non-empty ones cooperatively to their final CSR
-// position (bin blocks inside a group are empty; a CTA or warp per block
-// would be launch- and latency-bound).
+// Placement: each warp owns 32 consecutive blocks (one per lane).  The
+// blocks' outputs are contiguous in the final CSR, so the warp copies the
+// whole range flattened: output element j finds its block by a 5-step shuffle
+// search over the lanes' output offsets and reads from that block's staging
+// (4 elements per lane in flight; per-block serial copies were latency-bound).
+// Row offsets and vertex weights are then fixed per block.
 constexpr int kPlaceT = 256;
-__device__ __forceinline__ void warp_copy(int32_t *__restrict__ dc, int32_t *__restrict__ dw,
-                                          const int32_t *__restrict__ sc, const int32_t *__restrict__ sw, int T,
-                                          int lane) {
-  // four loads per lane in flight before the stores (the copy is latency-bound)
-  for (int q0 = 0; q0 < T; q0 += 128) {
-    int32_t c[4], w[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int q = q0 + lane + 32 * j;
-      if (q < T) { c[j] = __ldcs(sc + q); w[j] = __ldcs(sw + q); }
-    }
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int q = q0 + lane + 32 * j;
-      if (q < T) { dc[q] = c[j]; dw[q] = w[j]; }
-    }
-  }
-}
+enum : int { SRC_SC = 0, SRC_PB = 1, SRC_FB = 2, SRC_DENSE = 3 };
+
 __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t b0 = ((int64_t)blockIdx.x * (kPlaceT / 32) + (threadIdx.x >> 5)) * 32;
@@ -371,53 +357,72 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   const Layout &L = A.L;
   const int64_t mine = b0 + lane;
   BlockDesc dm{-1, 0, 0, 0};
-  int64_t Om = 0;
-  int Tm = 0;
-  bool need = false;
+  int64_t Om = A.blk_off[A.nblocks - 1] + A.blk_cnt[A.nblocks - 1];  // past the end: empty
+  int Tm = 0, src = SRC_SC;
+  int64_t soff = 0;
   if (mine < A.nblocks) {
     dm = A.blk[mine];
     Om = A.blk_off[mine];
     Tm = A.blk_cnt[mine];
-    need = Tm > 0 || rows_kind(dm.kind) || dm.sub == 0;
+    if (rows_kind(dm.kind) || dm.kind == B_RBM) {  // staged over the expansion staging
+      soff = L.upos(dm.row0) - L.upos(L.a_lo);
+    } else if (dm.kind == B_DENSE) {
+      src = SRC_DENSE;
+      soff = 2 * ((int64_t)A.big_idx[dm.row0] * L.n_c + (int64_t)dm.sub * kCap);
+    } else if (Tm > 0) {
+      const int64_t bk = A.bkt_ptr[A.big_idx[dm.row0]] + dm.sub;
+      if (A.fb_cnt[bk] >= 0) { src = SRC_FB; soff = A.fb_off[bk]; }
+      else { src = SRC_PB; soff = A.bkt_off[bk]; }
+    }
   }
   if (mine == A.nblocks - 1) A.row_ptr_c[L.a_hi - L.a_lo] = Om + Tm;
-  unsigned m = __ballot_sync(0xffffffffu, need);
+  const int64_t O0 = __shfl_sync(0xffffffffu, Om, 0);
+  const int64_t total = __shfl_sync(0xffffffffu, Om + Tm, 31) - O0;
+  const int32_t *dn = reinterpret_cast<const int32_t *>(A.dense);
+  for (int64_t j0 = 0; j0 < total; j0 += 128) {
+    int32_t c[4], w[4];
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      const int64_t j = j0 + lane + 32 * t;
+      int k = 0;  // last lane whose block starts at or before j
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const int64_t Oc = __shfl_sync(0xffffffffu, Om, k + step);
+        if (Oc - O0 <= j) k += step;
+      }
+      const int sk = __shfl_sync(0xffffffffu, src, k);
+      const int64_t sb = __shfl_sync(0xffffffffu, soff, k);
+      const int64_t r = j - (__shfl_sync(0xffffffffu, Om, k) - O0);  // index inside the block
+      if (j < total) {
+        if (sk == SRC_SC) { c[t] = __ldcs(A.sc_col + sb + r); w[t] = __ldcs(A.sc_wgt + sb + r); }
+        else if (sk == SRC_PB) { c[t] = __ldcs(A.pb_g + sb + r); w[t] = __ldcs(A.pw_g + sb + r); }
+        else if (sk == SRC_FB) { c[t] = __ldcs(A.fb_b + sb + r); w[t] = __ldcs(A.fb_w + sb + r); }
+        else { c[t] = dn[sb + 2 * r]; w[t] = dn[sb + 2 * r + 1]; }  // interleaved (b, w) pairs
+      }
+    }
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      const int64_t j = j0 + lane + 32 * t;
+      if (j < total) {
+        A.col_c[O0 + j] = c[t];
+        A.wgt_c[O0 + j] = w[t];
+      }
+    }
+  }
+  // per-block metadata: row offsets (rows blocks) / row start + vertex weight (skewed rows)
+  unsigned m = __ballot_sync(0xffffffffu, mine < A.nblocks && (rows_kind(dm.kind) || dm.sub == 0));
   while (m) {
-    const int j = __ffs(m) - 1;
+    const int jl = __ffs(m) - 1;
     m &= m - 1;
-    BlockDesc d;
-    d.kind = __shfl_sync(0xffffffffu, dm.kind, j);
-    d.row0 = __shfl_sync(0xffffffffu, dm.row0, j);
-    d.row1 = __shfl_sync(0xffffffffu, dm.row1, j);
-    d.sub = __shfl_sync(0xffffffffu, dm.sub, j);
-    const int64_t O = __shfl_sync(0xffffffffu, Om, j);
-    const int T = __shfl_sync(0xffffffffu, Tm, j);
-    if (rows_kind(d.kind)) {
-      const int64_t P0 = L.upos(d.row0) - L.upos(L.a_lo);
-      warp_copy(A.col_c + O, A.wgt_c + O, A.sc_col + P0, A.sc_wgt + P0, T, lane);
-      for (int a = d.row0 + lane; a < d.row1; a += 32) A.row_ptr_c[a - L.a_lo] += O;
-    } else {
-      if (d.kind == B_DENSE) {
-        const int32_t *st = reinterpret_cast<const int32_t *>(A.dense + (int64_t)A.big_idx[d.row0] * L.n_c +
-                                                              (int64_t)d.sub * kCap);
-        for (int q = lane; q < T; q += 32) {
-          A.col_c[O + q] = st[2 * q];
-          A.wgt_c[O + q] = st[2 * q + 1];
-        }
-      } else if (T > 0) {
-        const int64_t bk = A.bkt_ptr[A.big_idx[d.row0]] + d.sub;
-        if (A.fb_cnt[bk] >= 0) {
-          const int64_t f0 = A.fb_off[bk];
-          warp_copy(A.col_c + O, A.wgt_c + O, A.fb_b + f0, A.fb_w + f0, T, lane);
-        } else {
-          const int64_t q0 = A.bkt_off[bk];
-          warp_copy(A.col_c + O, A.wgt_c + O, A.pb_g + q0, A.pw_g + q0, T, lane);
-        }
-      }
-      if (d.sub == 0 && lane == 0) {  // the row's first block: row start and vertex weight
-        A.row_ptr_c[d.row0 - L.a_lo] = O;
-        A.vwgt_c[d.row0 - L.a_lo] = (int32_t)A.vw64[d.row0];  // bound checked by k_tiers
-      }
+    const int kind = __shfl_sync(0xffffffffu, dm.kind, jl);
+    const int32_t row0 = __shfl_sync(0xffffffffu, dm.row0, jl);
+    const int32_t row1 = __shfl_sync(0xffffffffu, dm.row1, jl);
+    const int64_t O = __shfl_sync(0xffffffffu, Om, jl);
+    if (rows_kind(kind)) {
+      for (int a = row0 + lane; a < row1; a += 32) A.row_ptr_c[a - L.a_lo] += O;
+    } else if (lane == 0) {  // the row's first block: row start and vertex weight
+      A.row_ptr_c[row0 - L.a_lo] = O;
+      A.vwgt_c[row0 - L.a_lo] = (int32_t)A.vw64[row0];  // bound checked by k_tiers
     }
   }
 }

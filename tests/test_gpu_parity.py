@@ -180,11 +180,17 @@ def test_construct_random_labels(P, ctx):
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
+@pytest.mark.parametrize("path", ["rbm", "bins"])
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
-def test_construct_size_classes(P, ctx, nc):
+def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     """R-MAT with random labels into nc aggregates: few labels give huge rows
     (DENSE when nc <= 32768, key-range buckets otherwise), many labels give
-    warp-piece and CTA-window rows."""
+    warp-piece and CTA-window rows.  path=bins forces the key-range bin pieces
+    instead of the bitmap-rank items (HEC_NO_RBM test hook)."""
+    if path == "bins":
+        if nc <= 32768:
+            pytest.skip("DENSE mode: no bitmap-rank items")
+        monkeypatch.setenv("HEC_NO_RBM", "1")
     rng = np.random.default_rng(15 + nc)
     g = gg.rmat(14 if nc < 20000 else 17, 16)
     g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
@@ -214,9 +220,12 @@ def test_construct_wide_piece_keys(P, ctx, monkeypatch):
     check_hierarchy(P, ctx, gg.config(2), 1000)
 
 
-def test_construct_duplicate_heavy_rows(P, ctx):
+@pytest.mark.parametrize("path", ["rbm", "bins"])
+def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
     """Skewed rows whose entries repeat few keys: key-range buckets far above a
     warp piece (CTA tier) and above a CTA block (fallback), next to ordinary rows."""
+    if path == "bins":
+        monkeypatch.setenv("HEC_NO_RBM", "1")
     rng = np.random.default_rng(22)
     n = 60000
     hub_targets = rng.integers(0, n, 4000)
@@ -235,6 +244,34 @@ def test_construct_duplicate_heavy_rows(P, ctx):
     M[:8] = 0  # all hubs in one coarse row
     M[hub_targets] = rng.integers(1, 40, hub_targets.size)  # targets collapse onto few keys
     M[rng.permutation(np.setdiff1d(np.arange(8, n), hub_targets))[:nc]] = np.arange(nc)
+    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+    assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
+
+
+def test_construct_rbm_rank_windows(P, ctx):
+    """Bitmap-rank bins with more distinct keys than one rank window (kRbmCap =
+    4096): a skewed row whose neighbours map densely into the low key range, so
+    its first bins hold ~7000 distinct keys each (several rank windows, staged
+    to the fallback scratch), next to whole-row items and warp pieces."""
+    rng = np.random.default_rng(23)
+    n, nc = 100000, 70000
+    edges = {}
+    hubs = np.arange(6)
+    nbrs = rng.choice(np.arange(6, n), 24000, replace=False)
+    for h in hubs:
+        for v in nbrs[h * 4000:(h + 1) * 4000]:
+            edges[(int(h), int(v))] = 1 + int(v) % 5
+    for _ in range(2 * n):
+        u, v = rng.integers(0, n, 2)
+        if u != v:
+            edges[(min(u, v), max(u, v))] = int(rng.integers(1, 9))
+    g = gg.from_edges(n, [(u, v, w) for (u, v), w in edges.items()])
+    M = np.empty(n, np.int32)
+    rest = np.setdiff1d(np.arange(n), np.concatenate([hubs, nbrs]))
+    M[hubs] = 0
+    M[nbrs] = 1 + np.arange(nbrs.size) % 20000  # hub row: ~20k distinct keys in [1, 20000]
+    M[rest] = rng.integers(0, nc, rest.size)
+    M[rng.permutation(rest)[:nc]] = np.arange(nc)
     cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
