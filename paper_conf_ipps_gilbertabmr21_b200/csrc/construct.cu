@@ -795,7 +795,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
                         const int32_t *__restrict__ fb_cnt, int32_t *__restrict__ blk_cnt,
                         int64_t *__restrict__ grp_end,
                         WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, RbmItem *__restrict__ list_r,
-                        unsigned *__restrict__ list_n, bool rbm,
+                        RbmItem *__restrict__ list_r2, unsigned *__restrict__ list_n, bool rbm,
                         const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
   const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   int tier = -1;  // 0 warp, 1 CTA, 2 bitmap-rank CTA
@@ -832,6 +832,8 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
         ri.hi = (int32_t)bin_lower(d.sub + 1, nb, L.n_c);
         ri.bk = (int32_t)bk;
       }
+      // size class (k_tiers lists: list_r front/back, list_r2 front/back)
+      tier = ri.n <= kHrMax0 ? 2 : ri.n <= kHrMax1 ? 3 : ri.n <= kHrMax2 ? 4 : 5;
     } else if (d.kind != B_BUCKET) tier = 1;
     else {
       const int64_t h = big_idx[d.row0];
@@ -851,17 +853,22 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
     }
   }
   const int lane = threadIdx.x & 31;
+  // list_n: [0] warp [1] CTA [2] list_r front [4] list_r back [5] list_r2 front [6] list_r2 back
 #pragma unroll
-  for (int q = 0; q < 3; ++q) {
+  for (int q = 0; q < 6; ++q) {
     const unsigned m = __ballot_sync(0xffffffffu, tier == q);
     if (!m) continue;
     const int leader = __ffs(m) - 1;
+    const int slot = q < 3 ? q : q + 1;
     unsigned base = 0;
-    if (lane == leader) base = atomicAdd(list_n + q, (unsigned)__popc(m));
+    if (lane == leader) base = atomicAdd(list_n + slot, (unsigned)__popc(m));
     base = __shfl_sync(0xffffffffu, base, leader);
     if (tier == q) {
-      const unsigned pos = base + __popc(m & ((1u << lane) - 1));
+      const int64_t pos = base + __popc(m & ((1u << lane) - 1));
       if (q == 2) list_r[pos] = ri;
+      else if (q == 3) list_r[nblocks - pos] = ri;  // lists hold nblocks + 1 items
+      else if (q == 4) list_r2[pos] = ri;
+      else if (q == 5) list_r2[nblocks - pos] = ri;
       else if (q) list_c[pos] = (int32_t)bi;
       else list_w[pos] = it;
     }
@@ -1088,7 +1095,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
-                ws_bytes(nblocks + 1, sizeof(RbmItem)) +
+                2 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
@@ -1111,7 +1118,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   WorkItem *list_w = arena_take<WorkItem>(W2, nblocks + 1);   // warp-tier work items
   int32_t *list_c = arena_take<int32_t>(W2, nblocks + 1);     // CTA-tier blocks
   int32_t *list_wide = arena_take<int32_t>(W2, nblocks + 1);  // blocks flagged for 64-bit sums
-  RbmItem *list_r = arena_take<RbmItem>(W2, nblocks + 1);     // bitmap-rank items
+  RbmItem *list_r = arena_take<RbmItem>(W2, nblocks + 1);     // rank items n <= 2048 (front / back)
+  RbmItem *list_r2 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n > 2048 (front / back)
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1252,7 +1260,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, list_r, counts + 10, rbm, vw64, err);
+                                              list_c, list_r, list_r2, counts + 10, rbm, vw64, err);
     HEC_LAUNCH_CHECK();
   }
 
@@ -1291,10 +1299,18 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   A.nlist = counts + 11;
   HEC_TRY(launch_rows(ctx, A, false));
   if (rbm) {
-    A.ritems = list_r;
-    A.nlist = counts + 12;
     A.ticket = counts + 13;
-    HEC_TRY(launch_rbm(ctx, A));
+    A.rcap = nblocks + 1;
+    // hash-rank size classes, then the bitmap-rank items above kHrMax2 entries
+    const struct { RbmItem *items; unsigned *n; int dir; } cls[4] = {
+        {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}, {list_r2, counts + 16, -1}};
+    for (int c = 0; c < 4; ++c) {
+      A.ritems = cls[c].items;
+      A.nlist = cls[c].n;
+      A.rdir = cls[c].dir;
+      if (c < 3) HEC_TRY(launch_hrank(ctx, A, c));
+      else HEC_TRY(launch_rbm(ctx, A));
+    }
     A.ticket = counts + 1;
   }
   phase_end(ctx, ph_rows);

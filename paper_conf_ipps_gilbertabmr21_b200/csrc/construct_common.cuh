@@ -231,6 +231,10 @@ struct WorkItem {
   int32_t R;
 };
 
+// Size classes of the rank items (k_tiers): n <= 1024, <= 2048, <= 4096 go to
+// k_hrank<128/256/512> (construct_hrank.cu), larger ones to k_rbm.
+constexpr int kHrMax0 = 1024, kHrMax1 = 2048, kHrMax2 = 4096;
+
 // A bitmap-rank item (construct_rbm.cu), self-contained so a CTA prefetches it:
 // entries [src, src + n) of sc_col/sc_wgt (B_RBM whole row) or pb_g/pw_g (bin),
 // keys in [lo, hi); row = the coarse row (its self entries are dropped).
@@ -254,6 +258,10 @@ __device__ __forceinline__ int64_t bin_lower(int64_t k, int64_t nb, int64_t n_c)
     else lo = mid + 1;
   }
   return lo;
+}
+
+__device__ __forceinline__ RbmItem rbm_at(const RbmItem *items, int dir, int64_t cap, int64_t i) {
+  return items[dir > 0 ? i : cap - 1 - i];
 }
 
 struct BlockDesc {
@@ -306,7 +314,9 @@ struct RowsArgs {
   unsigned long long *pstats;  // debug (HEC_PIECE_STATS): warp items / entries per kind x size class; nullable
   const int32_t *list;    // blocks of this launch (a tier list)
   const WorkItem *items;  // warp tier: the same, as work items
-  const RbmItem *ritems;  // bitmap-rank tier
+  const RbmItem *ritems;  // bitmap-rank / hash-rank tier (one size class per launch)
+  int32_t rdir;           // +1: items ritems[0 .. n); -1: ritems[rcap - 1], ritems[rcap - 2], ...
+  int64_t rcap;
   const unsigned *nlist;  // device count of `list` / `items`
 };
 
@@ -316,5 +326,6 @@ int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide);
 int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket);  // construct_pieces.cu
 int launch_place(hec_ctx *ctx, const RowsArgs &A);
 int launch_rbm(hec_ctx *ctx, const RowsArgs &A);  // construct_rbm.cu
+int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls);  // construct_hrank.cu (cls 0..2: n <= 1024/2048/4096)
 
 }  // namespace hec

@@ -1,0 +1,200 @@
+// construct_hrank.cu — ordered duplicate merge by shared-memory hash + key-range
+// bucket rank, several CTAs per SM (PAPER.md:L319-324
+// DEDUPWITHWTS: "deduplicate ... and sum the weights", L280: self loops omitted).
+//
+// Consumes the same items as k_rbm (construct_rbm.cu): one coarse row with
+// kPieceMax < U <= kRbmRow read from the expansion staging, or one key-range
+// bin of a partitioned row; keys lie in [lo, hi).  For an item of n <= NT*8
+// entries (all held in registers) the CTA
+//   1. merges duplicates in a shared-memory hash table (CAS on the key, add on
+//      the weight; the inserting entry "owns" the distinct key) -- the hash
+//      half of the paper's hash-vs-sort dedup, on B200's fast smem atomics;
+//   2. counts the distinct keys per order-preserving key-range bucket
+//      (bucket = floor((b - lo) * NB / (hi - lo)), NB >= n buckets, so a bucket
+//      holds ~1 key), scans the counts, and ranks each key inside its bucket by
+//      comparison -- the rank is the key's position in the sorted row, so no
+//      sorting pass runs;
+//   3. writes (b, sum) at its rank, in place over the item's own input range.
+// Work is O(n) per item with six CTA barriers; several CTAs per SM overlap
+// them.  Items with n > NT*8 entries are left to k_rbm.
+#include "construct_common.cuh"
+
+namespace hec {
+
+template <int NT>
+struct HrSmem {
+  static constexpr int kCapE = NT * 8;       // entries per item
+  static constexpr int kSlots = 2 * kCapE;   // hash slots (load <= 1/2)
+  int32_t key[kSlots];
+  uint32_t val[kSlots];
+  int32_t cnt[kCapE + 1];                    // bucket counts -> offsets
+  int32_t scr[kCapE];                        // distinct keys in bucket order
+  int32_t wsum[NT / 32 + 1];
+  int32_t nd;                                // distinct keys of the item
+};
+
+__device__ __forceinline__ uint32_t hr_hash(int32_t b) { return (uint32_t)b * 0x9E3779B1u; }
+
+// Block exclusive scan of c[0..nb) in place (nb <= NT * 8); returns the total.
+template <int NT>
+__device__ __forceinline__ int hr_scan(int32_t *c, int nb, int32_t *wsum) {
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  const int per = (nb + NT - 1) / NT;
+  const int beg = t * per;
+  int v[8];
+  int local = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    v[i] = (i < per && beg + i < nb) ? c[beg + i] : 0;
+    local += v[i];
+  }
+  int x = local;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[wid] = x;
+  __syncthreads();
+  int before = 0, total = 0;
+#pragma unroll
+  for (int w = 0; w < NT / 32; ++w) {
+    const int s = wsum[w];
+    before += w < wid ? s : 0;
+    total += s;
+  }
+  int run = before + x - local;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    if (i < per && beg + i < nb) c[beg + i] = run;
+    run += v[i];
+  }
+  return total;
+}
+
+template <int NT>
+__global__ void __launch_bounds__(NT, 1024 / NT) k_hrank(RowsArgs A) {
+  constexpr int kCapE = HrSmem<NT>::kCapE;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  HrSmem<NT> &S = *reinterpret_cast<HrSmem<NT> *>(smem_raw);
+  const int t = threadIdx.x;
+  const int64_t nitems = *A.nlist;
+  for (int i = t; i < HrSmem<NT>::kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
+  for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
+  if (t == 0) S.nd = 0;
+  __syncthreads();
+  for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
+    const RbmItem it = rbm_at(A.ritems, A.rdir, A.rcap, ii);
+    const int n = it.n;
+    const int32_t a = it.row, lo = it.lo;
+    int32_t *src_b = (it.bk < 0 ? A.sc_col : A.pb_g) + it.src;
+    int32_t *src_w = (it.bk < 0 ? A.sc_wgt : A.pw_g) + it.src;
+    // table geometry: NB buckets (power of two >= n), 2 NB hash slots
+    int lg = 0;
+    while ((1 << lg) < n) ++lg;
+    const int NB = 1 << lg;
+    const uint32_t hmask = 2u * NB - 1u;
+    const int hshift = 31 - lg;  // top lg + 1 bits of the hash
+    const float scale = (float)NB / (float)(it.hi - lo);
+    int32_t kb[8], kw[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int i = t + NT * k;
+      kb[k] = -1;
+      kw[k] = 0;
+      if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+    }
+    // ---- 1. hash merge; owners count their bucket
+    bool bad = false, wrap = false;
+    int slot[8], bpos[8];
+    unsigned own = 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (kb[k] == a) kb[k] = -1;  // self entry (L280)
+      if (kb[k] < 0) continue;
+      if (kb[k] < lo || kb[k] >= it.hi) { bad = true; kb[k] = -1; continue; }
+      uint32_t h = (hr_hash(kb[k]) >> hshift) & hmask;
+      while (true) {
+        const int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
+        if (old == kEmpty) { own |= 1u << k; break; }
+        if (old == kb[k]) break;
+        h = (h + 1) & hmask;
+      }
+      slot[k] = (int)h;
+      const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
+      wrap |= o + (uint32_t)kw[k] < o;
+      if (own & (1u << k)) {
+        int bk = (int)__fmul_rz((float)(kb[k] - lo), scale);
+        bk = bk < NB - 1 ? bk : NB - 1;
+        bpos[k] = atomicAdd(&S.cnt[bk], 1);
+        slot[k] |= bk << 16;  // slot < 2^14, bucket < 2^13
+      }
+    }
+    if (bad) atomicOr(A.err, ERR_INTERNAL);
+    if (wrap) atomicOr(A.err, ERR_OVERFLOW);
+    __syncthreads();
+    // ---- 2. bucket offsets; owners place their key in bucket order
+    const int D = hr_scan<NT>(S.cnt, NB, S.wsum);
+    if (D > kCapE) atomicOr(A.err, ERR_INTERNAL);
+    __syncthreads();
+    int boff[8], bend[8];
+    uint32_t sum[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (!(own & (1u << k))) continue;
+      const int bk = slot[k] >> 16;
+      boff[k] = S.cnt[bk];
+      bend[k] = bk + 1 < NB ? S.cnt[bk + 1] : D;
+      S.scr[boff[k] + bpos[k]] = kb[k];
+      sum[k] = S.val[slot[k] & 0xffff];
+    }
+    __syncthreads();
+    // ---- 3. rank inside the bucket, write at the rank, clean the owned slot
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (!(own & (1u << k))) continue;
+      int r = boff[k];
+      for (int j = boff[k]; j < bend[k]; ++j) r += S.scr[j] < kb[k];
+      if (sum[k] > 0x7fffffffu) atomicOr(A.err, ERR_OVERFLOW);
+      src_b[r] = kb[k];
+      src_w[r] = (int32_t)sum[k];
+      const int h = slot[k] & 0xffff;
+      S.key[h] = kEmpty;
+      S.val[h] = 0u;
+    }
+    for (int i = t; i < NB; i += NT) S.cnt[i] = 0;
+    if (t == 0) A.blk_cnt[it.bi] = D;
+    __syncthreads();
+  }
+}
+
+template <int NT>
+static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
+  static bool attr = false;
+  static int occ = 1;
+  const size_t smem = sizeof(HrSmem<NT>);
+  if (!attr) {
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_hrank<NT>, NT, smem));
+    if (occ < 1) occ = 1;
+    attr = true;
+  }
+  int64_t grid = (int64_t)ctx->num_sms * occ;
+  if (A.nblocks < grid) grid = A.nblocks;
+  if (grid < 1) return HEC_OK;
+  k_hrank<NT><<<(unsigned)grid, NT, smem, ctx->stream>>>(A);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
+// One size class of items (the list in A.ritems / A.nlist): cls 0, 1, 2 =
+// n <= 1024, 2048, 4096 on 128-, 256-, 512-thread CTAs.
+int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls) {
+  static_assert(HrSmem<128>::kCapE == kHrMax0 && HrSmem<256>::kCapE == kHrMax1 && HrSmem<512>::kCapE == kHrMax2,
+                "size classes");
+  if (cls == 0) return launch_hrank_t<128>(ctx, A);
+  if (cls == 1) return launch_hrank_t<256>(ctx, A);
+  return launch_hrank_t<512>(ctx, A);
+}
+
+}  // namespace hec

@@ -46,7 +46,7 @@ __device__ __forceinline__ int rbm_rank(const RbmSmem &S, int o) {
 __device__ __forceinline__ RbmItem rbm_item(const RowsArgs &A, int64_t i, int64_t nitems) {
   RbmItem it{};
   it.n = -1;
-  if (i < nitems) it = A.ritems[i];
+  if (i < nitems) it = rbm_at(A.ritems, A.rdir, A.rcap, i);
   return it;
 }
 

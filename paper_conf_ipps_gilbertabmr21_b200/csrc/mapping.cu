@@ -243,9 +243,184 @@ __global__ void k_fill_identity(int64_t n, int64_t vbase, int32_t *__restrict__ 
 
 static inline unsigned nblk(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
 
+// ------------------------------------------------- a1 heavy, segmented streaming
+// Entries are streamed in warp spans of kSpan = 512 (16-byte vector loads of col
+// and wgt, all issued up front).  Each warp marks the row starts / row ends that
+// fall in its span in warp-private shared bitmaps, then runs a segmented max of
+// the packed key (w << 32 | ~v) over the span.
+// A row ending in the span is final there if it also starts in the span;
+// otherwise the span's "head" value is combined by k_heavy_seg_fixup with the
+// "mid" values of the spans the row covers.  No CTA barriers: warps are
+// independent, so the stream never waits on a barrier.
+constexpr int kSpan = 512;
+constexpr int kSegWarps = 8;
+struct SegWarpSmem {
+  uint32_t head[kSpan / 32];
+  uint32_t end[kSpan / 32];
+  int32_t endrow[kSpan];
+};
+
+// x0: aligned index of span 0 (aligned index = entry + off; col/wgt - off are
+// 16-byte aligned); entries [ebase, ebase + nnz) belong to rows [0, n) of rp.
+__global__ void k_span_coords(int64_t n, int64_t nnz, const int64_t *__restrict__ rp, int64_t ebase,
+                              int64_t x0, int64_t off, int64_t nspans, int32_t *__restrict__ cx) {
+  const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (k > nspans) return;
+  if (k == nspans) { cx[k] = (int32_t)(n - 1); return; }
+  if (k == 0) { cx[k] = 0; return; }  // leading empty rows belong to span 0
+  int64_t e = x0 + k * kSpan - off;
+  if (e < ebase) e = ebase;
+  if (e > ebase + nnz - 1) e = ebase + nnz - 1;
+  int64_t lo = 0, hi = n - 1;  // largest r with rp[r] <= e
+  while (lo < hi) {
+    const int64_t mid = (lo + hi + 1) >> 1;
+    if (__ldg(rp + mid) <= e) lo = mid;
+    else hi = mid - 1;
+  }
+  cx[k] = (int32_t)lo;
+}
+
+// Lane l of the warp owns the 16 consecutive entries [16 l, 16 l + 16) of the
+// span: a sequential segmented max over them (resets at row starts, final H for
+// rows that start and end inside the lane), ONE warp scan of the lane
+// aggregates per span, then the lane's first row end (which may continue a row
+// from earlier lanes or spans) is resolved with the scanned prefix.
+// kVec: col/wgt share a 16-byte phase (int4 loads); else scalar loads.
+template <bool kVec>
+__global__ void __launch_bounds__(32 * kSegWarps, 3) k_heavy_seg(
+    int64_t n, int64_t nnz, const int64_t *__restrict__ rp, int64_t ebase, int64_t vbase, int64_t x0, int64_t off,
+    int64_t nspans, const int32_t *__restrict__ colA, const int32_t *__restrict__ wgtA,
+    const int32_t *__restrict__ cx, int32_t *__restrict__ H, uint64_t *__restrict__ head_key,
+    uint64_t *__restrict__ mid_key) {
+  __shared__ SegWarpSmem smem[kSegWarps];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t k = blockIdx.x * (int64_t)kSegWarps + wid;
+  if (k >= nspans) return;
+  SegWarpSmem &W = smem[wid];
+  const int64_t xs = x0 + k * kSpan;          // aligned index of the span start
+  const int64_t es = xs - off;                // entry index of the span start
+  const int64_t elo = ebase, ehi = ebase + nnz;
+  const bool interior = es >= elo && es + kSpan <= ehi;
+  // ---- loads first (lane: 16 consecutive entries = 4 x 16 B of col and of wgt)
+  int cc[16], ww[16];
+  if (kVec) {
+    const int4 *c4 = reinterpret_cast<const int4 *>(colA + xs) + 4 * lane;
+    const int4 *w4 = reinterpret_cast<const int4 *>(wgtA + xs) + 4 * lane;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int64_t e0 = es + 16 * lane + 4 * j;
+      int4 c = make_int4(0, 0, 0, 0), w = make_int4(0, 0, 0, 0);
+      if (interior || (e0 + 3 >= elo && e0 < ehi)) { c = __ldcs(c4 + j); w = __ldcs(w4 + j); }
+      cc[4 * j] = c.x; cc[4 * j + 1] = c.y; cc[4 * j + 2] = c.z; cc[4 * j + 3] = c.w;
+      ww[4 * j] = w.x; ww[4 * j + 1] = w.y; ww[4 * j + 2] = w.z; ww[4 * j + 3] = w.w;
+    }
+  } else {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const int64_t e = es + 16 * lane + q;
+      cc[q] = 0;
+      ww[q] = 0;
+      if (interior || (e >= elo && e < ehi)) { cc[q] = __ldcs(colA + e); ww[q] = __ldcs(wgtA + e); }
+    }
+  }
+  // ---- row starts / ends inside the span
+  if (lane < kSpan / 32) { W.head[lane] = 0u; W.end[lane] = 0u; }
+  __syncwarp();
+  const int64_t r0 = cx[k], r1 = cx[k + 1];
+  for (int64_t r = r0 + lane; r <= r1; r += 32) {
+    const int64_t s = __ldg(rp + r), e = __ldg(rp + r + 1);
+    if (s == e) {
+      H[vbase + r] = (int32_t)(vbase + r);  // isolated (idempotent)
+      continue;
+    }
+    const int64_t ps = s - es, pe = e - 1 - es;
+    if (ps >= 0 && ps < kSpan) atomicOr(&W.head[ps >> 5], 1u << (ps & 31));
+    if (pe >= 0 && pe < kSpan) {
+      atomicOr(&W.end[pe >> 5], 1u << (pe & 31));
+      W.endrow[pe] = (int32_t)r;
+    }
+  }
+  __syncwarp();
+  // ---- lane-sequential segmented max
+  const unsigned hb = (W.head[lane >> 1] >> (16 * (lane & 1))) & 0xffffu;
+  const unsigned eb = (W.end[lane >> 1] >> (16 * (lane & 1))) & 0xffffu;
+  if (!interior) {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const int64_t e = es + 16 * lane + q;
+      if (e < elo || e >= ehi) ww[q] = 0;  // key 0: never a maximum
+    }
+  }
+  uint64_t run = 0, pend = 0;
+  int pend_q = -1;  // the lane's first row end before any row start in the lane
+#pragma unroll
+  for (int q = 0; q < 16; ++q) {
+    const uint64_t key = ww[q] ? pack_key(ww[q], cc[q]) : 0ull;
+    if ((hb >> q) & 1u) run = key;
+    else run = key > run ? key : run;
+    if ((eb >> q) & 1u) {
+      if (hb & ((2u << q) - 1u)) H[vbase + W.endrow[16 * lane + q]] = key_vertex(run);
+      else if (pend_q < 0) { pend = run; pend_q = q; }
+    }
+  }
+  // ---- warp scan of the lane aggregates (segmented by "lane has a row start")
+  bool stop = hb != 0u || lane == 0;
+  uint64_t incl = run;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xffffffffu, incl, o);
+    const bool ys = __shfl_up_sync(0xffffffffu, stop, o);
+    if (lane >= o && !stop) {
+      incl = y > incl ? y : incl;
+      stop = ys;
+    }
+  }
+  uint64_t pre = __shfl_up_sync(0xffffffffu, incl, 1);  // running value before the lane
+  if (lane == 0) pre = 0;
+  const unsigned hm = __ballot_sync(0xffffffffu, hb != 0u);
+  if (pend_q >= 0) {
+    const uint64_t v = pre > pend ? pre : pend;
+    if (hm & ((1u << lane) - 1u)) H[vbase + W.endrow[16 * lane + pend_q]] = key_vertex(v);
+    else head_key[k] = v;  // the row began in an earlier span
+  }
+  if (lane == 31) {
+    const uint64_t last = hb ? run : (pre > run ? pre : run);
+    mid_key[k] = (eb >> 15) & 1u ? 0ull : last;
+  }
+}
+
+// Rows that end in span k but began in an earlier span s0: max of span k's head
+// value and the mid values of spans s0 .. k-1.  One warp per span.
+__global__ void k_heavy_seg_fixup(const int64_t *__restrict__ rp, int64_t vbase, int64_t x0, int64_t off,
+                                  int64_t nspans, const int32_t *__restrict__ cx,
+                                  const uint64_t *__restrict__ head_key, const uint64_t *__restrict__ mid_key,
+                                  int32_t *__restrict__ H) {
+  const int lane = threadIdx.x & 31;
+  const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (k >= nspans) return;
+  uint64_t key = head_key[k];
+  if (key == 0ull) return;
+  const int32_t x = cx[k];
+  const int64_t s0 = (__ldg(rp + x) + off - x0) / kSpan;
+  uint64_t m = lane == 0 ? key : 0ull;
+  for (int64_t s = s0 + lane; s < k; s += 32) {
+    const uint64_t y = mid_key[s];
+    m = y > m ? y : m;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const uint64_t y = __shfl_xor_sync(0xffffffffu, m, o);
+    m = y > m ? y : m;
+  }
+  if (lane == 0) H[vbase + x] = key_vertex(m);
+}
+
 static size_t heavy_ws(int64_t n, int64_t nnz) {
   int64_t ntiles = (n + nnz + kHvTile - 1) / kHvTile;
-  return ws_bytes(ntiles + 1, 8) + 2 * ws_bytes(ntiles + 1, 8);
+  int64_t nspans = nnz / kSpan + 2;
+  size_t a = ws_bytes(ntiles + 1, 8) + 2 * ws_bytes(ntiles + 1, 8);
+  size_t b = ws_bytes(nspans + 1, 4) + 2 * ws_bytes(nspans + 1, 8);
+  return a > b ? a : b;
 }
 
 // Heavy neighbours of rows [u0, u1): ebase = row_ptr[u0] and nnz of the range are
@@ -267,6 +442,33 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
   const int64_t *rp = g->row_ptr + u0;
   if (nnz == 0) {
     k_fill_identity<<<nblk(n, 256), 256, 0, ctx->stream>>>(n, u0, H);
+    HEC_LAUNCH_CHECK();
+    return HEC_OK;
+  }
+  const uintptr_t ca = (uintptr_t)g->col, wa = (uintptr_t)g->wgt;
+  const bool aligned16 = (ca & 15) == 0 && (wa & 15) == 0;
+  if (n < INT32_MAX && !(aligned16 && getenv("HEC_HEAVY_TILES") != nullptr)) {
+    // segmented streaming path; int4 loads when col/wgt share their 16-byte phase
+    const bool vec = (ca & 3) == 0 && (ca & 15) == (wa & 15);
+    const int64_t off = vec ? (int64_t)((ca & 15) >> 2) : 0;
+    const int64_t x0 = (ebase + off) & ~(int64_t)3;
+    const int64_t nspans = (ebase + off + nnz - x0 + kSpan - 1) / kSpan;
+    int32_t *cx = ws_take<int32_t>(ctx, nspans + 1);
+    uint64_t *head = ws_take<uint64_t>(ctx, nspans + 1);
+    uint64_t *mid = ws_take<uint64_t>(ctx, nspans + 1);
+    if (!cx || !head || !mid) { set_error("workspace under-reserved (heavy)"); return HEC_EINVAL; }
+    HEC_CUDA_TRY(cudaMemsetAsync(head, 0, sizeof(uint64_t) * nspans, ctx->stream));
+    k_span_coords<<<nblk(nspans + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, x0, off, nspans, cx);
+    HEC_LAUNCH_CHECK();
+    const int32_t *colA = g->col - off, *wgtA = g->wgt - off;
+    if (vec)
+      k_heavy_seg<true><<<nblk(nspans, kSegWarps), 32 * kSegWarps, 0, ctx->stream>>>(
+          n, nnz, rp, ebase, u0, x0, off, nspans, colA, wgtA, cx, H, head, mid);
+    else
+      k_heavy_seg<false><<<nblk(nspans, kSegWarps), 32 * kSegWarps, 0, ctx->stream>>>(
+          n, nnz, rp, ebase, u0, x0, off, nspans, colA, wgtA, cx, H, head, mid);
+    HEC_LAUNCH_CHECK();
+    k_heavy_seg_fixup<<<nblk(nspans * 32, 256), 256, 0, ctx->stream>>>(rp, u0, x0, off, nspans, cx, head, mid, H);
     HEC_LAUNCH_CHECK();
     return HEC_OK;
   }

@@ -98,6 +98,47 @@ def test_heavy_hub_rows_span_tiles(P, ctx):
     assert np.array_equal(H, o.heavy(g))
 
 
+def scattered_isolated_graph(n, rng, deg=6, iso_frac=0.1):
+    """Random graph whose isolated (empty) rows sit at the start, in the middle
+    and at the end of the vertex range, next to rows far longer than a span."""
+    iso = set(rng.choice(n, max(1, int(iso_frac * n)), replace=False).tolist()) | {0, 1, n // 2, n - 1}
+    live = np.array(sorted(set(range(n)) - iso))
+    edges = {}
+    for _ in range(deg * n // 2):
+        u, v = rng.choice(live, 2)
+        if u != v:
+            edges[(min(u, v), max(u, v))] = int(rng.integers(1, 6))
+    hub = int(live[len(live) // 3])
+    for v in live[::2]:
+        if v != hub:
+            edges[(min(hub, v), max(hub, v))] = int(rng.integers(1, 6))
+    return gg.from_edges(n, [(u, v, w) for (u, v), w in edges.items()])
+
+
+@pytest.mark.parametrize("path", ["spans", "tiles"])
+@pytest.mark.parametrize("phase", [0, 1, 2, 3, "mixed"])
+def test_heavy_isolated_and_unaligned(P, ctx, path, phase, monkeypatch):
+    """a1 with empty rows anywhere and col/wgt views that start 0-3 int32 past a
+    16-byte boundary (same phase: segmented span kernel; different phases: the
+    tile kernel).  path=tiles forces the merge-path tile kernel (test hook)."""
+    if path == "tiles":
+        monkeypatch.setenv("HEC_HEAVY_TILES", "1")
+    rng = np.random.default_rng(31 if phase == "mixed" else 31 + phase)
+    for n in (6, 700, 20000):
+        g = scattered_isolated_graph(n, rng)
+        pc, pw = (1, 3) if phase == "mixed" else (phase, phase)
+        cbuf = torch.zeros(g.nnz + 8, dtype=torch.int32, device="cuda")
+        wbuf = torch.zeros(g.nnz + 8, dtype=torch.int32, device="cuda")
+        col = cbuf[pc:pc + g.nnz]
+        wgt = wbuf[pw:pw + g.nnz]
+        col.copy_(torch.from_numpy(g.col))
+        wgt.copy_(torch.from_numpy(g.wgt))
+        dg = P.DeviceGraph(torch.from_numpy(g.row_ptr).cuda(), col, wgt, None)
+        H = P.hec_debug_heavy(ctx, dg).cpu().numpy()
+        assert np.array_equal(H, o.heavy(g))
+
+
+
 # ------------------------------------------------------------------ a3
 def test_roots_and_rounds_c1(P, ctx, golden_dir):
     ka = json.load(open(os.path.join(golden_dir, "survey_known_answers.json")))["C1"]
