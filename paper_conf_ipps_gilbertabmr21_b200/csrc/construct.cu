@@ -388,6 +388,109 @@ __global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restr
   }
 }
 
+// Expansion v2: a warp walks the members of its 4096-position chunk 32 at a
+// time (one coalesced load of their metadata per window).  Members with more
+// than kXBig positions in the chunk are streamed one by one by the whole warp;
+// the others are packed: a warp scan of their lengths gives every position of
+// the window a (member, offset) by a 5-step shuffle search, so short rows fill
+// all 32 lanes.  Four positions per lane are in flight per step (col, wgt,
+// then the M gathers).  No shared memory, no CTA barriers.
+constexpr int kXBig = 64;
+
+__device__ __forceinline__ void x2_copy4(const Layout &L, int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
+                                         const int64_t (&e)[4], const int64_t (&p)[4], unsigned ok) {
+  int32_t b[4], w[4];
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+    if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+    if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+    if (ok & (1u << u)) { __stcs(Sb + p[u], b[u]); __stcs(Sw + p[u], w[u]); }
+}
+
+__global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
+                                               int32_t *__restrict__ Sb, int32_t *__restrict__ Sw) {
+  const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
+  const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * kXT + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * kXT) >> 5;
+  for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
+    const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
+    int64_t i = warp_find_member(L, m_lo, m_hi, P);
+    while (true) {
+      const int64_t j = i + lane;
+      int64_t mp0 = P_hi, mp1 = P_hi, rs = 0;
+      if (j < m_hi) { mp0 = L.mpre[j]; mp1 = L.mpre[j + 1]; rs = mstart[j]; }
+      const int64_t ps = mp0 > P ? mp0 : P;
+      const int64_t pe = mp1 < Pend ? mp1 : Pend;
+      const int d = pe > ps ? (int)(pe - ps) : 0;
+      rs += ps - mp0;  // source entry of position ps
+      const int64_t pr = ps - P_lo;  // staging index of position ps
+      const bool big = d > kXBig;
+      // ---- packed short members
+      const int ds = big ? 0 : d;
+      int incl = ds;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += y;
+      }
+      const int excl = incl - ds;
+      const int T = __shfl_sync(0xffffffffu, incl, 31);
+      for (int base = 0; base < T; base += 128) {
+        int64_t e[4], p[4];
+        unsigned ok = 0;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int t = base + lane + 32 * u;
+          int lo = 0;  // largest lane with excl <= t
+#pragma unroll
+          for (int st = 16; st > 0; st >>= 1) {
+            const int c = lo + st;
+            const int v = __shfl_sync(0xffffffffu, excl, c & 31);
+            if (c < 32 && v <= t) lo = c;
+          }
+          const int64_t ors = __shfl_sync(0xffffffffu, rs, lo);
+          const int64_t opr = __shfl_sync(0xffffffffu, pr, lo);
+          const int oex = __shfl_sync(0xffffffffu, excl, lo);
+          e[u] = ors + (t - oex);
+          p[u] = opr + (t - oex);
+          if (t < T) ok |= 1u << u;
+        }
+        x2_copy4(L, Sb, Sw, e, p, ok);
+      }
+      // ---- long members, one at a time
+      unsigned bm = __ballot_sync(0xffffffffu, big);
+      while (bm) {
+        const int src = __ffs(bm) - 1;
+        bm &= bm - 1;
+        const int bd = __shfl_sync(0xffffffffu, d, src);
+        const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
+        const int64_t bpr = __shfl_sync(0xffffffffu, pr, src);
+        for (int base = 0; base < bd; base += 128) {
+          int64_t e[4], p[4];
+          unsigned ok = 0;
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int t = base + lane + 32 * u;
+            e[u] = brs + t;
+            p[u] = bpr + t;
+            if (t < bd) ok |= 1u << u;
+          }
+          x2_copy4(L, Sb, Sw, e, p, ok);
+        }
+      }
+      // the window reaches the chunk end (or the last member): done
+      if (__any_sync(0xffffffffu, mp1 >= Pend)) break;
+      i += 32;
+    }
+  }
+}
+
 // ------------------------------------------------------- a9 BUCKET partition
 // One CTA per unit (<= kUnit positions of one skewed row): a shared-memory
 // histogram over the row's key-range buckets (bucket = floor(b * nb / n_c)),
@@ -1135,7 +1238,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     const int64_t cap = (int64_t)ctx->num_sms * 8;
     if (grid > cap) grid = cap;
     if (grid > 0) {
-      k_expand<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
+      if (getenv("HEC_EXPAND_V1")) k_expand<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
+      else k_expand2<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
       HEC_LAUNCH_CHECK();
     }
     phase_end(ctx, phx);

@@ -27,7 +27,8 @@ struct HrSmem {
   static constexpr int kSlots = 2 * kCapE;   // hash slots (load <= 1/2)
   int32_t key[kSlots];
   uint32_t val[kSlots];
-  int32_t cnt[kCapE + 1];                    // bucket counts -> offsets
+  int32_t cnt[kCapE + 1];                    // bucket counts (zeroed by the scan)
+  int32_t offs[kCapE + 1];                   // bucket offsets
   int32_t scr[kCapE];                        // distinct keys in bucket order
   int32_t wsum[NT / 32 + 1];
   int32_t nd;                                // distinct keys of the item
@@ -35,9 +36,10 @@ struct HrSmem {
 
 __device__ __forceinline__ uint32_t hr_hash(int32_t b) { return (uint32_t)b * 0x9E3779B1u; }
 
-// Block exclusive scan of c[0..nb) in place (nb <= NT * 8); returns the total.
+// Block exclusive scan of c[0..nb) into o[0..nb] (nb <= NT * 8), zeroing c;
+// returns the total.
 template <int NT>
-__device__ __forceinline__ int hr_scan(int32_t *c, int nb, int32_t *wsum) {
+__device__ __forceinline__ int hr_scan(int32_t *c, int32_t *o, int nb, int32_t *wsum) {
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int per = (nb + NT - 1) / NT;
   const int beg = t * per;
@@ -45,7 +47,8 @@ __device__ __forceinline__ int hr_scan(int32_t *c, int nb, int32_t *wsum) {
   int local = 0;
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
-    v[i] = (i < per && beg + i < nb) ? c[beg + i] : 0;
+    v[i] = 0;
+    if (i < per && beg + i < nb) { v[i] = c[beg + i]; c[beg + i] = 0; }
     local += v[i];
   }
   int x = local;
@@ -66,14 +69,15 @@ __device__ __forceinline__ int hr_scan(int32_t *c, int nb, int32_t *wsum) {
   int run = before + x - local;
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
-    if (i < per && beg + i < nb) c[beg + i] = run;
+    if (i < per && beg + i < nb) o[beg + i] = run;
     run += v[i];
   }
+  if (t == NT - 1) o[nb] = total;
   return total;
 }
 
 template <int NT>
-__global__ void __launch_bounds__(NT, 1024 / NT) k_hrank(RowsArgs A) {
+__global__ void __launch_bounds__(NT, NT == 128 ? 9 : 1024 / NT) k_hrank(RowsArgs A) {
   constexpr int kCapE = HrSmem<NT>::kCapE;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   HrSmem<NT> &S = *reinterpret_cast<HrSmem<NT> *>(smem_raw);
@@ -83,15 +87,17 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank(RowsArgs A) {
   for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
   __syncthreads();
+  RbmItem nx{};
+  if (blockIdx.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, blockIdx.x);
   for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
-    const RbmItem it = rbm_at(A.ritems, A.rdir, A.rcap, ii);
+    const RbmItem it = nx;  // descriptor prefetched one item ahead
+    if (ii + gridDim.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, ii + gridDim.x);
     const int n = it.n;
     const int32_t a = it.row, lo = it.lo;
     int32_t *src_b = (it.bk < 0 ? A.sc_col : A.pb_g) + it.src;
     int32_t *src_w = (it.bk < 0 ? A.sc_wgt : A.pw_g) + it.src;
     // table geometry: NB buckets (power of two >= n), 2 NB hash slots
-    int lg = 0;
-    while ((1 << lg) < n) ++lg;
+    const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
     const int NB = 1 << lg;
     const uint32_t hmask = 2u * NB - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
@@ -134,35 +140,34 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank(RowsArgs A) {
     if (wrap) atomicOr(A.err, ERR_OVERFLOW);
     __syncthreads();
     // ---- 2. bucket offsets; owners place their key in bucket order
-    const int D = hr_scan<NT>(S.cnt, NB, S.wsum);
+    const int D = hr_scan<NT>(S.cnt, S.offs, NB, S.wsum);
     if (D > kCapE) atomicOr(A.err, ERR_INTERNAL);
     __syncthreads();
-    int boff[8], bend[8];
-    uint32_t sum[8];
+    int boff[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (!(own & (1u << k))) continue;
+      boff[k] = S.offs[slot[k] >> 16];
+      S.scr[boff[k] + bpos[k]] = kb[k];
+    }
+    __syncthreads();
+    // ---- 3. rank inside the bucket (its keys follow boff until the bucket
+    // changes), write at the rank, clean the owned slot
 #pragma unroll
     for (int k = 0; k < 8; ++k) {
       if (!(own & (1u << k))) continue;
       const int bk = slot[k] >> 16;
-      boff[k] = S.cnt[bk];
-      bend[k] = bk + 1 < NB ? S.cnt[bk + 1] : D;
-      S.scr[boff[k] + bpos[k]] = kb[k];
-      sum[k] = S.val[slot[k] & 0xffff];
-    }
-    __syncthreads();
-    // ---- 3. rank inside the bucket, write at the rank, clean the owned slot
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      if (!(own & (1u << k))) continue;
+      const int bend = S.offs[bk + 1];
       int r = boff[k];
-      for (int j = boff[k]; j < bend[k]; ++j) r += S.scr[j] < kb[k];
-      if (sum[k] > 0x7fffffffu) atomicOr(A.err, ERR_OVERFLOW);
-      src_b[r] = kb[k];
-      src_w[r] = (int32_t)sum[k];
+      for (int j = boff[k]; j < bend; ++j) r += S.scr[j] < kb[k];
       const int h = slot[k] & 0xffff;
+      const uint32_t sum = S.val[h];
+      if (sum > 0x7fffffffu) atomicOr(A.err, ERR_OVERFLOW);
+      src_b[r] = kb[k];
+      src_w[r] = (int32_t)sum;
       S.key[h] = kEmpty;
       S.val[h] = 0u;
     }
-    for (int i = t; i < NB; i += NT) S.cnt[i] = 0;
     if (t == 0) A.blk_cnt[it.bi] = D;
     __syncthreads();
   }
