@@ -1198,7 +1198,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
-                2 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
+                3 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
@@ -1223,6 +1223,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   int32_t *list_wide = arena_take<int32_t>(W2, nblocks + 1);  // blocks flagged for 64-bit sums
   RbmItem *list_r = arena_take<RbmItem>(W2, nblocks + 1);     // rank items n <= 2048 (front / back)
   RbmItem *list_r2 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n > 2048 (front / back)
+  RbmItem *list_redo = arena_take<RbmItem>(W2, nblocks + 1);  // n > 4096 items left to k_rbm
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1413,7 +1414,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
       A.nlist = cls[c].n;
       A.rdir = cls[c].dir;
       if (c < 3) HEC_TRY(launch_hrank(ctx, A, c));
-      else HEC_TRY(launch_rbm(ctx, A));
+      else if (getenv("HEC_NO_HRANK_BIG")) HEC_TRY(launch_rbm(ctx, A));
+      else {
+        // multi-round hash rank; items with too many distinct keys -> k_rbm
+        HEC_TRY(launch_hrank_big(ctx, A, list_redo, counts + 17));
+        A.ritems = list_redo;
+        A.nlist = counts + 17;
+        A.rdir = 1;
+        HEC_TRY(launch_rbm(ctx, A));
+      }
     }
     A.ticket = counts + 1;
   }
@@ -1463,7 +1472,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int ph_place = phase_begin(ctx, "place", 16.0 * (double)nnz_c + 16.0 * dnc);
   HEC_TRY(launch_place(ctx, A));
   phase_end(ctx, ph_place);
-  phase_set_bytes(ctx, ph_rows, 8.0 * (double)small_vol + 12.0 * dnc);
+  // rows phase: staged / partitioned entries read (8 B each; DENSE rows were
+  // accumulated in rows_skew), distinct entries staged (8 B), row_ptr_c + vwgt_c
+  phase_set_bytes(ctx, ph_rows, 8.0 * (double)(small_vol + (dense ? 0 : big_vol)) + 8.0 * (double)nnz_c + 12.0 * dnc);
   if (nblocks == 0) HEC_CUDA_TRY(cudaMemsetAsync(out->row_ptr, 0, sizeof(int64_t) * (n_out + 1), s));
   ctx->stats.nnz_c = out->nnz_c;
   return HEC_OK;

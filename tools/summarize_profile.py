@@ -33,7 +33,8 @@ PHASE = {
     "k_block_desc": "rows", "k_block_ends": "rows", "k_rows": "rows", "BlkCntIn": "rows",
     "k_pieces": "rows", "k_tiers": "rows", "k_wide_list": "rows", "k_expand": "expand",
     "k_bucket_blocks": "rows_skew",
-    "k_place": "place",
+    "k_place": "place", "k_hrank": "rows", "k_rbm": "rows", "k_span_coords": "heavy",
+    "k_row_bins": "rows_skew", "k_part_warp": "rows_skew", "k_seg_fill": "rows_skew", "RowUIn": "rows_skew",
 }
 
 
