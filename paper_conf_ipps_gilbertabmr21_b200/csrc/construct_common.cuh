@@ -327,5 +327,6 @@ int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket);  // constr
 int launch_place(hec_ctx *ctx, const RowsArgs &A);
 int launch_rbm(hec_ctx *ctx, const RowsArgs &A);  // construct_rbm.cu
 int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls);  // construct_hrank.cu (cls 0..2: n <= 1024/2048/4096)
+int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo);  // n > 4096
 
 }  // namespace hec

@@ -173,6 +173,137 @@ __global__ void __launch_bounds__(NT, NT == 128 ? 9 : 1024 / NT) k_hrank(RowsArg
   }
 }
 
+// Items above NT*8 entries (rank class 3): the entries are merged into the hash
+// table round by round (NT*8 per round); the distinct keys are then taken from
+// the table itself (sweep: bucket counts, scan, placement in bucket order,
+// rank).  An item whose distinct keys would push the table past 3/8 load is
+// abandoned (its slots cleared) and appended to the redo list for k_rbm.
+template <int NT>
+__global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem *__restrict__ redo,
+                                                          unsigned *__restrict__ nredo) {
+  constexpr int kCapE = HrSmem<NT>::kCapE;
+  constexpr int kSlots = HrSmem<NT>::kSlots;
+  constexpr int kMaxD = (3 * kSlots) / 8;  // abandon threshold (in-flight inserts stay below kSlots)
+  static_assert(kMaxD + kCapE < kSlots, "probe loops must terminate");
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  HrSmem<NT> &S = *reinterpret_cast<HrSmem<NT> *>(smem_raw);
+  const int t = threadIdx.x;
+  const int64_t nitems = *A.nlist;
+  for (int i = t; i < kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
+  for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
+  if (t == 0) S.nd = 0;
+  __syncthreads();
+  for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
+    const RbmItem it = rbm_at(A.ritems, A.rdir, A.rcap, ii);
+    const int32_t a = it.row, lo = it.lo;
+    int32_t *src_b = (it.bk < 0 ? A.sc_col : A.pb_g) + it.src;
+    int32_t *src_w = (it.bk < 0 ? A.sc_wgt : A.pw_g) + it.src;
+    const uint32_t hmask = kSlots - 1u;
+    constexpr int kLg = 31 - __builtin_ctz(kSlots);  // hash shift: top log2(kSlots) bits
+    bool bad = false, wrap = false, full = false;
+    for (int64_t r0 = 0; r0 < it.n && !full; r0 += kCapE) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int64_t i = r0 + t + NT * k;
+        int32_t b = -1, w = 0;
+        if (i < it.n) { b = __ldcs(src_b + i); w = __ldcs(src_w + i); }
+        if (b == a) b = -1;  // self entry (L280)
+        if (b < 0) continue;
+        if (b < lo || b >= it.hi) { bad = true; continue; }
+        uint32_t h = (hr_hash(b) >> kLg) & hmask;
+        bool placed = true;
+        while (true) {
+          const int32_t old = S.key[h];
+          if (old == b) break;
+          if (old == kEmpty) {
+            if (*(volatile int32_t *)&S.nd >= kMaxD) { placed = false; break; }
+            const int32_t o2 = atomicCAS(&S.key[h], kEmpty, b);
+            if (o2 == kEmpty) { atomicAdd(&S.nd, 1); break; }
+            if (o2 == b) break;
+          }
+          h = (h + 1) & hmask;
+        }
+        if (!placed) continue;
+        const uint32_t o = atomicAdd(&S.val[h], (uint32_t)w);
+        wrap |= o + (uint32_t)w < o;
+      }
+      __syncthreads();
+      full = S.nd >= kMaxD;
+      __syncthreads();
+    }
+    if (bad) atomicOr(A.err, ERR_INTERNAL);
+    if (full) {  // too many distinct keys: clear, hand the item to k_rbm
+      for (int i = t; i < kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
+      if (t == 0) {
+        redo[atomicAdd(nredo, 1u)] = it;
+        S.nd = 0;
+      }
+      __syncthreads();
+      continue;
+    }
+    if (wrap) atomicOr(A.err, ERR_OVERFLOW);
+    // ---- distinct keys from the table: bucket counts
+    const int D = S.nd;
+    int lgb = D <= 1 ? 0 : 32 - __clz(D - 1);
+    const int NB = 1 << lgb;  // <= kCapE
+    const float scale = (float)NB / (float)(it.hi - lo);
+    for (int sl = t; sl < kSlots; sl += NT) {
+      const int32_t b = S.key[sl];
+      if (b == kEmpty) continue;
+      int bk = (int)__fmul_rz((float)(b - lo), scale);
+      bk = bk < NB - 1 ? bk : NB - 1;
+      atomicAdd(&S.cnt[bk], 1);
+    }
+    __syncthreads();
+    hr_scan<NT>(S.cnt, S.offs, NB, S.wsum);  // counts zeroed, offsets in offs
+    __syncthreads();
+    for (int sl = t; sl < kSlots; sl += NT) {  // place keys in bucket order (cnt reused as cursors)
+      const int32_t b = S.key[sl];
+      if (b == kEmpty) continue;
+      int bk = (int)__fmul_rz((float)(b - lo), scale);
+      bk = bk < NB - 1 ? bk : NB - 1;
+      S.scr[S.offs[bk] + atomicAdd(&S.cnt[bk], 1)] = b;
+    }
+    __syncthreads();
+    for (int sl = t; sl < kSlots; sl += NT) {
+      const int32_t b = S.key[sl];
+      if (b == kEmpty) continue;
+      int bk = (int)__fmul_rz((float)(b - lo), scale);
+      bk = bk < NB - 1 ? bk : NB - 1;
+      int r = S.offs[bk];
+      for (int j = S.offs[bk]; j < S.offs[bk + 1]; ++j) r += S.scr[j] < b;
+      const uint32_t sum = S.val[sl];
+      if (sum > 0x7fffffffu) atomicOr(A.err, ERR_OVERFLOW);
+      src_b[r] = b;
+      src_w[r] = (int32_t)sum;
+    }
+    __syncthreads();
+    for (int sl = t; sl < kSlots; sl += NT) { S.key[sl] = kEmpty; S.val[sl] = 0u; }
+    for (int i = t; i < NB; i += NT) S.cnt[i] = 0;
+    if (t == 0) {
+      A.blk_cnt[it.bi] = D;
+      S.nd = 0;
+    }
+    __syncthreads();
+  }
+}
+
+int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo) {
+  constexpr int NT = 512;
+  static bool attr = false;
+  const size_t smem = sizeof(HrSmem<NT>);
+  if (!attr) {
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank_big<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = true;
+  }
+  int64_t grid = (int64_t)ctx->num_sms * 2;
+  if (A.nblocks < grid) grid = A.nblocks;
+  if (grid < 1) return HEC_OK;
+  k_hrank_big<NT><<<(unsigned)grid, NT, smem, ctx->stream>>>(A, redo, nredo);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
 template <int NT>
 static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
   static bool attr = false;
