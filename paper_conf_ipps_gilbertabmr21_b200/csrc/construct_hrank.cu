@@ -28,7 +28,7 @@ struct HrSmem {
   int32_t key[kSlots];
   uint32_t val[kSlots];
   int32_t cnt[kCapE + 1];                    // bucket counts (zeroed by the scan)
-  int32_t offs[kCapE + 1];                   // bucket offsets
+  uint16_t offs[kCapE + 2];                  // bucket offsets (<= kCapE)
   int32_t scr[kCapE];                        // distinct keys in bucket order
   int32_t wsum[NT / 32 + 1];
   int32_t nd;                                // distinct keys of the item
@@ -39,7 +39,7 @@ __device__ __forceinline__ uint32_t hr_hash(int32_t b) { return (uint32_t)b * 0x
 // Block exclusive scan of c[0..nb) into o[0..nb] (nb <= NT * 8), zeroing c;
 // returns the total.
 template <int NT>
-__device__ __forceinline__ int hr_scan(int32_t *c, int32_t *o, int nb, int32_t *wsum) {
+__device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t *wsum) {
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int per = (nb + NT - 1) / NT;
   const int beg = t * per;
@@ -69,10 +69,10 @@ __device__ __forceinline__ int hr_scan(int32_t *c, int32_t *o, int nb, int32_t *
   int run = before + x - local;
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
-    if (i < per && beg + i < nb) o[beg + i] = run;
+    if (i < per && beg + i < nb) o[beg + i] = (uint16_t)run;
     run += v[i];
   }
-  if (t == NT - 1) o[nb] = total;
+  if (t == NT - 1) o[nb] = (uint16_t)total;
   return total;
 }
 

@@ -350,6 +350,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
 constexpr int kPlaceT = 256;
 enum : int { SRC_SC = 0, SRC_PB = 1, SRC_FB = 2, SRC_DENSE = 3 };
 
+constexpr int kPlaceBig = 96;
 __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t b0 = ((int64_t)blockIdx.x * (kPlaceT / 32) + (threadIdx.x >> 5)) * 32;
@@ -379,21 +380,36 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   const int64_t O0 = __shfl_sync(0xffffffffu, Om, 0);
   const int64_t total = __shfl_sync(0xffffffffu, Om + Tm, 31) - O0;
   const int32_t *dn = reinterpret_cast<const int32_t *>(A.dense);
-  for (int64_t j0 = 0; j0 < total; j0 += 128) {
+  // blocks with >= kPlaceBig entries: copied one at a time by the whole warp
+  // (8 entries per lane in flight); the others packed, entry -> block by a
+  // 5-step shuffle search over the lanes' block offsets
+  const bool bigb = Tm >= kPlaceBig;
+  const int64_t Ps = bigb ? 0 : Tm;  // packed sizes
+  int64_t pincl = Ps;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int64_t y = __shfl_up_sync(0xffffffffu, pincl, o);
+    if (lane >= o) pincl += y;
+  }
+  const int64_t pex = pincl - Ps;
+  const int64_t ptot = __shfl_sync(0xffffffffu, pincl, 31);
+  for (int64_t j0 = 0; j0 < ptot; j0 += 128) {
     int32_t c[4], w[4];
+    int64_t dst[4];
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
       const int64_t j = j0 + lane + 32 * t;
-      int k = 0;  // last lane whose block starts at or before j
+      int k = 0;  // last lane whose packed range starts at or before j
 #pragma unroll
       for (int step = 16; step > 0; step >>= 1) {
-        const int64_t Oc = __shfl_sync(0xffffffffu, Om, k + step);
-        if (Oc - O0 <= j) k += step;
+        const int64_t Pc = __shfl_sync(0xffffffffu, pex, k + step);
+        if (Pc <= j) k += step;
       }
       const int sk = __shfl_sync(0xffffffffu, src, k);
       const int64_t sb = __shfl_sync(0xffffffffu, soff, k);
-      const int64_t r = j - (__shfl_sync(0xffffffffu, Om, k) - O0);  // index inside the block
-      if (j < total) {
+      const int64_t r = j - __shfl_sync(0xffffffffu, pex, k);  // index inside the block
+      dst[t] = __shfl_sync(0xffffffffu, Om, k) + r;
+      if (j < ptot) {
         if (sk == SRC_SC) { c[t] = __ldcs(A.sc_col + sb + r); w[t] = __ldcs(A.sc_wgt + sb + r); }
         else if (sk == SRC_PB) { c[t] = __ldcs(A.pb_g + sb + r); w[t] = __ldcs(A.pw_g + sb + r); }
         else if (sk == SRC_FB) { c[t] = __ldcs(A.fb_b + sb + r); w[t] = __ldcs(A.fb_w + sb + r); }
@@ -403,9 +419,37 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
       const int64_t j = j0 + lane + 32 * t;
-      if (j < total) {
-        A.col_c[O0 + j] = c[t];
-        A.wgt_c[O0 + j] = w[t];
+      if (j < ptot) {
+        __stcs(A.col_c + dst[t], c[t]);
+        __stcs(A.wgt_c + dst[t], w[t]);
+      }
+    }
+  }
+  unsigned bmask = __ballot_sync(0xffffffffu, bigb);
+  while (bmask) {
+    const int jl = __ffs(bmask) - 1;
+    bmask &= bmask - 1;
+    const int sk = __shfl_sync(0xffffffffu, src, jl);
+    const int64_t sb = __shfl_sync(0xffffffffu, soff, jl);
+    const int64_t O = __shfl_sync(0xffffffffu, Om, jl);
+    const int T = __shfl_sync(0xffffffffu, Tm, jl);
+    const int32_t *sc, *sw;
+    int stride = 1;
+    if (sk == SRC_SC) { sc = A.sc_col + sb; sw = A.sc_wgt + sb; }
+    else if (sk == SRC_PB) { sc = A.pb_g + sb; sw = A.pw_g + sb; }
+    else if (sk == SRC_FB) { sc = A.fb_b + sb; sw = A.fb_w + sb; }
+    else { sc = dn + sb; sw = dn + sb + 1; stride = 2; }
+    for (int r0 = 0; r0 < T; r0 += 256) {
+      int32_t c[8], w[8];
+#pragma unroll
+      for (int t = 0; t < 8; ++t) {
+        const int r = r0 + lane + 32 * t;
+        if (r < T) { c[t] = __ldcs(sc + (int64_t)stride * r); w[t] = __ldcs(sw + (int64_t)stride * r); }
+      }
+#pragma unroll
+      for (int t = 0; t < 8; ++t) {
+        const int r = r0 + lane + 32 * t;
+        if (r < T) { __stcs(A.col_c + O + r, c[t]); __stcs(A.wgt_c + O + r, w[t]); }
       }
     }
   }
