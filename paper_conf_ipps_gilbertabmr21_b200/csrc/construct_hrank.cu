@@ -83,6 +83,9 @@ __global__ void __launch_bounds__(NT, NT == 128 ? 9 : 1024 / NT) k_hrank(RowsArg
   HrSmem<NT> &S = *reinterpret_cast<HrSmem<NT> *>(smem_raw);
   const int t = threadIdx.x;
   const int64_t nitems = *A.nlist;
+  // kernel-argument pointers held in registers (not re-read per slot)
+  int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
+  int *const err = A.err;
   for (int i = t; i < HrSmem<NT>::kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
   for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
@@ -94,14 +97,15 @@ __global__ void __launch_bounds__(NT, NT == 128 ? 9 : 1024 / NT) k_hrank(RowsArg
     if (ii + gridDim.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, ii + gridDim.x);
     const int n = it.n;
     const int32_t a = it.row, lo = it.lo;
-    int32_t *src_b = (it.bk < 0 ? A.sc_col : A.pb_g) + it.src;
-    int32_t *src_w = (it.bk < 0 ? A.sc_wgt : A.pw_g) + it.src;
+    int32_t *const src_b = (it.bk < 0 ? scb : pbg) + it.src;
+    int32_t *const src_w = (it.bk < 0 ? scw : pwg) + it.src;
     // table geometry: NB buckets (power of two >= n), 2 NB hash slots
     const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
     const int NB = 1 << lg;
     const uint32_t hmask = 2u * NB - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
-    const float scale = (float)NB / (float)(it.hi - lo);
+    // any positive scale keeps the buckets monotone in b (approximate division)
+    const float scale = __fdividef((float)NB, (float)(it.hi - lo));
     int32_t kb[8], kw[8];
 #pragma unroll
     for (int k = 0; k < 8; ++k) {
@@ -110,15 +114,15 @@ __global__ void __launch_bounds__(NT, NT == 128 ? 9 : 1024 / NT) k_hrank(RowsArg
       kw[k] = 0;
       if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
     }
-    // ---- 1. hash merge; owners count their bucket
-    bool bad = false, wrap = false;
+    // ---- 1. hash merge; owners count their bucket (keys lie in [lo, hi) by
+    // construction of the items: whole rows span [0, n_c), bins their range)
+    bool wrap = false;
     int slot[8], bpos[8];
     unsigned own = 0;
 #pragma unroll
     for (int k = 0; k < 8; ++k) {
       if (kb[k] == a) kb[k] = -1;  // self entry (L280)
       if (kb[k] < 0) continue;
-      if (kb[k] < lo || kb[k] >= it.hi) { bad = true; kb[k] = -1; continue; }
       uint32_t h = (hr_hash(kb[k]) >> hshift) & hmask;
       while (true) {
         const int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
@@ -136,12 +140,10 @@ __global__ void __launch_bounds__(NT, NT == 128 ? 9 : 1024 / NT) k_hrank(RowsArg
         slot[k] |= bk << 16;  // slot < 2^14, bucket < 2^13
       }
     }
-    if (bad) atomicOr(A.err, ERR_INTERNAL);
-    if (wrap) atomicOr(A.err, ERR_OVERFLOW);
+    if (wrap) atomicOr(err, ERR_OVERFLOW);
     __syncthreads();
     // ---- 2. bucket offsets; owners place their key in bucket order
     const int D = hr_scan<NT>(S.cnt, S.offs, NB, S.wsum);
-    if (D > kCapE) atomicOr(A.err, ERR_INTERNAL);
     __syncthreads();
     int boff[8];
 #pragma unroll
@@ -162,7 +164,7 @@ __global__ void __launch_bounds__(NT, NT == 128 ? 9 : 1024 / NT) k_hrank(RowsArg
       for (int j = boff[k]; j < bend; ++j) r += S.scr[j] < kb[k];
       const int h = slot[k] & 0xffff;
       const uint32_t sum = S.val[h];
-      if (sum > 0x7fffffffu) atomicOr(A.err, ERR_OVERFLOW);
+      if (sum > 0x7fffffffu) atomicOr(err, ERR_OVERFLOW);
       src_b[r] = kb[k];
       src_w[r] = (int32_t)sum;
       S.key[h] = kEmpty;
