@@ -397,97 +397,122 @@ __global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restr
 // then the M gathers).  No shared memory, no CTA barriers.
 constexpr int kXBig = 64;
 
-__device__ __forceinline__ void x2_copy4(const Layout &L, int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
-                                         const int64_t (&e)[4], const int64_t (&p)[4], unsigned ok) {
-  int32_t b[4], w[4];
-#pragma unroll
-  for (int u = 0; u < 4; ++u)
-    if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
-#pragma unroll
-  for (int u = 0; u < 4; ++u)
-    if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
-#pragma unroll
-  for (int u = 0; u < 4; ++u)
-    if (ok & (1u << u)) { __stcs(Sb + p[u], b[u]); __stcs(Sw + p[u], w[u]); }
-}
-
-__global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
-                                               int32_t *__restrict__ Sb, int32_t *__restrict__ Sw) {
-  const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
-  const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
+// Walk the member-edge positions [P, Pend) (all inside members [.., m_hi)):
+// sink(e[4], p[4], ok) receives, per step, up to four positions per lane (e:
+// source entry in col/wgt, p: position).  With skip != nullptr, members whose
+// coarse row has skip[M[member]] >= 0 are passed over (DENSE rows, expanded by
+// their accumulation kernel instead).
+template <typename Sink>
+__device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restrict__ mstart, int64_t m_lo,
+                                        int64_t m_hi, int64_t P, int64_t Pend, const int32_t *__restrict__ skip,
+                                        Sink &sink) {
   const int lane = threadIdx.x & 31;
-  const int64_t gw = ((int64_t)blockIdx.x * kXT + threadIdx.x) >> 5;
-  const int64_t nw = ((int64_t)gridDim.x * kXT) >> 5;
-  for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
-    const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
-    int64_t i = warp_find_member(L, m_lo, m_hi, P);
-    while (true) {
-      const int64_t j = i + lane;
-      int64_t mp0 = P_hi, mp1 = P_hi, rs = 0;
-      if (j < m_hi) { mp0 = L.mpre[j]; mp1 = L.mpre[j + 1]; rs = mstart[j]; }
-      const int64_t ps = mp0 > P ? mp0 : P;
-      const int64_t pe = mp1 < Pend ? mp1 : Pend;
-      const int d = pe > ps ? (int)(pe - ps) : 0;
-      rs += ps - mp0;  // source entry of position ps
-      const int64_t pr = ps - P_lo;  // staging index of position ps
-      const bool big = d > kXBig;
-      // ---- packed short members
-      const int ds = big ? 0 : d;
-      int incl = ds;
+  int64_t i = warp_find_member(L, m_lo, m_hi, P);
+  while (true) {
+    const int64_t j = i + lane;
+    int64_t mp0 = L.mpre[m_hi], mp1 = mp0, rs = 0;
+    bool skipped = false;
+    if (j < m_hi) {
+      mp0 = L.mpre[j];
+      mp1 = L.mpre[j + 1];
+      rs = mstart[j];
+      if (skip) skipped = skip[L.M[L.members[j]]] >= 0;
+    }
+    const int64_t ps = mp0 > P ? mp0 : P;
+    const int64_t pe = mp1 < Pend ? mp1 : Pend;
+    const int d = (pe > ps && !skipped) ? (int)(pe - ps) : 0;
+    rs += ps - mp0;  // source entry of position ps
+    const bool big = d > kXBig;
+    // ---- packed short members
+    const int ds = big ? 0 : d;
+    int incl = ds;
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += y;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    const int excl = incl - ds;
+    const int T = __shfl_sync(0xffffffffu, incl, 31);
+    for (int base = 0; base < T; base += 128) {
+      int64_t e[4], p[4];
+      unsigned ok = 0;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int t = base + lane + 32 * u;
+        int lo = 0;  // largest lane with excl <= t
+#pragma unroll
+        for (int st = 16; st > 0; st >>= 1) {
+          const int c = lo + st;
+          const int v = __shfl_sync(0xffffffffu, excl, c & 31);
+          if (c < 32 && v <= t) lo = c;
+        }
+        const int64_t ors = __shfl_sync(0xffffffffu, rs, lo);
+        const int64_t ops = __shfl_sync(0xffffffffu, ps, lo);
+        const int oex = __shfl_sync(0xffffffffu, excl, lo);
+        e[u] = ors + (t - oex);
+        p[u] = ops + (t - oex);
+        if (t < T) ok |= 1u << u;
       }
-      const int excl = incl - ds;
-      const int T = __shfl_sync(0xffffffffu, incl, 31);
-      for (int base = 0; base < T; base += 128) {
+      sink(e, p, ok);
+    }
+    // ---- long members, one at a time
+    unsigned bm = __ballot_sync(0xffffffffu, big);
+    while (bm) {
+      const int src = __ffs(bm) - 1;
+      bm &= bm - 1;
+      const int bd = __shfl_sync(0xffffffffu, d, src);
+      const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
+      const int64_t bps = __shfl_sync(0xffffffffu, ps, src);
+      for (int base = 0; base < bd; base += 128) {
         int64_t e[4], p[4];
         unsigned ok = 0;
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const int t = base + lane + 32 * u;
-          int lo = 0;  // largest lane with excl <= t
-#pragma unroll
-          for (int st = 16; st > 0; st >>= 1) {
-            const int c = lo + st;
-            const int v = __shfl_sync(0xffffffffu, excl, c & 31);
-            if (c < 32 && v <= t) lo = c;
-          }
-          const int64_t ors = __shfl_sync(0xffffffffu, rs, lo);
-          const int64_t opr = __shfl_sync(0xffffffffu, pr, lo);
-          const int oex = __shfl_sync(0xffffffffu, excl, lo);
-          e[u] = ors + (t - oex);
-          p[u] = opr + (t - oex);
-          if (t < T) ok |= 1u << u;
+          e[u] = brs + t;
+          p[u] = bps + t;
+          if (t < bd) ok |= 1u << u;
         }
-        x2_copy4(L, Sb, Sw, e, p, ok);
+        sink(e, p, ok);
       }
-      // ---- long members, one at a time
-      unsigned bm = __ballot_sync(0xffffffffu, big);
-      while (bm) {
-        const int src = __ffs(bm) - 1;
-        bm &= bm - 1;
-        const int bd = __shfl_sync(0xffffffffu, d, src);
-        const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
-        const int64_t bpr = __shfl_sync(0xffffffffu, pr, src);
-        for (int base = 0; base < bd; base += 128) {
-          int64_t e[4], p[4];
-          unsigned ok = 0;
-#pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            const int t = base + lane + 32 * u;
-            e[u] = brs + t;
-            p[u] = bpr + t;
-            if (t < bd) ok |= 1u << u;
-          }
-          x2_copy4(L, Sb, Sw, e, p, ok);
-        }
-      }
-      // the window reaches the chunk end (or the last member): done
-      if (__any_sync(0xffffffffu, mp1 >= Pend)) break;
-      i += 32;
     }
+    // the window reaches the chunk end (or the last member): done
+    if (__any_sync(0xffffffffu, mp1 >= Pend)) break;
+    i += 32;
+  }
+}
+
+// sink of the expansion: (M[v], w) to the staging at position - P_lo
+struct StageSink {
+  const Layout &L;
+  int32_t *__restrict__ Sb, *__restrict__ Sw;
+  int64_t P_lo;
+  __device__ __forceinline__ void operator()(const int64_t (&e)[4], const int64_t (&p)[4], unsigned ok) {
+    int32_t b[4], w[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (ok & (1u << u)) { __stcs(Sb + (p[u] - P_lo), b[u]); __stcs(Sw + (p[u] - P_lo), w[u]); }
+  }
+};
+
+// skip: big_idx in DENSE mode (those rows are expanded by k_dense_accum2), else nullptr
+__global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
+                                               int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
+                                               const int32_t *__restrict__ skip) {
+  const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
+  const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
+  const int64_t gw = ((int64_t)blockIdx.x * kXT + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * kXT) >> 5;
+  StageSink sink{L, Sb, Sw, P_lo};
+  for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
+    const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
+    x2_walk(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
   }
 }
 
@@ -1077,6 +1102,80 @@ __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
   }
 }
 
+// DENSE rows fused with their expansion: a persistent CTA takes units of
+// kDenseUnit member-edge positions of one big row; each warp walks its
+// kDenseUnit/16 positions of the row's member rows (x2_walk), gathers M[v] and
+// adds w into the shared-memory accumulator of the row (uint32: a partial sum
+// above INT32_MAX or a wrap means the coarse weight overflows -- ERR_OVERFLOW
+// here or in k_rows); the accumulator is merged into dense[h] when the CTA
+// moves to another row.  The staging is never written for these rows.
+struct AccSink {
+  const Layout &L;
+  uint32_t *acc;
+  int32_t a;
+  bool wrap;
+  __device__ __forceinline__ void operator()(const int64_t (&e)[4], const int64_t (&p)[4], unsigned ok) {
+    (void)p;
+    int32_t b[4], w[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if ((ok & (1u << u)) && b[u] != a) {  // self entries dropped (L280)
+        const uint32_t o = atomicAdd(acc + b[u], (uint32_t)w[u]);
+        wrap |= o + (uint32_t)w[u] < o;
+      }
+  }
+};
+
+__global__ void __launch_bounds__(kT) k_dense_accum2(DenseArgs A, const int64_t *__restrict__ mstart,
+                                                    int *__restrict__ err) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  uint32_t *acc = reinterpret_cast<uint32_t *>(smem_raw);
+  __shared__ int64_t s_unit;
+  const Layout &L = A.L;
+  const int nc = (int)L.n_c;
+  const int wid = threadIdx.x >> 5;
+  constexpr int kSlice = kDenseUnit / (kT / 32);
+  for (int b = threadIdx.x; b < nc; b += kT) acc[b] = 0u;
+  int64_t cur_h = -1;
+  bool wrap = false;
+  while (true) {
+    if (threadIdx.x == 0) s_unit = (int64_t)atomicAdd(A.ticket, 1u);
+    __syncthreads();
+    const int64_t unit = s_unit;
+    const int64_t h = unit < A.nunits ? A.unit_row[unit] : -1;
+    if (cur_h >= 0 && h != cur_h) {  // merge the accumulator of the previous row
+      unsigned long long *dst = A.dense + cur_h * (int64_t)nc;
+      for (int b = threadIdx.x; b < nc; b += kT) {
+        const uint32_t v = acc[b];
+        if (v) {
+          if (v > 0x7fffffffu) wrap = true;
+          atomicAdd(dst + b, (unsigned long long)v);
+          acc[b] = 0u;
+        }
+      }
+      __syncthreads();
+    }
+    if (h < 0) break;
+    cur_h = h;
+    const int32_t a = A.big_list[h];
+    const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kDenseUnit;
+    const int64_t Pe = min(P0 + (int64_t)kDenseUnit, L.upos(a + 1));
+    const int64_t Pw = P0 + (int64_t)wid * kSlice;
+    const int64_t Pwe = min(Pw + (int64_t)kSlice, Pe);
+    AccSink sink{L, acc, a, false};
+    if (Pw < Pwe) x2_walk(L, mstart, L.member_ptr[a], L.member_ptr[a + 1], Pw, Pwe, nullptr, sink);
+    wrap |= sink.wrap;
+    __syncthreads();
+  }
+  if (wrap) atomicOr(err, ERR_OVERFLOW);
+}
+
 // ---------------------------------------------------------------- driver
 size_t ws_bytes_construct(int64_t n, int64_t nnz, int64_t n_c) {
   (void)nnz;
@@ -1161,6 +1260,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t n_out = a_hi - a_lo;  // rows produced by this call
   Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi};
   const bool dense = n_c <= kDenseMax;
+  // DENSE rows expanded inside their accumulation (HEC_DENSE_STAGED: staged v1, test hook)
+  const bool fused_dense = dense && getenv("HEC_DENSE_STAGED") == nullptr;
   // bitmap-rank items replace the bin pieces when the key range fits the
   // shared-memory bitmap (HEC_NO_RBM: test / tuning hook for the bin-piece path)
   const bool rbm = !dense && n_c <= kRbmRange && getenv("HEC_NO_RBM") == nullptr;
@@ -1240,7 +1341,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     if (grid > cap) grid = cap;
     if (grid > 0) {
       if (getenv("HEC_EXPAND_V1")) k_expand<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
-      else k_expand2<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
+      else k_expand2<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, fused_dense ? big_idx : nullptr);
       HEC_LAUNCH_CHECK();
     }
     phase_end(ctx, phx);
@@ -1275,6 +1376,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
                                       (int)sizeof(FbSmem)));
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_dense_accum, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)(4 * kDenseMax)));
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_dense_accum2, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)(4 * kDenseMax)));
     attr = true;
   }
 
@@ -1292,9 +1395,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_CUDA_TRY(cudaMemsetAsync(dn_arr, 0, sizeof(unsigned long long) * nbig * n_c, s));
     DenseArgs D{L, big_list, nbig, unit_ptr, unit_row, nunits, counts + 2, dn_arr, sc_col, sc_wgt};
     int occ = 1;
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum, kT, 4 * (size_t)n_c));
+    if (fused_dense) HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum2, kT, 4 * (size_t)n_c));
+    else HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum, kT, 4 * (size_t)n_c));
     if (occ < 1) occ = 1;
-    k_dense_accum<<<ctx->num_sms * occ, kT, 4 * (size_t)n_c, s>>>(D);
+    if (fused_dense) k_dense_accum2<<<ctx->num_sms * occ, kT, 4 * (size_t)n_c, s>>>(D, mstart, err);
+    else k_dense_accum<<<ctx->num_sms * occ, kT, 4 * (size_t)n_c, s>>>(D);
     HEC_LAUNCH_CHECK();
     A.dense = dn_arr;
   } else if (nbig > 0) {

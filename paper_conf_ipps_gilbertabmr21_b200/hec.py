@@ -11,6 +11,7 @@ build_coarse_graph.
 from __future__ import annotations
 
 import ctypes
+import weakref
 from dataclasses import dataclass
 
 import torch
@@ -96,6 +97,7 @@ class Context:
             check(L.hec_ctx_create(ctypes.c_void_p(self.stream.cuda_stream), self._alloc_cb,
                                    self._free_cb, None, ctypes.byref(h)), "hec_ctx_create")
         self.h = h
+        self._owned = weakref.WeakSet()  # live results: freed before the context
         if validate:
             self.set_validate(True)
 
@@ -128,6 +130,8 @@ class Context:
 
     def close(self):
         if getattr(self, "h", None):
+            for r in list(getattr(self, "_owned", ())):
+                r.free()  # results use the context's allocator: free them first
             load().hec_ctx_destroy(self.h)
             self.h = None
 
@@ -229,6 +233,7 @@ class CoarseGraph:
 
     def __init__(self, ctx: Context, handle: ctypes.c_void_p):
         self.ctx, self.h = ctx, handle
+        ctx._owned.add(self)
         v = HecGraph()
         check(load().hec_csr_view(handle, ctypes.byref(v)), "hec_csr_view")
         self.graph = _graph_from_view(ctx, v)
@@ -268,6 +273,7 @@ class Hierarchy:
     def __init__(self, ctx: Context, handle: ctypes.c_void_p):
         L = load()
         self.ctx, self.h = ctx, handle
+        ctx._owned.add(self)
         self.stop_reason = L.hec_hierarchy_stop_reason(handle)
         self.discarded_n_c = int(L.hec_hierarchy_discarded_n_c(handle))
         self.levels: list[Level] = []

@@ -221,7 +221,7 @@ def test_construct_random_labels(P, ctx):
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["rbm", "bins"])
+@pytest.mark.parametrize("path", ["rbm", "bins", "staged"])
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
 def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     """R-MAT with random labels into nc aggregates: few labels give huge rows
@@ -232,6 +232,10 @@ def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
         if nc <= 32768:
             pytest.skip("DENSE mode: no bitmap-rank items")
         monkeypatch.setenv("HEC_NO_RBM", "1")
+    if path == "staged":  # DENSE rows through the staging (v1) instead of the fused expansion
+        if nc > 32768:
+            pytest.skip("BUCKET mode: no DENSE rows")
+        monkeypatch.setenv("HEC_DENSE_STAGED", "1")
     rng = np.random.default_rng(15 + nc)
     g = gg.rmat(14 if nc < 20000 else 17, 16)
     g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
@@ -315,6 +319,28 @@ def test_construct_rbm_rank_windows(P, ctx):
     M[rng.permutation(rest)[:nc]] = np.arange(nc)
     cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
+
+
+@pytest.mark.parametrize("staged", [False, True])
+def test_construct_dense_row_overflow(P, ctx, staged, monkeypatch):
+    """A DENSE skewed row (a hub whose 6000 leaves collapse onto one coarse
+    vertex): a coarse weight above INT32_MAX is reported, one just below is exact."""
+    if staged:
+        monkeypatch.setenv("HEC_DENSE_STAGED", "1")
+    n = 6001
+    M = np.ones(n, np.int32)
+    M[0] = 0
+    M[1] = 2  # a third aggregate keeps the hub row's keys from being a single value
+    for w, ok in ((2**20, False), ((2**31 - 1) // 6000, True)):
+        g = gg.from_edges(n, [(0, v, w) for v in range(1, n)])
+        Mt = torch.from_numpy(M).cuda()
+        if ok:
+            cg = P.build_coarse_graph(ctx, dev(P, g), Mt, 3)
+            assert_csr_equal(cg.graph, o.coarsen(g, M, 3))
+        else:
+            with pytest.raises(P.HecError) as e:
+                P.build_coarse_graph(ctx, dev(P, g), Mt, 3)
+            assert e.value.code == P.HEC_EOVERFLOW
 
 
 def test_construct_overflow_detected(P, ctx):
