@@ -402,7 +402,7 @@ constexpr int kXBig = 64;
 // source entry in col/wgt, p: position).  With skip != nullptr, members whose
 // coarse row has skip[M[member]] >= 0 are passed over (DENSE rows, expanded by
 // their accumulation kernel instead).
-template <typename Sink>
+template <int kLong, typename Sink>
 __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restrict__ mstart, int64_t m_lo,
                                         int64_t m_hi, int64_t P, int64_t Pend, const int32_t *__restrict__ skip,
                                         Sink &sink) {
@@ -463,11 +463,11 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
       const int bd = __shfl_sync(0xffffffffu, d, src);
       const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
       const int64_t bps = __shfl_sync(0xffffffffu, ps, src);
-      for (int base = 0; base < bd; base += 128) {
-        int64_t e[4], p[4];
+      for (int base = 0; base < bd; base += 32 * kLong) {  // kLong positions per lane in flight
+        int64_t e[kLong], p[kLong];
         unsigned ok = 0;
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
+        for (int u = 0; u < kLong; ++u) {
           const int t = base + lane + 32 * u;
           e[u] = brs + t;
           p[u] = bps + t;
@@ -487,16 +487,17 @@ struct StageSink {
   const Layout &L;
   int32_t *__restrict__ Sb, *__restrict__ Sw;
   int64_t P_lo;
-  __device__ __forceinline__ void operator()(const int64_t (&e)[4], const int64_t (&p)[4], unsigned ok) {
-    int32_t b[4], w[4];
+  template <int N>
+  __device__ __forceinline__ void operator()(const int64_t (&e)[N], const int64_t (&p)[N], unsigned ok) {
+    int32_t b[N], w[N];
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) { __stcs(Sb + (p[u] - P_lo), b[u]); __stcs(Sw + (p[u] - P_lo), w[u]); }
   }
 };
@@ -512,7 +513,7 @@ __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__rest
   StageSink sink{L, Sb, Sw, P_lo};
   for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
     const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
-    x2_walk(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
+    x2_walk<4>(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
   }
 }
 
@@ -1114,17 +1115,18 @@ struct AccSink {
   uint32_t *acc;
   int32_t a;
   bool wrap;
-  __device__ __forceinline__ void operator()(const int64_t (&e)[4], const int64_t (&p)[4], unsigned ok) {
+  template <int N>
+  __device__ __forceinline__ void operator()(const int64_t (&e)[N], const int64_t (&p)[N], unsigned ok) {
     (void)p;
-    int32_t b[4], w[4];
+    int32_t b[N], w[N];
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < N; ++u)
       if ((ok & (1u << u)) && b[u] != a) {  // self entries dropped (L280)
         const uint32_t o = atomicAdd(acc + b[u], (uint32_t)w[u]);
         wrap |= o + (uint32_t)w[u] < o;
@@ -1169,7 +1171,7 @@ __global__ void __launch_bounds__(kT) k_dense_accum2(DenseArgs A, const int64_t 
     const int64_t Pw = P0 + (int64_t)wid * kSlice;
     const int64_t Pwe = min(Pw + (int64_t)kSlice, Pe);
     AccSink sink{L, acc, a, false};
-    if (Pw < Pwe) x2_walk(L, mstart, L.member_ptr[a], L.member_ptr[a + 1], Pw, Pwe, nullptr, sink);
+    if (Pw < Pwe) x2_walk<8>(L, mstart, L.member_ptr[a], L.member_ptr[a + 1], Pw, Pwe, nullptr, sink);
     wrap |= sink.wrap;
     __syncthreads();
   }

@@ -286,26 +286,26 @@ __global__ void k_span_coords(int64_t n, int64_t nnz, const int64_t *__restrict_
 // aggregates per span, then the lane's first row end (which may continue a row
 // from earlier lanes or spans) is resolved with the scanned prefix.
 // kVec: col/wgt share a 16-byte phase (int4 loads); else scalar loads.
+struct SegArgs {
+  int64_t n, nnz;
+  const int64_t *rp;
+  int64_t ebase, vbase, x0, off, nspans;
+  const int32_t *colA, *wgtA;
+  const int32_t *cx;
+  int32_t *H;
+  uint64_t *head_key, *mid_key;
+};
+
+// lane's 16 consecutive entries of span k (4 x 16 B of col and of wgt, or scalars)
 template <bool kVec>
-__global__ void __launch_bounds__(32 * kSegWarps, 3) k_heavy_seg(
-    int64_t n, int64_t nnz, const int64_t *__restrict__ rp, int64_t ebase, int64_t vbase, int64_t x0, int64_t off,
-    int64_t nspans, const int32_t *__restrict__ colA, const int32_t *__restrict__ wgtA,
-    const int32_t *__restrict__ cx, int32_t *__restrict__ H, uint64_t *__restrict__ head_key,
-    uint64_t *__restrict__ mid_key) {
-  __shared__ SegWarpSmem smem[kSegWarps];
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const int64_t k = blockIdx.x * (int64_t)kSegWarps + wid;
-  if (k >= nspans) return;
-  SegWarpSmem &W = smem[wid];
-  const int64_t xs = x0 + k * kSpan;          // aligned index of the span start
-  const int64_t es = xs - off;                // entry index of the span start
-  const int64_t elo = ebase, ehi = ebase + nnz;
+__device__ __forceinline__ void seg_load(const SegArgs &A, int64_t k, int (&cc)[16], int (&ww)[16]) {
+  const int lane = threadIdx.x & 31;
+  const int64_t xs = A.x0 + k * kSpan, es = xs - A.off;
+  const int64_t elo = A.ebase, ehi = A.ebase + A.nnz;
   const bool interior = es >= elo && es + kSpan <= ehi;
-  // ---- loads first (lane: 16 consecutive entries = 4 x 16 B of col and of wgt)
-  int cc[16], ww[16];
   if (kVec) {
-    const int4 *c4 = reinterpret_cast<const int4 *>(colA + xs) + 4 * lane;
-    const int4 *w4 = reinterpret_cast<const int4 *>(wgtA + xs) + 4 * lane;
+    const int4 *c4 = reinterpret_cast<const int4 *>(A.colA + xs) + 4 * lane;
+    const int4 *w4 = reinterpret_cast<const int4 *>(A.wgtA + xs) + 4 * lane;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       const int64_t e0 = es + 16 * lane + 4 * j;
@@ -320,17 +320,28 @@ __global__ void __launch_bounds__(32 * kSegWarps, 3) k_heavy_seg(
       const int64_t e = es + 16 * lane + q;
       cc[q] = 0;
       ww[q] = 0;
-      if (interior || (e >= elo && e < ehi)) { cc[q] = __ldcs(colA + e); ww[q] = __ldcs(wgtA + e); }
+      if (interior || (e >= elo && e < ehi)) { cc[q] = __ldcs(A.colA + e); ww[q] = __ldcs(A.wgtA + e); }
     }
   }
-  // ---- row starts / ends inside the span
+}
+
+// Span k with its entries in cc/ww: row starts/ends of the span as warp-private
+// bitmaps, lane-sequential segmented max, ONE warp scan of the lane aggregates,
+// then the lane's first row end (which may continue a row from earlier lanes or
+// spans) resolved with the scanned prefix.
+__device__ __forceinline__ void seg_process(const SegArgs &A, int64_t k, SegWarpSmem &W, const int (&cc)[16],
+                                            int (&ww)[16]) {
+  const int lane = threadIdx.x & 31;
+  const int64_t xs = A.x0 + k * kSpan, es = xs - A.off;
+  const int64_t elo = A.ebase, ehi = A.ebase + A.nnz;
+  const bool interior = es >= elo && es + kSpan <= ehi;
   if (lane < kSpan / 32) { W.head[lane] = 0u; W.end[lane] = 0u; }
   __syncwarp();
-  const int64_t r0 = cx[k], r1 = cx[k + 1];
+  const int64_t r0 = A.cx[k], r1 = A.cx[k + 1];
   for (int64_t r = r0 + lane; r <= r1; r += 32) {
-    const int64_t s = __ldg(rp + r), e = __ldg(rp + r + 1);
+    const int64_t s = __ldg(A.rp + r), e = __ldg(A.rp + r + 1);
     if (s == e) {
-      H[vbase + r] = (int32_t)(vbase + r);  // isolated (idempotent)
+      A.H[A.vbase + r] = (int32_t)(A.vbase + r);  // isolated (idempotent)
       continue;
     }
     const int64_t ps = s - es, pe = e - 1 - es;
@@ -341,7 +352,6 @@ __global__ void __launch_bounds__(32 * kSegWarps, 3) k_heavy_seg(
     }
   }
   __syncwarp();
-  // ---- lane-sequential segmented max
   const unsigned hb = (W.head[lane >> 1] >> (16 * (lane & 1))) & 0xffffu;
   const unsigned eb = (W.end[lane >> 1] >> (16 * (lane & 1))) & 0xffffu;
   if (!interior) {
@@ -359,11 +369,10 @@ __global__ void __launch_bounds__(32 * kSegWarps, 3) k_heavy_seg(
     if ((hb >> q) & 1u) run = key;
     else run = key > run ? key : run;
     if ((eb >> q) & 1u) {
-      if (hb & ((2u << q) - 1u)) H[vbase + W.endrow[16 * lane + q]] = key_vertex(run);
+      if (hb & ((2u << q) - 1u)) A.H[A.vbase + W.endrow[16 * lane + q]] = key_vertex(run);
       else if (pend_q < 0) { pend = run; pend_q = q; }
     }
   }
-  // ---- warp scan of the lane aggregates (segmented by "lane has a row start")
   bool stop = hb != 0u || lane == 0;
   uint64_t incl = run;
 #pragma unroll
@@ -380,12 +389,38 @@ __global__ void __launch_bounds__(32 * kSegWarps, 3) k_heavy_seg(
   const unsigned hm = __ballot_sync(0xffffffffu, hb != 0u);
   if (pend_q >= 0) {
     const uint64_t v = pre > pend ? pre : pend;
-    if (hm & ((1u << lane) - 1u)) H[vbase + W.endrow[16 * lane + pend_q]] = key_vertex(v);
-    else head_key[k] = v;  // the row began in an earlier span
+    if (hm & ((1u << lane) - 1u)) A.H[A.vbase + W.endrow[16 * lane + pend_q]] = key_vertex(v);
+    else A.head_key[k] = v;  // the row began in an earlier span
   }
   if (lane == 31) {
     const uint64_t last = hb ? run : (pre > run ? pre : run);
-    mid_key[k] = (eb >> 15) & 1u ? 0ull : last;
+    A.mid_key[k] = (eb >> 15) & 1u ? 0ull : last;
+  }
+  __syncwarp();
+}
+
+// Persistent warps stride over the spans; the next span's 8 x 16 B per lane are
+// loaded before the current span is processed, so every warp keeps a span of
+// loads in flight while it computes.
+template <bool kVec>
+__global__ void __launch_bounds__(32 * kSegWarps, 2) k_heavy_seg(SegArgs A) {
+  __shared__ SegWarpSmem smem[kSegWarps];
+  const int wid = threadIdx.x >> 5;
+  SegWarpSmem &W = smem[wid];
+  const int64_t nw = (int64_t)gridDim.x * kSegWarps;
+  int64_t k = blockIdx.x * (int64_t)kSegWarps + wid;
+  if (k >= A.nspans) return;
+  int cc[16], ww[16];
+  seg_load<kVec>(A, k, cc, ww);
+  while (true) {
+    const int64_t kn = k + nw;
+    int nc[16], nw_[16];
+    if (kn < A.nspans) seg_load<kVec>(A, kn, nc, nw_);
+    seg_process(A, k, W, cc, ww);
+    if (kn >= A.nspans) break;
+    k = kn;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) { cc[q] = nc[q]; ww[q] = nw_[q]; }
   }
 }
 
@@ -460,13 +495,18 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
     HEC_CUDA_TRY(cudaMemsetAsync(head, 0, sizeof(uint64_t) * nspans, ctx->stream));
     k_span_coords<<<nblk(nspans + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, x0, off, nspans, cx);
     HEC_LAUNCH_CHECK();
-    const int32_t *colA = g->col - off, *wgtA = g->wgt - off;
-    if (vec)
-      k_heavy_seg<true><<<nblk(nspans, kSegWarps), 32 * kSegWarps, 0, ctx->stream>>>(
-          n, nnz, rp, ebase, u0, x0, off, nspans, colA, wgtA, cx, H, head, mid);
-    else
-      k_heavy_seg<false><<<nblk(nspans, kSegWarps), 32 * kSegWarps, 0, ctx->stream>>>(
-          n, nnz, rp, ebase, u0, x0, off, nspans, colA, wgtA, cx, H, head, mid);
+    SegArgs SA{n, nnz, rp, ebase, u0, x0, off, nspans, g->col - off, g->wgt - off, cx, H, head, mid};
+    static int occ[2] = {0, 0};
+    if (!occ[vec]) {
+      if (vec) HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_heavy_seg<true>, 32 * kSegWarps, 0));
+      else HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_heavy_seg<false>, 32 * kSegWarps, 0));
+      if (occ[vec] < 1) occ[vec] = 1;
+    }
+    int64_t grid = (int64_t)ctx->num_sms * occ[vec];
+    const int64_t want = (nspans + kSegWarps - 1) / kSegWarps;
+    if (want < grid) grid = want;
+    if (vec) k_heavy_seg<true><<<(unsigned)grid, 32 * kSegWarps, 0, ctx->stream>>>(SA);
+    else k_heavy_seg<false><<<(unsigned)grid, 32 * kSegWarps, 0, ctx->stream>>>(SA);
     HEC_LAUNCH_CHECK();
     k_heavy_seg_fixup<<<nblk(nspans * 32, 256), 256, 0, ctx->stream>>>(rp, u0, x0, off, nspans, cx, head, mid, H);
     HEC_LAUNCH_CHECK();
