@@ -1032,6 +1032,7 @@ struct DenseArgs {
 // (one 4096-entry unit per round trip left the kernel latency-bound).
 constexpr int kDenseIt = 16;
 constexpr int kDenseUnit = kT * kDenseIt;
+constexpr int kDenseUnit2 = 4 * kDenseUnit;  // fused DENSE units: 2048 positions per warp, one barrier
 
 __global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -1142,7 +1143,7 @@ __global__ void __launch_bounds__(kT) k_dense_accum2(DenseArgs A, const int64_t 
   const Layout &L = A.L;
   const int nc = (int)L.n_c;
   const int wid = threadIdx.x >> 5;
-  constexpr int kSlice = kDenseUnit / (kT / 32);
+  constexpr int kSlice = kDenseUnit2 / (kT / 32);
   for (int b = threadIdx.x; b < nc; b += kT) acc[b] = 0u;
   int64_t cur_h = -1;
   bool wrap = false;
@@ -1166,8 +1167,8 @@ __global__ void __launch_bounds__(kT) k_dense_accum2(DenseArgs A, const int64_t 
     if (h < 0) break;
     cur_h = h;
     const int32_t a = A.big_list[h];
-    const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kDenseUnit;
-    const int64_t Pe = min(P0 + (int64_t)kDenseUnit, L.upos(a + 1));
+    const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kDenseUnit2;
+    const int64_t Pe = min(P0 + (int64_t)kDenseUnit2, L.upos(a + 1));
     const int64_t Pw = P0 + (int64_t)wid * kSlice;
     const int64_t Pwe = min(Pw + (int64_t)kSlice, Pe);
     AccSink sink{L, acc, a, false};
@@ -1284,7 +1285,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t small_vol = r0[1], big_vol = r0[2];
   const int64_t nbig = r0[4] & 0xffffffffLL;
   if (nbig > 0) {
-    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)kDenseUnit : (int64_t)kUnit,
+    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)(fused_dense ? kDenseUnit2 : kDenseUnit) : (int64_t)kUnit,
                                              dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
                          st[4], unit_ptr + nbig));
     if (!dense) HEC_TRY(chained_scan(ctx, nbig, BucketsIn{L, big_list, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + nbig));

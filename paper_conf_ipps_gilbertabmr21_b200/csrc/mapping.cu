@@ -425,29 +425,24 @@ __global__ void __launch_bounds__(32 * kSegWarps, 2) k_heavy_seg(SegArgs A) {
 }
 
 // Rows that end in span k but began in an earlier span s0: max of span k's head
-// value and the mid values of spans s0 .. k-1.  One warp per span.
+// value and the mid values of spans s0 .. k-1.  One thread per span (a row
+// longer than a few spans is rare; its thread loops over independent loads).
 __global__ void k_heavy_seg_fixup(const int64_t *__restrict__ rp, int64_t vbase, int64_t x0, int64_t off,
                                   int64_t nspans, const int32_t *__restrict__ cx,
                                   const uint64_t *__restrict__ head_key, const uint64_t *__restrict__ mid_key,
                                   int32_t *__restrict__ H) {
-  const int lane = threadIdx.x & 31;
-  const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= nspans) return;
-  uint64_t key = head_key[k];
-  if (key == 0ull) return;
+  uint64_t m = head_key[k];
+  if (m == 0ull) return;
   const int32_t x = cx[k];
   const int64_t s0 = (__ldg(rp + x) + off - x0) / kSpan;
-  uint64_t m = lane == 0 ? key : 0ull;
-  for (int64_t s = s0 + lane; s < k; s += 32) {
+#pragma unroll 4
+  for (int64_t s = s0; s < k; ++s) {
     const uint64_t y = mid_key[s];
     m = y > m ? y : m;
   }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const uint64_t y = __shfl_xor_sync(0xffffffffu, m, o);
-    m = y > m ? y : m;
-  }
-  if (lane == 0) H[vbase + x] = key_vertex(m);
+  H[vbase + x] = key_vertex(m);
 }
 
 static size_t heavy_ws(int64_t n, int64_t nnz) {
@@ -508,7 +503,7 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
     if (vec) k_heavy_seg<true><<<(unsigned)grid, 32 * kSegWarps, 0, ctx->stream>>>(SA);
     else k_heavy_seg<false><<<(unsigned)grid, 32 * kSegWarps, 0, ctx->stream>>>(SA);
     HEC_LAUNCH_CHECK();
-    k_heavy_seg_fixup<<<nblk(nspans * 32, 256), 256, 0, ctx->stream>>>(rp, u0, x0, off, nspans, cx, head, mid, H);
+    k_heavy_seg_fixup<<<nblk(nspans, 256), 256, 0, ctx->stream>>>(rp, u0, x0, off, nspans, cx, head, mid, H);
     HEC_LAUNCH_CHECK();
     return HEC_OK;
   }
