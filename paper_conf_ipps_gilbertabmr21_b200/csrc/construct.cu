@@ -599,27 +599,30 @@ __device__ __forceinline__ void unit_hist(const PartArgs &A, const UnitInfo &u, 
   __syncthreads();
 }
 
-__global__ void __launch_bounds__(kT) k_part_count(PartArgs A, unsigned *__restrict__ bkt_cnt) {
+// The unit's slice of each bin is reserved here: the returned running count
+// is the unit's offset inside the bin (ubase), so the write pass needs no
+// second histogram.
+__global__ void __launch_bounds__(kT) k_part_count(PartArgs A, unsigned *__restrict__ bkt_cnt,
+                                                   int32_t *__restrict__ ubase) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   const UnitInfo u = unit_info(A, blockIdx.x);
   unit_hist(A, u, S);
+  int32_t *ub = ubase + (int64_t)blockIdx.x * kPartHist;
   for (int i = threadIdx.x; i < u.nb; i += kT)
-    if (S.hist[i]) atomicAdd(bkt_cnt + u.b0 + i, (unsigned)S.hist[i]);
+    if (S.hist[i]) ub[i] = (int32_t)atomicAdd(bkt_cnt + u.b0 + i, (unsigned)S.hist[i]);
 }
 
 __global__ void __launch_bounds__(kT) k_part_write(PartArgs A, const int64_t *__restrict__ bkt_off,
-                                                   unsigned *__restrict__ bkt_cur, int32_t *__restrict__ pb,
+                                                   const int32_t *__restrict__ ubase, int32_t *__restrict__ pb,
                                                    int32_t *__restrict__ pw) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   const UnitInfo u = unit_info(A, blockIdx.x);
-  unit_hist(A, u, S);
   const int64_t off0 = bkt_off[u.b0];
-  for (int i = threadIdx.x; i < u.nb; i += kT) {
-    const int c = S.hist[i];
-    if (c) S.base[i] = (int32_t)(bkt_off[u.b0 + i] - off0) + (int32_t)atomicAdd(bkt_cur + u.b0 + i, (unsigned)c);
-  }
+  const int32_t *ub = ubase + (int64_t)blockIdx.x * kPartHist;
+  for (int i = threadIdx.x; i < u.nb; i += kT)  // (slots of bins the unit never hits stay unused)
+    S.base[i] = (int32_t)(bkt_off[u.b0 + i] - off0) + ub[i];
   __syncthreads();
   const int32_t *Sb = A.Sb + u.p0, *Sw = A.Sw + u.p0;
   int32_t *pbr = pb + off0, *pwr = pw + off0;
@@ -1310,6 +1313,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     if (nbig > 0 && dense) b2 += ws_bytes((size_t)nbig * n_c, 8);
     if (nbig > 0 && !dense) {
       b2 += 2 * ws_bytes(nbkt + 1, 4) + 2 * ws_bytes(nbkt + 1, 8) + ws_bytes(nbkt + 1, 4);
+      b2 += ws_bytes((size_t)nunits * kPartHist + 1, 4);  // ubase
       b2 += 4 * ws_bytes((size_t)big_vol + 1, 4) + scan_ws_bytes(nbkt);
       b2 += ws_bytes(nbkt + 1, 8) + ws_bytes(2 * nbkt + 2, 4);
       b2 += ws_bytes(nbkt + 1, 4);  // bin_row
@@ -1407,7 +1411,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.dense = dn_arr;
   } else if (nbig > 0) {
     unsigned *bkt_cnt = arena_take<unsigned>(W2, nbkt + 1);
-    unsigned *bkt_cur = arena_take<unsigned>(W2, nbkt + 1);
+    int32_t *ubase = arena_take<int32_t>(W2, (size_t)nunits * kPartHist + 1);  // unit offsets inside bins
     int64_t *bkt_off = arena_take<int64_t>(W2, nbkt + 1);
     int64_t *fb_off = arena_take<int64_t>(W2, nbkt + 1);
     int32_t *fb_cnt = arena_take<int32_t>(W2, nbkt + 1);
@@ -1419,17 +1423,16 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     int32_t *fb_w = arena_take<int32_t>(W2, (size_t)big_vol + 1);
     if (!fb_w) { set_error("workspace under-reserved (buckets)"); return HEC_EINVAL; }
     HEC_CUDA_TRY(cudaMemsetAsync(bkt_cnt, 0, sizeof(unsigned) * (nbkt + 1), s));
-    HEC_CUDA_TRY(cudaMemsetAsync(bkt_cur, 0, sizeof(unsigned) * (nbkt + 1), s));
     int64_t *prow = arena_take<int64_t>(W2, nbig + 1);
     if (!prow) { set_error("workspace under-reserved (prow)"); return HEC_EINVAL; }
     HEC_TRY(chained_scan(ctx, nbig, RowUIn{L, big_list}, PtrOut{prow}, stb, prow + nbig));
     PartArgs PA{L, big_list, nbig, unit_ptr, unit_row, bkt_ptr, sc_col, sc_wgt};
     if (nunits > 0) {  // rows above kWarpRowMax: CTA units count, per-row scan, scatter
-      k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt);
+      k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
       HEC_LAUNCH_CHECK();
       k_row_bins<<<nblk(nbig * 32, 256), 256, 0, s>>>(PA, prow, bkt_cnt, bkt_off);
       HEC_LAUNCH_CHECK();
-      k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, bkt_cur, pb, pw);
+      k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, ubase, pb, pw);
       HEC_LAUNCH_CHECK();
     }
     k_part_warp<<<nblk(nbig * 32, kPWT), kPWT, 0, s>>>(PA, prow, bkt_off, bkt_cnt, pb, pw);
