@@ -116,13 +116,14 @@ def level_bytes(levels, g0_n, g0_nnz):
     return tot
 
 
-def traffic_from_profiles(kernel_phase):
-    """ncu dram bytes per launch of the dominant kernel, if a capture was committed."""
+def traffic_from_profiles(config, kernel_phase):
+    """ncu dram bytes per step of the dominant phase for this workload, if a
+    capture was committed (profiles/ncu_traffic.json, keyed by config)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
         return None
-    d = json.load(open(p))
-    return d.get(kernel_phase)
+    d = json.load(open(p)).get(f"C{config}")
+    return d.get(kernel_phase) if d else None
 
 
 def run_oracle_sample(reps):
@@ -255,7 +256,7 @@ def main():
     dom = max(prof.items(), key=lambda kv: kv[1]["ms"])
     dom_name, d = dom
     achieved = d["bytes"] / (d["ms"] / 1e3) / 1e9 if d["ms"] > 0 else 0.0
-    traffic = traffic_from_profiles(dom_name)
+    traffic = traffic_from_profiles(args.config, dom_name)
     B = level_bytes(levels, g.n, g.nnz)
     phases = {k: {"ms_per_step": v["ms"] / args.steps, "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] else 0,
                   "share": v["ms"] / (ms * args.steps)} for k, v in sorted(prof.items(), key=lambda kv: -kv[1]["ms"])}

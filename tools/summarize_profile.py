@@ -85,8 +85,14 @@ def main():
         lines.append(f"{k:12s} {t / 1e6:9.3f} ms {100 * t / tot:5.1f}%  DRAM {b / 1e9:8.3f} GB")
         traffic[k] = b
     open(os.path.join(PROF, f"{tag}_launches.txt"), "w").write("\n".join(lines) + "\n")
-    json.dump({"tag": tag, "source": f"profiles/{tag}_launches.csv", "unit": "bytes per step",
-               **traffic}, open(os.path.join(PROF, "ncu_traffic.json"), "w"), indent=1)
+    # per workload (tag r1_c4_... -> "C4"): bench.py reads the entry of its own config
+    cfg = next(("C" + p[1:] for p in tag.split("_") if p[:1] == "c" and p[1:].isdigit()), tag)
+    tp = os.path.join(PROF, "ncu_traffic.json")
+    allt = json.load(open(tp)) if os.path.exists(tp) else {}
+    if "tag" in allt:  # old single-workload layout
+        allt = {}
+    allt[cfg] = {"tag": tag, "source": f"profiles/{tag}_launches.csv", "unit": "bytes per step", **traffic}
+    json.dump(allt, open(tp, "w"), indent=1)
     print("\n".join(lines))
     if len(sys.argv) > 3:
         rep = sys.argv[3]
