@@ -927,7 +927,8 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
                         const int32_t *__restrict__ fb_cnt, int32_t *__restrict__ blk_cnt,
                         int64_t *__restrict__ grp_end,
                         WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, RbmItem *__restrict__ list_r,
-                        RbmItem *__restrict__ list_r2, unsigned *__restrict__ list_n, bool rbm,
+                        RbmItem *__restrict__ list_r2, RbmItem *__restrict__ list_d, unsigned *__restrict__ list_n,
+                        bool rbm, bool direct,
                         const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
   const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   int tier = -1;  // 0 warp, 1 CTA, 2 bitmap-rank CTA
@@ -966,6 +967,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
       }
       // size class (k_tiers lists: list_r front/back, list_r2 front/back)
       tier = ri.n <= kHrMax0 ? 2 : ri.n <= kHrMax1 ? 3 : ri.n <= kHrMax2 ? 4 : 5;
+      if (direct && ri.bk >= 0 && ri.hi - ri.lo <= kDirectR) tier = 6;  // direct-indexed bin
     } else if (d.kind != B_BUCKET) tier = 1;
     else {
       const int64_t h = big_idx[d.row0];
@@ -986,12 +988,13 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
   }
   const int lane = threadIdx.x & 31;
   // list_n: [0] warp [1] CTA [2] list_r front [4] list_r back [5] list_r2 front [6] list_r2 back
+  //         [8] list_d
 #pragma unroll
-  for (int q = 0; q < 6; ++q) {
+  for (int q = 0; q < 7; ++q) {
     const unsigned m = __ballot_sync(0xffffffffu, tier == q);
     if (!m) continue;
     const int leader = __ffs(m) - 1;
-    const int slot = q < 3 ? q : q + 1;
+    const int slot = q < 3 ? q : q < 6 ? q + 1 : 8;
     unsigned base = 0;
     if (lane == leader) base = atomicAdd(list_n + slot, (unsigned)__popc(m));
     base = __shfl_sync(0xffffffffu, base, leader);
@@ -1001,6 +1004,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
       else if (q == 3) list_r[nblocks - pos] = ri;  // lists hold nblocks + 1 items
       else if (q == 4) list_r2[pos] = ri;
       else if (q == 5) list_r2[nblocks - pos] = ri;
+      else if (q == 6) list_d[pos] = ri;
       else if (q) list_c[pos] = (int32_t)bi;
       else list_w[pos] = it;
     }
@@ -1305,7 +1309,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
-                3 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
+                4 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
@@ -1332,6 +1336,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   RbmItem *list_r = arena_take<RbmItem>(W2, nblocks + 1);     // rank items n <= 2048 (front / back)
   RbmItem *list_r2 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n > 2048 (front / back)
   RbmItem *list_redo = arena_take<RbmItem>(W2, nblocks + 1);  // n > 4096 items left to k_rbm
+  RbmItem *list_d = arena_take<RbmItem>(W2, nblocks + 1);     // direct-indexed bins (k_drank)
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1476,7 +1481,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, list_r, list_r2, counts + 10, rbm, vw64, err);
+                                              list_c, list_r, list_r2, list_d, counts + 10, rbm,
+                                              getenv("HEC_NO_DRANK") == nullptr, vw64, err);
     HEC_LAUNCH_CHECK();
   }
 
@@ -1535,6 +1541,10 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
         HEC_TRY(launch_rbm(ctx, A));
       }
     }
+    A.ritems = list_d;
+    A.nlist = counts + 18;
+    A.rdir = 1;
+    HEC_TRY(launch_drank(ctx, A));
     A.ticket = counts + 1;
   }
   phase_end(ctx, ph_rows);

@@ -306,6 +306,101 @@ int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *n
   return HEC_OK;
 }
 
+// Bins whose key range is at most kDirectR keys (bins of the largest skewed
+// rows): the range itself is the table.  Every entry adds its weight at
+// b - lo (one shared-memory atomic, no probing); a scan over the range's
+// non-zero counters then gives every distinct key its rank, and each thread
+// writes its slice of keys in order -- already sorted, no hashing, no ranking
+// pass.  Items of any length (rounds of NT*8 entries, no barrier between rounds).
+constexpr int kDrT = 256;
+static_assert(kDirectR == kDrT * 16, "16 counters per thread");
+__global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
+  __shared__ uint32_t val[kDirectR];
+  __shared__ int32_t wsum[kDrT / 32];
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  const int64_t nitems = *A.nlist;
+  int32_t *const pbg = A.pb_g, *const pwg = A.pw_g;
+  for (int i = t; i < kDirectR; i += kDrT) val[i] = 0u;
+  __syncthreads();
+  for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
+    const RbmItem it = rbm_at(A.ritems, A.rdir, A.rcap, ii);
+    const int32_t a = it.row, lo = it.lo;
+    int32_t *const src_b = pbg + it.src;  // bins only (it.bk >= 0)
+    int32_t *const src_w = pwg + it.src;
+    bool wrap = false;
+    for (int64_t r0 = 0; r0 < it.n; r0 += 8 * kDrT) {
+      int32_t kb[8], kw[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int64_t i = r0 + t + kDrT * k;
+        kb[k] = -1;
+        kw[k] = 0;
+        if (i < it.n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        if (kb[k] < 0 || kb[k] == a) continue;  // self entry (L280)
+        const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
+        wrap |= o + (uint32_t)kw[k] < o;
+      }
+    }
+    if (wrap) atomicOr(A.err, ERR_OVERFLOW);
+    __syncthreads();
+    // thread t owns counters [16 t, 16 t + 16): count, block scan, write in order
+    uint32_t v[16];
+    int c = 0;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      v[q] = val[16 * t + q];
+      c += v[q] != 0u;
+    }
+    int x = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[wid] = x;
+    __syncthreads();
+    int before = 0, D = 0;
+#pragma unroll
+    for (int w = 0; w < kDrT / 32; ++w) {
+      const int sw = wsum[w];
+      before += w < wid ? sw : 0;
+      D += sw;
+    }
+    int pos = before + x - c;
+    bool over = false;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      if (v[q] != 0u) {
+        over |= v[q] > 0x7fffffffu;
+        src_b[pos] = lo + 16 * t + q;
+        src_w[pos] = (int32_t)v[q];
+        ++pos;
+        val[16 * t + q] = 0u;
+      }
+    }
+    if (over) atomicOr(A.err, ERR_OVERFLOW);
+    if (t == 0) A.blk_cnt[it.bi] = D;
+    __syncthreads();
+  }
+}
+
+int launch_drank(hec_ctx *ctx, const RowsArgs &A) {
+  static int occ = 0;
+  if (!occ) {
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank, kDrT, 0));
+    if (occ < 1) occ = 1;
+  }
+  int64_t grid = (int64_t)ctx->num_sms * occ;
+  if (A.nblocks < grid) grid = A.nblocks;
+  if (grid < 1) return HEC_OK;
+  k_drank<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
 template <int NT>
 static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
   static bool attr = false;

@@ -293,6 +293,32 @@ def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
+@pytest.mark.parametrize("path", ["direct", "hash"])
+def test_construct_direct_bins(P, ctx, path, monkeypatch):
+    """A hub row of 100k entries whose keys fall in [1, 3001): its key-range
+    bins are narrow (<= 4096 keys) and hold ~25k entries each, so they take the
+    direct-indexed counters (k_drank, several rounds per bin); path=hash forces
+    the hash-rank kernels (HEC_NO_DRANK test hook)."""
+    if path == "hash":
+        monkeypatch.setenv("HEC_NO_DRANK", "1")
+    rng = np.random.default_rng(24)
+    n, nc = 150000, 40000
+    edges = {(0, v): 1 + v % 5 for v in range(1, 100001)}
+    for _ in range(2 * n):
+        u, v = rng.integers(1, n, 2)
+        if u != v:
+            edges[(min(u, v), max(u, v))] = int(rng.integers(1, 9))
+    g = gg.from_edges(n, [(u, v, w) for (u, v), w in edges.items()])
+    M = np.empty(n, np.int32)
+    M[0] = 0
+    M[1:100001] = 1 + np.arange(1, 100001) % 3000
+    rest = np.arange(100001, n)
+    M[rest] = rng.integers(3001, nc, rest.size)
+    M[rest[:nc - 3001]] = np.arange(3001, nc)
+    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+    assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
+
+
 def test_construct_rbm_rank_windows(P, ctx):
     """Bitmap-rank bins with more distinct keys than one rank window (kRbmCap =
     4096): a skewed row whose neighbours map densely into the low key range, so
