@@ -154,6 +154,9 @@ constexpr int kUnit = 65536;     // member-edge positions per partition CTA
 __host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c, bool rbm = false) {
   const int64_t avg = rbm ? kRbmBinAvg : kBucketAvg;
   int64_t nb = (U + avg - 1) / avg;
+  // rows holding >= 1/16 of the key range in entries: bins no wider than
+  // kDirectR keys (>= 256 entries each on average) for the direct-indexed kernel
+  if (rbm && U >= n_c / 16 && nb < (n_c + kDirectR - 1) / kDirectR) nb = (n_c + kDirectR - 1) / kDirectR;
   if (nb > kPartHist) nb = kPartHist;
   if (nb > n_c) nb = n_c;
   return nb < 1 ? 1 : nb;
@@ -1274,7 +1277,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const bool fused_dense = dense && getenv("HEC_DENSE_STAGED") == nullptr;
   // bitmap-rank items replace the bin pieces when the key range fits the
   // shared-memory bitmap (HEC_NO_RBM: test / tuning hook for the bin-piece path)
-  const bool rbm = !dense && n_c <= kRbmRange && getenv("HEC_NO_RBM") == nullptr;
+  const bool rbm = n_c <= kRbmRange && getenv("HEC_NO_RBM") == nullptr;  // DENSE levels too (small rows)
   const int64_t big_thr = rbm ? (int64_t)kRbmRow : big_threshold_host(dense);
   k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_thr, big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));

@@ -228,9 +228,7 @@ def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     (DENSE when nc <= 32768, key-range buckets otherwise), many labels give
     warp-piece and CTA-window rows.  path=bins forces the key-range bin pieces
     instead of the bitmap-rank items (HEC_NO_RBM test hook)."""
-    if path == "bins":
-        if nc <= 32768:
-            pytest.skip("DENSE mode: no bitmap-rank items")
+    if path == "bins":  # DENSE levels: small rows through the k_rows blocks instead of rank items
         monkeypatch.setenv("HEC_NO_RBM", "1")
     if path == "staged":  # DENSE rows through the staging (v1) instead of the fused expansion
         if nc > 32768:
