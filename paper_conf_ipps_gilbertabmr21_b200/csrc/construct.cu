@@ -193,8 +193,10 @@ __global__ void k_block_desc(Layout L, const int64_t *__restrict__ blk_ptr, cons
   int64_t b0 = blk_ptr[a], b1 = blk_ptr[a + 1];
   if (b1 == b0) return;
   if (big_idx[a] >= 0) {
-    if (dense)
-      for (int64_t k = b0; k < b1; ++k) blk[k] = BlockDesc{B_DENSE, (int32_t)a, (int32_t)a + 1, (int32_t)(k - b0)};
+    // BUCKET bins are (re)written by k_bucket_blocks after the partition; their
+    // kind is set here already so that work split by kind before then is exact
+    const int32_t kind = dense ? B_DENSE : B_BUCKET;
+    for (int64_t k = b0; k < b1; ++k) blk[k] = BlockDesc{kind, (int32_t)a, (int32_t)a + 1, (int32_t)(k - b0)};
   } else {
     const int64_t U = L.U(a);
     if (U <= kPieceMax) blk[b0] = BlockDesc{B_PIECE, (int32_t)a, -1, 0};
@@ -931,13 +933,15 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
                         int64_t *__restrict__ grp_end,
                         WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, RbmItem *__restrict__ list_r,
                         RbmItem *__restrict__ list_r2, RbmItem *__restrict__ list_d, unsigned *__restrict__ list_n,
-                        bool rbm, bool direct,
+                        bool rbm, bool direct, int mode,
                         const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
   const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   int tier = -1;  // 0 warp, 1 CTA, 2 bitmap-rank CTA
   WorkItem it{0, (int32_t)bi, 0, 0, 0};
   RbmItem ri{};
-  if (bi < nblocks) {
+  // mode 0: every block; 1: all but key-range bins; 2: bins only (split launch)
+  const bool take = bi < nblocks && (mode == 0 || ((blk[bi].kind == B_BUCKET) == (mode == 2)));
+  if (take) {
     const BlockDesc d = blk[bi];
     it.row0 = d.row0;
     // vertex weight of a skewed row (written by k_place): int32 bound
@@ -1312,7 +1316,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
-                4 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
+                6 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
@@ -1396,8 +1400,73 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     attr = true;
   }
 
+  // ---- overlap: whole rows (pieces, rank items) on the aux stream while the
+  // skewed rows are partitioned on the main stream; they share no data but
+  // the staging, which both only read (rank items rewrite their own rows)
+  const bool direct = getenv("HEC_NO_DRANK") == nullptr;
+  // (opt-in, HEC_OVERLAP=1: measured 4 % slower on C4 -- the partition and the
+  // rank kernels compete for shared memory and both are latency-bound)
+  const bool overlap = rbm && !dense && nbig > 0 && nblocks > 0 && getenv("HEC_OVERLAP") != nullptr;
+  RbmItem *list_rb = nullptr, *list_rb2 = nullptr;  // bins' rank items (overlap mode)
+  // an error return between fork and join must not leave aux work touching the workspace
+  struct AuxGuard {
+    hec_ctx *c = nullptr;
+    ~AuxGuard() {
+      if (c) cudaStreamSynchronize(c->aux);
+    }
+  } aux_guard;
+  int ph_rows = -1;
+  if (overlap) {
+    list_rb = arena_take<RbmItem>(W2, nblocks + 1);
+    list_rb2 = arena_take<RbmItem>(W2, nblocks + 1);
+    if (!list_rb2) { set_error("workspace under-reserved (bin lists)"); return HEC_EINVAL; }
+    if (!ctx->aux) {
+      HEC_CUDA_TRY(cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking));
+      HEC_CUDA_TRY(cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming));
+      HEC_CUDA_TRY(cudaEventCreateWithFlags(&ctx->ev_join, cudaEventDisableTiming));
+    }
+    HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
+    HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
+    A.row_ptr_c = out->row_ptr;
+    A.vwgt_c = out->vwgt;
+    // one phase for the overlapped partition + dedup (their times cannot be split)
+    ph_rows = phase_begin(ctx, "rows", 8.0 * (double)(small_vol + big_vol) + 8.0 * (double)big_vol);
+    k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
+    HEC_LAUNCH_CHECK();
+    HEC_CUDA_TRY(cudaEventRecord(ctx->ev_fork, s));
+    HEC_CUDA_TRY(cudaStreamWaitEvent(ctx->aux, ctx->ev_fork, 0));
+    aux_guard.c = ctx;
+    cudaStream_t main_s = ctx->stream;
+    ctx->stream = ctx->aux;
+    int rc = HEC_OK;
+    k_tiers<<<nblk(nblocks, 256), 256, 0, ctx->aux>>>(L, nblocks, blk, big_idx, bkt_ptr, nullptr, nullptr, nullptr, blk_cnt,
+                                                     grp_end, list_w, list_c, list_r, list_r2, list_d, counts + 10, rbm,
+                                                     direct, 1, vw64, err);
+    ctx->launches++;
+    if (cudaGetLastError() != cudaSuccess) rc = HEC_ECUDA;
+    RowsArgs B = A;
+    B.items = list_w;
+    B.nlist = counts + 10;
+    if (rc == HEC_OK) rc = launch_pieces(ctx, B, counts + 5);
+    B.rcap = nblocks + 1;
+    const struct { RbmItem *items; unsigned *n; int dir; } wcls[3] = {
+        {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}};
+    for (int c = 0; c < 3 && rc == HEC_OK; ++c) {
+      B.ritems = wcls[c].items;
+      B.nlist = wcls[c].n;
+      B.rdir = wcls[c].dir;
+      rc = launch_hrank(ctx, B, c);
+    }
+    if (rc == HEC_OK && cudaEventRecord(ctx->ev_join, ctx->aux) != cudaSuccess) rc = HEC_ECUDA;
+    ctx->stream = main_s;
+    if (rc != HEC_OK) {
+      cudaStreamSynchronize(ctx->aux);
+      return rc;
+    }
+  }
+
   // ---- a9 skewed rows
-  const int ph_skew = phase_begin(ctx, "rows_skew", 8.0 * (double)big_vol);
+  const int ph_skew = overlap ? -1 : phase_begin(ctx, "rows_skew", 8.0 * (double)big_vol);
   int32_t *unit_row = nullptr;
   if (nbig > 0) {
     unit_row = arena_take<int32_t>(W2, nunits + 1);
@@ -1477,21 +1546,26 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.fb_b_w = fb_b;
     A.fb_w_w = fb_w;
   }
-  phase_end(ctx, ph_skew);
+  if (ph_skew >= 0) phase_end(ctx, ph_skew);
   // counts: [5] pieces ticket [8] wide list [10] warp list [11] CTA list [12] bitmap-rank list
   //         [13] bitmap-rank ticket
-  if (nblocks > 0) {
+  if (nblocks > 0 && !overlap) {
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, list_r, list_r2, list_d, counts + 10, rbm,
-                                              getenv("HEC_NO_DRANK") == nullptr, vw64, err);
+                                              list_c, list_r, list_r2, list_d, counts + 10, rbm, direct, 0, vw64, err);
+    HEC_LAUNCH_CHECK();
+  } else if (nblocks > 0) {  // the whole rows are already in flight on the aux stream: bins now
+    k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
+                                              list_c, list_rb, list_rb2, list_d, counts + 20, rbm, direct, 2, vw64, err);
     HEC_LAUNCH_CHECK();
   }
 
   // ---- work blocks (a8/a9 output), then placement (a10)
-  HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
-  HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
+  if (!overlap) {
+    HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
+    HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
+  }
   out->n_c = n_out;
   A.row_ptr_c = out->row_ptr;
   A.vwgt_c = out->vwgt;
@@ -1500,7 +1574,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_TRY(dev_alloc(ctx, (void **)&trace, sizeof(long long) * 4 * (nblocks + 1)));
     A.trace = trace;
   }
-  const int ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
+  if (!overlap) ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
   A.items = list_w;
   A.nlist = counts + 10;
   unsigned long long *pstats = nullptr;
@@ -1509,7 +1583,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_CUDA_TRY(cudaMemsetAsync(pstats, 0, 16 * sizeof(unsigned long long), s));
     A.pstats = pstats;
   }
-  HEC_TRY(launch_pieces(ctx, A, counts + 5));
+  if (!overlap) HEC_TRY(launch_pieces(ctx, A, counts + 5));
   if (pstats) {
     unsigned long long h[16];
     HEC_CUDA_TRY(cudaMemcpyAsync(h, pstats, sizeof h, cudaMemcpyDeviceToHost, s));
@@ -1520,19 +1594,26 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     dev_free(ctx, pstats);
     A.pstats = nullptr;
   }
-  A.list = list_c;
-  A.nlist = counts + 11;
-  HEC_TRY(launch_rows(ctx, A, false));
+  if (!overlap) {
+    A.list = list_c;
+    A.nlist = counts + 11;
+    HEC_TRY(launch_rows(ctx, A, false));
+  }
   if (rbm) {
     A.ticket = counts + 13;
     A.rcap = nblocks + 1;
     // hash-rank size classes, then the bitmap-rank items above kHrMax2 entries
-    const struct { RbmItem *items; unsigned *n; int dir; } cls[4] = {
+    // (overlap mode: classes 0-2 of the whole rows ran on the aux stream; here the bins)
+    struct RankList { RbmItem *items; unsigned *n; int dir; };
+    const RankList cls[4] = {
         {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}, {list_r2, counts + 16, -1}};
+    const RankList bcls[4] = {
+        {list_rb, counts + 22, 1}, {list_rb, counts + 24, -1}, {list_rb2, counts + 25, 1}, {list_rb2, counts + 26, -1}};
     for (int c = 0; c < 4; ++c) {
-      A.ritems = cls[c].items;
-      A.nlist = cls[c].n;
-      A.rdir = cls[c].dir;
+      const RankList &C = overlap ? bcls[c] : cls[c];
+      A.ritems = C.items;
+      A.nlist = C.n;
+      A.rdir = C.dir;
       if (c < 3) HEC_TRY(launch_hrank(ctx, A, c));
       else if (getenv("HEC_NO_HRANK_BIG")) HEC_TRY(launch_rbm(ctx, A));
       else {
@@ -1545,10 +1626,17 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
       }
     }
     A.ritems = list_d;
-    A.nlist = counts + 18;
+    A.nlist = overlap ? counts + 28 : counts + 18;
     A.rdir = 1;
     HEC_TRY(launch_drank(ctx, A));
     A.ticket = counts + 1;
+  }
+  if (overlap) {  // join the whole rows; CTA-tier blocks (if any) after both
+    HEC_CUDA_TRY(cudaStreamWaitEvent(s, ctx->ev_join, 0));
+    aux_guard.c = nullptr;  // main is ordered after the aux work from here on
+    A.list = list_c;
+    A.nlist = counts + 11;
+    HEC_TRY(launch_rows(ctx, A, false));
   }
   phase_end(ctx, ph_rows);
   if (trace) {
@@ -1598,7 +1686,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   phase_end(ctx, ph_place);
   // rows phase: staged / partitioned entries read (8 B each; DENSE rows were
   // accumulated in rows_skew), distinct entries staged (8 B), row_ptr_c + vwgt_c
-  phase_set_bytes(ctx, ph_rows, 8.0 * (double)(small_vol + (dense ? 0 : big_vol)) + 8.0 * (double)nnz_c + 12.0 * dnc);
+  // (overlap mode: the partition's pair writes are in this phase too)
+  phase_set_bytes(ctx, ph_rows, 8.0 * (double)(small_vol + (dense ? 0 : big_vol)) + 8.0 * (double)nnz_c + 12.0 * dnc +
+                                    (overlap ? 8.0 * (double)big_vol : 0.0));
   if (nblocks == 0) HEC_CUDA_TRY(cudaMemsetAsync(out->row_ptr, 0, sizeof(int64_t) * (n_out + 1), s));
   ctx->stats.nnz_c = out->nnz_c;
   return HEC_OK;

@@ -291,7 +291,7 @@ def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["direct", "hash"])
+@pytest.mark.parametrize("path", ["direct", "hash", "overlap"])
 def test_construct_direct_bins(P, ctx, path, monkeypatch):
     """A hub row of 100k entries whose keys fall in [1, 3001): its key-range
     bins are narrow (<= 4096 keys) and hold ~25k entries each, so they take the
@@ -299,6 +299,8 @@ def test_construct_direct_bins(P, ctx, path, monkeypatch):
     the hash-rank kernels (HEC_NO_DRANK test hook)."""
     if path == "hash":
         monkeypatch.setenv("HEC_NO_DRANK", "1")
+    if path == "overlap":  # whole rows on the second stream during the partition (HEC_OVERLAP)
+        monkeypatch.setenv("HEC_OVERLAP", "1")
     rng = np.random.default_rng(24)
     n, nc = 150000, 40000
     edges = {(0, v): 1 + v % 5 for v in range(1, 100001)}
