@@ -149,7 +149,7 @@ __global__ void k_big_rows(Layout L, int64_t big_thr, int32_t *__restrict__ big_
 }
 
 constexpr int kPartHist = 8192;  // buckets per skewed row (bounds the partition's smem tables)
-constexpr int kUnit = 65536;     // member-edge positions per partition CTA
+constexpr int kUnit = 32768;     // member-edge positions per partition CTA
 
 __host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c, bool rbm = false) {
   const int64_t avg = rbm ? kRbmBinAvg : kBucketAvg;
