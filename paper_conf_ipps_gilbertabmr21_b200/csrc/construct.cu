@@ -407,7 +407,7 @@ constexpr int kXBig = 64;
 // source entry in col/wgt, p: position).  With skip != nullptr, members whose
 // coarse row has skip[M[member]] >= 0 are passed over (DENSE rows, expanded by
 // their accumulation kernel instead).
-template <int kLong, typename Sink>
+template <int kLong, typename Sink, int kShort = 4>
 __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restrict__ mstart, int64_t m_lo,
                                         int64_t m_hi, int64_t P, int64_t Pend, const int32_t *__restrict__ skip,
                                         Sink &sink) {
@@ -438,11 +438,11 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
     }
     const int excl = incl - ds;
     const int T = __shfl_sync(0xffffffffu, incl, 31);
-    for (int base = 0; base < T; base += 128) {
-      int64_t e[4], p[4];
+    for (int base = 0; base < T; base += 32 * kShort) {
+      int64_t e[kShort], p[kShort];
       unsigned ok = 0;
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < kShort; ++u) {
         const int t = base + lane + 32 * u;
         int lo = 0;  // largest lane with excl <= t
 #pragma unroll
@@ -508,6 +508,7 @@ struct StageSink {
 };
 
 // skip: big_idx in DENSE mode (those rows are expanded by k_dense_accum2), else nullptr
+constexpr int kXPer = 4;  // positions per lane in flight (8: spills at 3 CTAs/SM, no gain)
 __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
                                                int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
                                                const int32_t *__restrict__ skip) {
@@ -518,7 +519,7 @@ __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__rest
   StageSink sink{L, Sb, Sw, P_lo};
   for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
     const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
-    x2_walk<4>(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
+    x2_walk<kXPer, StageSink, kXPer>(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
   }
 }
 
@@ -932,7 +933,8 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
                         const int32_t *__restrict__ fb_cnt, int32_t *__restrict__ blk_cnt,
                         int64_t *__restrict__ grp_end,
                         WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, RbmItem *__restrict__ list_r,
-                        RbmItem *__restrict__ list_r2, RbmItem *__restrict__ list_d, unsigned *__restrict__ list_n,
+                        RbmItem *__restrict__ list_r2, RbmItem *__restrict__ list_d, RbmItem *__restrict__ list_r3,
+                        unsigned *__restrict__ list_n,
                         bool rbm, bool direct, int mode,
                         const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
   const int64_t bi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -973,7 +975,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
         ri.bk = (int32_t)bk;
       }
       // size class (k_tiers lists: list_r front/back, list_r2 front/back)
-      tier = ri.n <= kHrMax0 ? 2 : ri.n <= kHrMax1 ? 3 : ri.n <= kHrMax2 ? 4 : 5;
+      tier = ri.n <= kHrMaxS ? 7 : ri.n <= kHrMax0 ? 2 : ri.n <= kHrMax1 ? 3 : ri.n <= kHrMax2 ? 4 : 5;
       if (direct && ri.bk >= 0 && ri.hi - ri.lo <= kDirectR) tier = 6;  // direct-indexed bin
     } else if (d.kind != B_BUCKET) tier = 1;
     else {
@@ -995,13 +997,13 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
   }
   const int lane = threadIdx.x & 31;
   // list_n: [0] warp [1] CTA [2] list_r front [4] list_r back [5] list_r2 front [6] list_r2 back
-  //         [8] list_d
+  //         [8] list_d [3] list_r3 (n <= kHrMaxS)
 #pragma unroll
-  for (int q = 0; q < 7; ++q) {
+  for (int q = 0; q < 8; ++q) {
     const unsigned m = __ballot_sync(0xffffffffu, tier == q);
     if (!m) continue;
     const int leader = __ffs(m) - 1;
-    const int slot = q < 3 ? q : q < 6 ? q + 1 : 8;
+    const int slot = q < 3 ? q : q < 6 ? q + 1 : q == 6 ? 8 : 3;
     unsigned base = 0;
     if (lane == leader) base = atomicAdd(list_n + slot, (unsigned)__popc(m));
     base = __shfl_sync(0xffffffffu, base, leader);
@@ -1012,6 +1014,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
       else if (q == 4) list_r2[pos] = ri;
       else if (q == 5) list_r2[nblocks - pos] = ri;
       else if (q == 6) list_d[pos] = ri;
+      else if (q == 7) list_r3[pos] = ri;
       else if (q) list_c[pos] = (int32_t)bi;
       else list_w[pos] = it;
     }
@@ -1316,7 +1319,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
-                6 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
+                8 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
@@ -1344,6 +1347,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   RbmItem *list_r2 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n > 2048 (front / back)
   RbmItem *list_redo = arena_take<RbmItem>(W2, nblocks + 1);  // n > 4096 items left to k_rbm
   RbmItem *list_d = arena_take<RbmItem>(W2, nblocks + 1);     // direct-indexed bins (k_drank)
+  RbmItem *list_r3 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n <= kHrMaxS
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1407,7 +1411,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // (opt-in, HEC_OVERLAP=1: measured 4 % slower on C4 -- the partition and the
   // rank kernels compete for shared memory and both are latency-bound)
   const bool overlap = rbm && !dense && nbig > 0 && nblocks > 0 && getenv("HEC_OVERLAP") != nullptr;
-  RbmItem *list_rb = nullptr, *list_rb2 = nullptr;  // bins' rank items (overlap mode)
+  RbmItem *list_rb = nullptr, *list_rb2 = nullptr, *list_rb3 = nullptr;  // bins' rank items (overlap mode)
   // an error return between fork and join must not leave aux work touching the workspace
   struct AuxGuard {
     hec_ctx *c = nullptr;
@@ -1419,7 +1423,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (overlap) {
     list_rb = arena_take<RbmItem>(W2, nblocks + 1);
     list_rb2 = arena_take<RbmItem>(W2, nblocks + 1);
-    if (!list_rb2) { set_error("workspace under-reserved (bin lists)"); return HEC_EINVAL; }
+    list_rb3 = arena_take<RbmItem>(W2, nblocks + 1);
+    if (!list_rb3) { set_error("workspace under-reserved (bin lists)"); return HEC_EINVAL; }
     if (!ctx->aux) {
       HEC_CUDA_TRY(cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking));
       HEC_CUDA_TRY(cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming));
@@ -1440,8 +1445,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     ctx->stream = ctx->aux;
     int rc = HEC_OK;
     k_tiers<<<nblk(nblocks, 256), 256, 0, ctx->aux>>>(L, nblocks, blk, big_idx, bkt_ptr, nullptr, nullptr, nullptr, blk_cnt,
-                                                     grp_end, list_w, list_c, list_r, list_r2, list_d, counts + 10, rbm,
-                                                     direct, 1, vw64, err);
+                                                     grp_end, list_w, list_c, list_r, list_r2, list_d, list_r3, counts + 10,
+                                                     rbm, direct, 1, vw64, err);
     ctx->launches++;
     if (cudaGetLastError() != cudaSuccess) rc = HEC_ECUDA;
     RowsArgs B = A;
@@ -1449,13 +1454,13 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     B.nlist = counts + 10;
     if (rc == HEC_OK) rc = launch_pieces(ctx, B, counts + 5);
     B.rcap = nblocks + 1;
-    const struct { RbmItem *items; unsigned *n; int dir; } wcls[3] = {
-        {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}};
-    for (int c = 0; c < 3 && rc == HEC_OK; ++c) {
+    const struct { RbmItem *items; unsigned *n; int dir; } wcls[4] = {
+        {list_r3, counts + 13, 1}, {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}};
+    for (int c = 0; c < 4 && rc == HEC_OK; ++c) {
       B.ritems = wcls[c].items;
       B.nlist = wcls[c].n;
       B.rdir = wcls[c].dir;
-      rc = launch_hrank(ctx, B, c);
+      rc = launch_hrank(ctx, B, c - 1);
     }
     if (rc == HEC_OK && cudaEventRecord(ctx->ev_join, ctx->aux) != cudaSuccess) rc = HEC_ECUDA;
     ctx->stream = main_s;
@@ -1553,11 +1558,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, list_r, list_r2, list_d, counts + 10, rbm, direct, 0, vw64, err);
+                                              list_c, list_r, list_r2, list_d, list_r3, counts + 10, rbm, direct, 0, vw64, err);
     HEC_LAUNCH_CHECK();
   } else if (nblocks > 0) {  // the whole rows are already in flight on the aux stream: bins now
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, list_rb, list_rb2, list_d, counts + 20, rbm, direct, 2, vw64, err);
+                                              list_c, list_rb, list_rb2, list_d, list_rb3, counts + 20, rbm, direct, 2, vw64, err);
     HEC_LAUNCH_CHECK();
   }
 
@@ -1600,17 +1605,17 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     HEC_TRY(launch_rows(ctx, A, false));
   }
   if (rbm) {
-    A.ticket = counts + 13;
+    A.ticket = counts + 30;  // (unused by the rank kernels)
     A.rcap = nblocks + 1;
     // hash-rank size classes, then the bitmap-rank items above kHrMax2 entries
     // (overlap mode: classes 0-2 of the whole rows ran on the aux stream; here the bins)
     struct RankList { RbmItem *items; unsigned *n; int dir; };
-    const RankList cls[4] = {
+    const RankList cls[5] = {{list_r3, counts + 13, 1},
         {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}, {list_r2, counts + 16, -1}};
-    const RankList bcls[4] = {
+    const RankList bcls[5] = {{list_rb3, counts + 23, 1},
         {list_rb, counts + 22, 1}, {list_rb, counts + 24, -1}, {list_rb2, counts + 25, 1}, {list_rb2, counts + 26, -1}};
-    for (int c = 0; c < 4; ++c) {
-      const RankList &C = overlap ? bcls[c] : cls[c];
+    for (int c = -1; c < 4; ++c) {
+      const RankList &C = overlap ? bcls[c + 1] : cls[c + 1];
       A.ritems = C.items;
       A.nlist = C.n;
       A.rdir = C.dir;

@@ -420,11 +420,13 @@ static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
   return HEC_OK;
 }
 
-// One size class of items (the list in A.ritems / A.nlist): cls 0, 1, 2 =
-// n <= 1024, 2048, 4096 on 128-, 256-, 512-thread CTAs.
+// One size class of items (the list in A.ritems / A.nlist): cls -1, 0, 1, 2 =
+// n <= 512, 1024, 2048, 4096 on 64-, 128-, 256-, 512-thread CTAs.
 int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls) {
-  static_assert(HrSmem<128>::kCapE == kHrMax0 && HrSmem<256>::kCapE == kHrMax1 && HrSmem<512>::kCapE == kHrMax2,
+  static_assert(HrSmem<64>::kCapE == kHrMaxS && HrSmem<128>::kCapE == kHrMax0 && HrSmem<256>::kCapE == kHrMax1 &&
+                    HrSmem<512>::kCapE == kHrMax2,
                 "size classes");
+  if (cls < 0) return launch_hrank_t<64>(ctx, A);  // two warps per item: barriers among 64 threads
   if (cls == 0) return launch_hrank_t<128>(ctx, A);
   if (cls == 1) return launch_hrank_t<256>(ctx, A);
   return launch_hrank_t<512>(ctx, A);
