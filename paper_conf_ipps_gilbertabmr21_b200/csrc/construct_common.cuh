@@ -29,7 +29,7 @@ constexpr int32_t kEmpty = -1;
 // partitioned into bins of ~kRbmBinAvg entries, each bin an item.
 constexpr int64_t kRbmRange = 917504;  // keys covered by the shared-memory bitmap
 constexpr int kRbmRow = 4096;
-constexpr int kRbmBinAvg = 2048;
+constexpr int kRbmBinAvg = 1024;
 constexpr int kRbmCap = 4096;          // distinct keys per rank window
 
 enum : int32_t { B_SMALL = 0, B_BUCKET = 1, B_DENSE = 2, B_PIECE = 3, B_RBM = 4 };
