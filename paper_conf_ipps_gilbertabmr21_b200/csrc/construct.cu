@@ -407,7 +407,7 @@ constexpr int kXBig = 64;
 // source entry in col/wgt, p: position).  With skip != nullptr, members whose
 // coarse row has skip[M[member]] >= 0 are passed over (DENSE rows, expanded by
 // their accumulation kernel instead).
-template <int kLong, typename Sink, int kShort = 4>
+template <int kLong, typename Sink, int kShort = 4, typename IdxT = int64_t>
 __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restrict__ mstart, int64_t m_lo,
                                         int64_t m_hi, int64_t P, int64_t Pend, const int32_t *__restrict__ skip,
                                         Sink &sink) {
@@ -439,7 +439,7 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
     const int excl = incl - ds;
     const int T = __shfl_sync(0xffffffffu, incl, 31);
     for (int base = 0; base < T; base += 32 * kShort) {
-      int64_t e[kShort], p[kShort];
+      IdxT e[kShort], p[kShort];
       unsigned ok = 0;
 #pragma unroll
       for (int u = 0; u < kShort; ++u) {
@@ -454,8 +454,8 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
         const int64_t ors = __shfl_sync(0xffffffffu, rs, lo);
         const int64_t ops = __shfl_sync(0xffffffffu, ps, lo);
         const int oex = __shfl_sync(0xffffffffu, excl, lo);
-        e[u] = ors + (t - oex);
-        p[u] = ops + (t - oex);
+        e[u] = (IdxT)(ors + (t - oex));
+        p[u] = (IdxT)(ops + (t - oex));
         if (t < T) ok |= 1u << u;
       }
       sink(e, p, ok);
@@ -469,13 +469,13 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
       const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
       const int64_t bps = __shfl_sync(0xffffffffu, ps, src);
       for (int base = 0; base < bd; base += 32 * kLong) {  // kLong positions per lane in flight
-        int64_t e[kLong], p[kLong];
+        IdxT e[kLong], p[kLong];
         unsigned ok = 0;
 #pragma unroll
         for (int u = 0; u < kLong; ++u) {
           const int t = base + lane + 32 * u;
-          e[u] = brs + t;
-          p[u] = bps + t;
+          e[u] = (IdxT)(brs + t);
+          p[u] = (IdxT)(bps + t);
           if (t < bd) ok |= 1u << u;
         }
         sink(e, p, ok);
@@ -492,8 +492,8 @@ struct StageSink {
   const Layout &L;
   int32_t *__restrict__ Sb, *__restrict__ Sw;
   int64_t P_lo;
-  template <int N>
-  __device__ __forceinline__ void operator()(const int64_t (&e)[N], const int64_t (&p)[N], unsigned ok) {
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
     int32_t b[N], w[N];
 #pragma unroll
     for (int u = 0; u < N; ++u)
@@ -503,12 +503,12 @@ struct StageSink {
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
 #pragma unroll
     for (int u = 0; u < N; ++u)
-      if (ok & (1u << u)) { __stcs(Sb + (p[u] - P_lo), b[u]); __stcs(Sw + (p[u] - P_lo), w[u]); }
+      if (ok & (1u << u)) { __stcs(Sb + ((int64_t)p[u] - P_lo), b[u]); __stcs(Sw + ((int64_t)p[u] - P_lo), w[u]); }
   }
 };
 
 // skip: big_idx in DENSE mode (those rows are expanded by k_dense_accum2), else nullptr
-constexpr int kXPer = 4;  // positions per lane in flight (8: spills at 3 CTAs/SM, no gain)
+template <typename IdxT, int kPer>
 __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
                                                int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
                                                const int32_t *__restrict__ skip) {
@@ -519,7 +519,7 @@ __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__rest
   StageSink sink{L, Sb, Sw, P_lo};
   for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
     const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
-    x2_walk<kXPer, StageSink, kXPer>(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
+    x2_walk<kPer, StageSink, kPer, IdxT>(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
   }
 }
 
@@ -576,7 +576,7 @@ __device__ __forceinline__ int part_bucket(const UnitInfo &u, int32_t b) {
   return k < u.nb - 1 ? k : u.nb - 1;
 }
 
-constexpr int kPartU = 8;  // loads in flight per thread in the partition passes
+constexpr int kPartU = 16;  // loads in flight per thread in the partition passes
 
 // Bucket of the entry, or -1 for a self entry (dropped, L280) / past the unit.
 __device__ __forceinline__ int entry_bucket(const UnitInfo &u, int32_t b) {
@@ -1133,8 +1133,8 @@ struct AccSink {
   uint32_t *acc;
   int32_t a;
   bool wrap;
-  template <int N>
-  __device__ __forceinline__ void operator()(const int64_t (&e)[N], const int64_t (&p)[N], unsigned ok) {
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
     (void)p;
     int32_t b[N], w[N];
 #pragma unroll
@@ -1364,7 +1364,10 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     if (grid > cap) grid = cap;
     if (grid > 0) {
       if (getenv("HEC_EXPAND_V1")) k_expand<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
-      else k_expand2<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, fused_dense ? big_idx : nullptr);
+      else if (g->nnz < ((int64_t)1 << 32) && getenv("HEC_EXPAND_W64") == nullptr)  // 32-bit entry / position indices
+        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, fused_dense ? big_idx : nullptr);
+      else
+        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, fused_dense ? big_idx : nullptr);
       HEC_LAUNCH_CHECK();
     }
     phase_end(ctx, phx);
