@@ -157,6 +157,8 @@ __host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c, 
   // rows holding >= 1/16 of the key range in entries: bins no wider than
   // kDirectR keys (>= 256 entries each on average) for the direct-indexed kernel
   if (rbm && U >= n_c / 16 && nb < (n_c + kDirectR - 1) / kDirectR) nb = (n_c + kDirectR - 1) / kDirectR;
+  // k_rbm (items with too many distinct keys) needs bins no wider than kRbmRange keys
+  if (rbm && nb < (n_c + kRbmRange - 1) / kRbmRange) nb = (n_c + kRbmRange - 1) / kRbmRange;
   if (nb > kPartHist) nb = kPartHist;
   if (nb > n_c) nb = n_c;
   return nb < 1 ? 1 : nb;
@@ -1284,7 +1286,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const bool fused_dense = dense && getenv("HEC_DENSE_STAGED") == nullptr;
   // bitmap-rank items replace the bin pieces when the key range fits the
   // shared-memory bitmap (HEC_NO_RBM: test / tuning hook for the bin-piece path)
-  const bool rbm = n_c <= kRbmRange && getenv("HEC_NO_RBM") == nullptr;  // DENSE levels too (small rows)
+  // rank items for every level (DENSE levels: the small rows); bins are kept
+  // <= kRbmRange keys wide (row_buckets) for the bitmap-rank fallback
+  const bool rbm = getenv("HEC_NO_RBM") == nullptr;
   const int64_t big_thr = rbm ? (int64_t)kRbmRow : big_threshold_host(dense);
   k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_thr, big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));
