@@ -291,8 +291,9 @@ def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["direct", "hash", "overlap"])
-def test_construct_direct_bins(P, ctx, path, monkeypatch):
+@pytest.mark.parametrize("hot", [False, True])
+@pytest.mark.parametrize("path", ["direct", "direct_noagg", "hash", "overlap"])
+def test_construct_direct_bins(P, ctx, path, hot, monkeypatch):
     """A hub row of 100k entries whose keys fall in [1, 3001): its key-range
     bins are narrow (<= 4096 keys) and hold ~25k entries each, so they take the
     direct-indexed counters (k_drank, several rounds per bin); path=hash forces
@@ -301,9 +302,14 @@ def test_construct_direct_bins(P, ctx, path, monkeypatch):
         monkeypatch.setenv("HEC_NO_DRANK", "1")
     if path == "overlap":  # whole rows on the second stream during the partition (HEC_OVERLAP)
         monkeypatch.setenv("HEC_OVERLAP", "1")
+    if path == "direct_noagg":  # plain shared-memory atomics (no warp match + reduce)
+        monkeypatch.setenv("HEC_DRANK_AGG", "0")
     rng = np.random.default_rng(24)
     n, nc = 150000, 40000
-    edges = {(0, v): 1 + v % 5 for v in range(1, 100001)}
+    # hot: the hub's 100k entries fall on 30 keys (whole warps of equal keys)
+    # with weights > 2^16 (both 16-bit halves of the warp sums)
+    nk, w0 = (30, 70000) if hot else (3000, 1)
+    edges = {(0, v): w0 + v % 5 for v in range(1, 100001)}
     for _ in range(2 * n):
         u, v = rng.integers(1, n, 2)
         if u != v:
@@ -311,10 +317,10 @@ def test_construct_direct_bins(P, ctx, path, monkeypatch):
     g = gg.from_edges(n, [(u, v, w) for (u, v), w in edges.items()])
     M = np.empty(n, np.int32)
     M[0] = 0
-    M[1:100001] = 1 + np.arange(1, 100001) % 3000
+    M[1:100001] = 1 + np.arange(1, 100001) % nk
     rest = np.arange(100001, n)
-    M[rest] = rng.integers(3001, nc, rest.size)
-    M[rest[:nc - 3001]] = np.arange(3001, nc)
+    M[rest] = rng.integers(nk + 1, nc, rest.size)
+    M[rest[:nc - nk - 1]] = np.arange(nk + 1, nc)
     cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
@@ -463,9 +469,15 @@ def digest_levels(Hg):
     return out
 
 
-@pytest.mark.parametrize("cfg", [2, 3, 4])
+@pytest.mark.parametrize("cfg", [2, 3, 4, 5])
 def test_hierarchy_full_size_digests(P, ctx, golden_dir, cfg):
-    d = json.load(open(os.path.join(golden_dir, "oracle_digests.json")))[str(cfg)]
+    """Whole hierarchy at BASELINE.json's full sizes (C5 = R-MAT s26 ef16, the
+    one-GPU launch configuration bench.py --config 5 times) against the oracle's
+    per-level digests (tests/golden/make_digests.py, oracle/ only)."""
+    dd = json.load(open(os.path.join(golden_dir, "oracle_digests.json")))
+    if str(cfg) not in dd:
+        pytest.skip(f"no oracle digest for C{cfg} (python tests/golden/make_digests.py {cfg})")
+    d = dd[str(cfg)]
     g = gg.config(cfg)
     assert gg.sha16(g.row_ptr, g.col) == d["sha_G0"]
     Hg = P.coarsen_hierarchy(ctx, dev(P, g), d["cutoff"], d["seed"])
