@@ -17,8 +17,6 @@
 //   3. writes (b, sum) at its rank, in place over the item's own input range.
 // Work is O(n) per item with six CTA barriers; several CTAs per SM overlap
 // them.  Items with n > NT*8 entries are left to k_rbm.
-#include <cstdlib>
-
 #include "construct_common.cuh"
 
 namespace hec {
@@ -314,12 +312,8 @@ int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *n
 // non-zero counters then gives every distinct key its rank, and each thread
 // writes its slice of keys in order -- already sorted, no hashing, no ranking
 // pass.  Items of any length (rounds of NT*8 entries, no barrier between rounds).
-// AGG: entries of a warp with equal keys are first combined (match + reduce)
-// so that one lane adds their sum -- hub keys of duplicate-heavy levels
-// otherwise serialise the shared-memory atomics of a warp.
 constexpr int kDrT = 256;
 static_assert(kDirectR == kDrT * 16, "16 counters per thread");
-template <bool AGG>
 __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
   __shared__ uint32_t val[kDirectR];
   __shared__ int32_t wsum[kDrT / 32];
@@ -345,24 +339,9 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
       }
 #pragma unroll
       for (int k = 0; k < 8; ++k) {
-        const bool ok = kb[k] >= 0 && kb[k] != a;  // self entry (L280)
-        if (AGG) {
-          const unsigned act = __ballot_sync(0xffffffffu, ok);  // every round is warp-uniform
-          if (!ok) continue;
-          const unsigned peers = __match_any_sync(act, kb[k]);
-          // 16-bit halves: the group sum is exact in 64 bits (overflow check)
-          const uint32_t s_lo = __reduce_add_sync(peers, (uint32_t)kw[k] & 0xffffu);
-          const uint32_t s_hi = __reduce_add_sync(peers, (uint32_t)kw[k] >> 16);
-          if (lane != __ffs(peers) - 1) continue;
-          const uint64_t tot = ((uint64_t)s_hi << 16) + s_lo;
-          wrap |= tot > 0xffffffffull;
-          const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)tot);
-          wrap |= o + (uint32_t)tot < o;
-        } else {
-          if (!ok) continue;
-          const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
-          wrap |= o + (uint32_t)kw[k] < o;
-        }
+        if (kb[k] < 0 || kb[k] == a) continue;  // self entry (L280)
+        const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
+        wrap |= o + (uint32_t)kw[k] < o;
       }
     }
     if (wrap) atomicOr(A.err, ERR_OVERFLOW);
@@ -412,19 +391,14 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
 
 int launch_drank(hec_ctx *ctx, const RowsArgs &A) {
   static int occ = 0;
-  const char *e = getenv("HEC_DRANK_AGG");  // tuning / test hook: 0 = plain atomics
-  const bool agg = e == nullptr || e[0] != '0';
   if (!occ) {
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank<true>, kDrT, 0));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank, kDrT, 0));
     if (occ < 1) occ = 1;
   }
   int64_t grid = (int64_t)ctx->num_sms * occ;
   if (A.nblocks < grid) grid = A.nblocks;
   if (grid < 1) return HEC_OK;
-  if (agg)
-    k_drank<true><<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A);
-  else
-    k_drank<false><<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A);
+  k_drank<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }

@@ -292,7 +292,7 @@ def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
 
 
 @pytest.mark.parametrize("hot", [False, True])
-@pytest.mark.parametrize("path", ["direct", "direct_noagg", "hash", "overlap"])
+@pytest.mark.parametrize("path", ["direct", "hash", "overlap"])
 def test_construct_direct_bins(P, ctx, path, hot, monkeypatch):
     """A hub row of 100k entries whose keys fall in [1, 3001): its key-range
     bins are narrow (<= 4096 keys) and hold ~25k entries each, so they take the
@@ -302,12 +302,10 @@ def test_construct_direct_bins(P, ctx, path, hot, monkeypatch):
         monkeypatch.setenv("HEC_NO_DRANK", "1")
     if path == "overlap":  # whole rows on the second stream during the partition (HEC_OVERLAP)
         monkeypatch.setenv("HEC_OVERLAP", "1")
-    if path == "direct_noagg":  # plain shared-memory atomics (no warp match + reduce)
-        monkeypatch.setenv("HEC_DRANK_AGG", "0")
     rng = np.random.default_rng(24)
     n, nc = 150000, 40000
-    # hot: the hub's 100k entries fall on 30 keys (whole warps of equal keys)
-    # with weights > 2^16 (both 16-bit halves of the warp sums)
+    # hot: the hub's 100k entries fall on 30 keys (whole warps of equal keys,
+    # sums of ~2.3e8 per key)
     nk, w0 = (30, 70000) if hot else (3000, 1)
     edges = {(0, v): w0 + v % 5 for v in range(1, 100001)}
     for _ in range(2 * n):
