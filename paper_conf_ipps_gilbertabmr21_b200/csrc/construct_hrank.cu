@@ -347,13 +347,11 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
     if (wrap) atomicOr(A.err, ERR_OVERFLOW);
     __syncthreads();
     // thread t owns counters [16 t, 16 t + 16): count, block scan, write in order
-    // only the item's key range [lo, hi) holds counts
-    const int range = it.hi - lo;
     uint32_t v[16];
     int c = 0;
 #pragma unroll
     for (int q = 0; q < 16; ++q) {
-      v[q] = 16 * t + q < range ? val[16 * t + q] : 0u;
+      v[q] = val[16 * t + q];
       c += v[q] != 0u;
     }
     int x = c;
