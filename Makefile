@@ -10,6 +10,7 @@ ARCH    := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
            --expt-relaxed-constexpr -Iinclude
 CU_SRC  := $(wildcard $(PKG)/csrc/*.cu)
+CU_OBJ  := $(patsubst $(PKG)/csrc/%.cu,build/%.o,$(CU_SRC))
 CU_HDR  := $(wildcard $(PKG)/csrc/*.cuh) include/hec.h
 
 all: graphgen oracle hec
@@ -23,10 +24,14 @@ oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
 	$(CC) -O2 -std=c11 -Wall -Wextra -fPIC -shared -o $@ oracle/oracle.c
 
 hec: $(PKG)/libhec.so
-$(PKG)/libhec.so: $(CU_SRC) $(CU_HDR) Makefile
-	$(NVCC) $(NVFLAGS) -Xptxas -v -shared -o $@ $(CU_SRC) -lcudart 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
+build/%.o: $(PKG)/csrc/%.cu $(CU_HDR) Makefile
+	@mkdir -p build
+	$(NVCC) $(NVFLAGS) -Xptxas -v -c -o $@ $< 2> build/$*.ptxas.log || (cat build/$*.ptxas.log; exit 1)
+$(PKG)/libhec.so: $(CU_OBJ)
+	$(NVCC) $(ARCH) -shared -o $@ $(CU_OBJ) -lcudart
+	@cat build/*.ptxas.log > $(PKG)/ptxas.log
 
 clean:
-	rm -f graphgen/libgraphgen.so oracle/liboracle.so $(PKG)/libhec.so
+	rm -rf build graphgen/libgraphgen.so oracle/liboracle.so $(PKG)/libhec.so
 
 .PHONY: all graphgen oracle hec clean

@@ -11,8 +11,9 @@ workload's G0, which is resident in HBM when the timed region starts.
   e2e     same metric through the C-ABI call with host buffers: pinned-host ->
           device copy of G0 and a device -> host read of the coarsest graph and
           the level sizes inside the timed region
-  roofline  dominant phase: algorithmic bytes / CUDA-event device time, vs the
-          measured HBM copy bandwidth in MEASURED_PEAKS.json
+  roofline  the dominant part (mapping or construction of one level): SURVEY
+          §8(d) compulsory bytes / its CUDA-event device time, vs the measured HBM
+          copy bandwidth in MEASURED_PEAKS.json; `levels` gives B_l / T_l per level
   cpu_baseline  the CPU oracle (single thread) on a bounded sample
 
 usage: python bench.py [--gpus N] [--steps K] [--warmup W] [--config 4] [--impl ours|reference]
@@ -106,6 +107,10 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(rows)}
 
 
+MAPPING_PHASES = ("heavy", "rounds", "relabel")
+CONSTRUCTION_PHASES = ("bucket", "expand", "rows_skew", "rows", "place")
+
+
 def level_bytes(levels, g0_n, g0_nnz):
     """B_l = 16 nnz + 8 nnz_c + 28 n + 12 n_c per built level."""
     tot = 0.0
@@ -116,14 +121,42 @@ def level_bytes(levels, g0_n, g0_nnz):
     return tot
 
 
-def traffic_from_profiles(config, kernel_phase):
-    """ncu dram bytes per step of the dominant phase for this workload, if a
-    capture was committed (profiles/ncu_traffic.json, keyed by config)."""
+def mapping_bytes(n, nnz):
+    """a1-a5 compulsory bytes: col + wgt once, row_ptr, M written."""
+    return 8.0 * nnz + 12.0 * n
+
+
+def construction_bytes(n, nnz, nc, nnzc):
+    """a7-a10 compulsory bytes: col + wgt once, col_c + wgt_c once,
+    row_ptr, M, vwgt in; row_ptr_c, vwgt_c out."""
+    return 8.0 * nnz + 8.0 * nnzc + 16.0 * n + 12.0 * nc
+
+
+def source_stamp():
+    """sha256[:16] over the CUDA sources: ties a committed ncu capture to the code it measured."""
+    import glob
+    import hashlib
+    h = hashlib.sha256()
+    for f in sorted(glob.glob(os.path.join(ROOT, "paper_conf_ipps_gilbertabmr21_b200", "csrc", "*.cu*"))):
+        h.update(open(f, "rb").read())
+    return h.hexdigest()[:16]
+
+
+def traffic_from_profiles(config, level, part):
+    """ncu dram bytes (read + write) of one hierarchy's `part` ("mapping" /
+    "construction") at `level`, from the committed capture of this workload
+    (profiles/ncu_traffic.json, written by tools/ncu_traffic.py).  A capture
+    of other CUDA sources is stale and ignored (returns None)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
-        return None
+        return None, None
     d = json.load(open(p)).get(f"C{config}")
-    return d.get(kernel_phase) if d else None
+    if not d or d.get("source_stamp") != source_stamp():
+        return None, (d or {}).get("source_stamp")
+    lv = d.get("levels", [])
+    if level >= len(lv):
+        return None, d.get("source_stamp")
+    return lv[level].get(f"{part}_dram"), d.get("source_stamp")
 
 
 def run_oracle_sample(reps):
@@ -182,6 +215,21 @@ def main():
     rank, local_rank, world = env_rank()
     if args.impl == "reference":
         return reference_arm(args, rank, world)
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # one process per GPU: re-exec under torchrun (the driver's launch form)
+        import torch
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            print(json.dumps({"error": f"--gpus {args.gpus} requested but only {have} CUDA device(s) visible"}),
+                  flush=True)
+            return 2
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(29500 + os.getpid() % 1000),
+               os.path.abspath(__file__)] + sys.argv[1:]
+        return subprocess.call(cmd)
+    if world != args.gpus:
+        print(json.dumps({"error": f"--gpus {args.gpus} but WORLD_SIZE={world}"}), flush=True)
+        return 2
 
     import numpy as np
     import torch
@@ -242,6 +290,7 @@ def main():
     barrier()
     ms = ev0.elapsed_time(ev1) / args.steps
     prof = ctx.profile()
+    prof_lv = ctx.profile(by_level=True)
     launches = ctx.launches()
     ctx.set_profiling(False)
     if dist:
@@ -251,15 +300,35 @@ def main():
     # strong scaling: one graph per job, every level partitioned over the ranks
     value = m0 / (ms / 1e3)
 
-    # ---- roofline of the dominant phase
+    # ---- per-level records and the roofline (SURVEY §8(d) compulsory bytes)
     peak, peak_src = peaks()
-    dom = max(prof.items(), key=lambda kv: kv[1]["ms"])
-    dom_name, d = dom
-    achieved = d["bytes"] / (d["ms"] / 1e3) / 1e9 if d["ms"] > 0 else 0.0
-    traffic = traffic_from_profiles(args.config, dom_name)
     B = level_bytes(levels, g.n, g.nnz)
+    per_level = []
+    parts = []  # (ms per step, level, part, algorithmic bytes)
+    n_l, nnz_l = g.n, g.nnz
+    n_levels = max([lv for (_, lv) in prof_lv] + [-1]) + 1
+    for l in range(n_levels):
+        built = l < len(levels)
+        nc, nnzc = levels[l] if built else (None, None)
+        t_l = prof_lv.get(("level", l), {}).get("ms", 0.0) / args.steps
+        t_map = sum(prof_lv.get((k, l), {}).get("ms", 0.0) for k in MAPPING_PHASES) / args.steps
+        t_con = sum(prof_lv.get((k, l), {}).get("ms", 0.0) for k in CONSTRUCTION_PHASES) / args.steps
+        b_l = (16 * nnz_l + 8 * nnzc + 28 * n_l + 12 * nc) if built else mapping_bytes(n_l, nnz_l)
+        rec = {"level": l, "n": n_l, "nnz": nnz_l, "n_c": nc, "nnz_c": nnzc, "built": built,
+               "ms": t_l, "B": b_l, "GBps": b_l / (t_l / 1e3) / 1e9 if t_l else None,
+               "frac": (b_l / (t_l / 1e3) / 1e9 / peak) if t_l else None,
+               "mapping_ms": t_map, "construction_ms": t_con if built else 0.0}
+        per_level.append(rec)
+        parts.append((t_map, l, "mapping", mapping_bytes(n_l, nnz_l)))
+        if built:
+            parts.append((t_con, l, "construction", construction_bytes(n_l, nnz_l, nc, nnzc)))
+            n_l, nnz_l = nc, nnzc
+    t_dom, l_dom, part_dom, b_dom = max(parts) if parts else (0.0, 0, "mapping", 0.0)
+    achieved = b_dom / (t_dom / 1e3) / 1e9 if t_dom > 0 else 0.0
+    traffic, stamp = traffic_from_profiles(args.config, l_dom, part_dom)
     phases = {k: {"ms_per_step": v["ms"] / args.steps, "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] else 0,
-                  "share": v["ms"] / (ms * args.steps)} for k, v in sorted(prof.items(), key=lambda kv: -kv[1]["ms"])}
+                  "share": v["ms"] / (ms * args.steps)}
+              for k, v in sorted(prof.items(), key=lambda kv: -kv[1]["ms"]) if k != "level"}
 
     # ---- e2e through host buffers
     e2e = None
@@ -331,8 +400,15 @@ def main():
             "time_to_cutoff_ms": ms,
             "hierarchy_GBps": B / (ms / 1e3) / 1e9,
             "hierarchy_frac_of_peak": B / (ms / 1e3) / 1e9 / peak,
-            "roofline": {"bound": "hbm", "kernel": dom_name, "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src},
+            "roofline": {"bound": "hbm", "kernel": f"{part_dom} of level {l_dom}", "achieved": achieved,
+                         "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                         "algorithmic_bytes": b_dom, "ms": t_dom,
+                         "bytes_rule": ("SURVEY 8(d): mapping 8 nnz + 12 n; construction 8 nnz + 8 nnz_c + "
+                                        "16 n + 12 n_c"),
+                         "traffic_source": (f"profiles/ncu_traffic.json (source stamp {stamp})" if traffic
+                                            else f"no ncu capture of these sources ({source_stamp()})"),
+                         "peak_source": peak_src},
+            "levels": per_level,
             "phases": phases,
             "cpu_baseline": cpu,
             "e2e": e2e,

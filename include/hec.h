@@ -171,12 +171,18 @@ HEC_API void hec_hierarchy_free(hec_hierarchy *h);
  * summed device time, number of calls and the algorithmic bytes (compulsory
  * traffic: each input read once, each output written once).
  * Phases: "heavy" (a1), "rounds" (a3), "relabel" (a4+a5), "bucket" (a7),
- * "rows_small", "rows_mid" (a8), "rows_skew" (a9), "place" (a10). */
+ * "expand", "rows_skew", "rows" (a8/a9), "place" (a10), and inside
+ * coarsen_hierarchy one "level" phase per level l spanning its mapping and
+ * construction, with SURVEY §8(d)'s compulsory bytes
+ *   B_l = 16 nnz + 8 nnz_c + 28 n + 12 n_c   (built level)
+ *   B_l = 8 nnz + 12 n                       (discarded level: mapping only).
+ * Entries are accumulated per (phase, level). */
 typedef struct {
   char name[24];
   double ms;         /* summed device time */
   int64_t calls;
   double bytes;      /* summed algorithmic bytes */
+  int32_t level;     /* coarsen_hierarchy level index l (fine graph G_l), -1 outside a hierarchy */
 } hec_phase_time;
 HEC_API int hec_ctx_set_profiling(hec_ctx *ctx, int on);
 /* Clears the accumulated phase times and the launch counter. */

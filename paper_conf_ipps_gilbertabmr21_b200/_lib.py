@@ -38,7 +38,7 @@ class HecStats(ctypes.Structure):
 
 class HecPhaseTime(ctypes.Structure):
     _fields_ = [("name", ctypes.c_char * 24), ("ms", ctypes.c_double), ("calls", ctypes.c_int64),
-                ("bytes", ctypes.c_double)]
+                ("bytes", ctypes.c_double), ("level", ctypes.c_int32)]
 
 
 ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)

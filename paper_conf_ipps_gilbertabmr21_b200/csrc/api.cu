@@ -83,7 +83,7 @@ static cudaEvent_t take_event(hec_ctx *ctx) {
 
 int phase_begin(hec_ctx *ctx, const char *name, double bytes) {
   if (!ctx->prof_on) return -1;
-  hec_ctx::PhaseRec r{name, take_event(ctx), take_event(ctx), bytes};
+  hec_ctx::PhaseRec r{name, take_event(ctx), take_event(ctx), bytes, ctx->prof_level};
   cudaEventRecord(r.a, ctx->stream);
   ctx->prof_pending.push_back(r);
   return (int)ctx->prof_pending.size() - 1;
@@ -106,11 +106,12 @@ static void resolve_profile(hec_ctx *ctx) {
     cudaEventElapsedTime(&ms, r.a, r.b);
     hec_ctx::PhaseAcc *acc = nullptr;
     for (auto &x : ctx->prof_acc)
-      if (x.name == r.name) acc = &x;
+      if (x.name == r.name && x.level == r.level) acc = &x;
     if (!acc) {
       ctx->prof_acc.push_back(hec_ctx::PhaseAcc{});
       acc = &ctx->prof_acc.back();
       acc->name = r.name;
+      acc->level = r.level;
     }
     acc->ms += ms;
     acc->bytes += r.bytes;
@@ -267,6 +268,7 @@ HEC_API int hec_ctx_profile(hec_ctx *ctx, hec_phase_time *out, int max, int *cou
       out[k].ms = x.ms;
       out[k].calls = x.calls;
       out[k].bytes = x.bytes;
+      out[k].level = x.level;
     }
     ++k;
   }
@@ -403,6 +405,10 @@ HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff,
     int32_t *M = nullptr;
     rc = dev_alloc(ctx, (void **)&M, sizeof(int32_t) * cur.n);
     if (rc != HEC_OK) break;
+    // one "level" phase per level: mapping + construction (SURVEY §8(d) B_l);
+    // a discarded level is its mapping only (B = 8 nnz + 12 n)
+    ctx->prof_level = level;
+    const int ph_level = phase_begin(ctx, "level", 8.0 * (double)cur.nnz + 12.0 * (double)cur.n);
     size_t ws = 0;
     ws_bytes_mapping(cur.n, cur.nnz, &ws);
     rc = ws_reserve(ctx, ws);
@@ -413,6 +419,7 @@ HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff,
     if (rc != HEC_OK) { dev_free(ctx, M); break; }
     ctx->stats.rounds = r.rounds;
     ctx->stats.n_c = r.n_c;
+    phase_end(ctx, ph_level);  // (extended below when the level is built)
     if (r.n_c < discard_below) {
       h->stop_reason = HEC_STOP_DISCARD;
       h->discarded_n_c = r.n_c;
@@ -436,6 +443,9 @@ HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff,
       dev_free(ctx, M);
       break;
     }
+    phase_end(ctx, ph_level);
+    phase_set_bytes(ctx, ph_level, 16.0 * (double)cur.nnz + 8.0 * (double)L.g.nnz_c + 28.0 * (double)cur.n +
+                                       12.0 * (double)L.g.n_c);
     h->levels.push_back(L);
     cur.n = L.g.n_c;
     cur.nnz = L.g.nnz_c;
@@ -445,6 +455,7 @@ HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff,
     cur.vwgt = L.g.vwgt;
     ++level;
   }
+  ctx->prof_level = -1;
   if (rc != HEC_OK) {
     hec_hierarchy_free(h);
     return rc;

@@ -98,15 +98,18 @@ struct hec_ctx {
   // profiling (hec_ctx_set_profiling)
   int64_t launches = 0;
   int prof_on = 0;
+  int prof_level = -1;  // hierarchy level of the phases being recorded (-1: single calls)
   struct PhaseRec {
     const char *name;
     cudaEvent_t a, b;
     double bytes;
+    int level;
   };
   std::vector<PhaseRec> prof_pending;
   std::vector<cudaEvent_t> prof_pool;
   struct PhaseAcc {
     std::string name;
+    int level = -1;
     double ms = 0, bytes = 0;
     int64_t calls = 0;
   };

@@ -551,13 +551,20 @@ struct RoundArgs {
   uint8_t *rootflag;
   int32_t *blocked;
   int32_t *wl[2];
-  unsigned *cnt;      // [kMaxTrackedRounds + 2] per-round next-list sizes (zeroed)
+  unsigned *cnt;      // [3] next-list sizes, rotating by round (zeroed)
   int32_t *rounds_out;
   GridBarrier bar;
 };
-constexpr int kMaxTrackedRounds = 4096;
 constexpr int kSoloThreshold = 8192;  // finish small residuals in one CTA
 constexpr int kRoundBlock = 512;
+
+// Round r appends its next worklist to cnt[r % 3] and zeroes cnt[(r + 1) % 3]
+// before its barrier.  That counter was last appended in round r - 2 and read
+// right after barrier r - 2, i.e. by every CTA before it arrived at barrier
+// r - 1; its next appends (round r + 1) follow barrier r, which orders the
+// zeroing store before them.  (A single reused counter reset after the barrier
+// would race with the next round's appends.)
+__device__ __forceinline__ unsigned *round_counter(const RoundArgs &A, int r) { return A.cnt + r % 3; }
 
 // decide(r) for u, then scatter(r+1); returns true if u stays undecided.
 __device__ __forceinline__ bool round_step(const RoundArgs &A, uint32_t u, int r) {
@@ -595,7 +602,8 @@ __global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
   __shared__ unsigned s_len;
   // ---- grid-wide rounds
   while (true) {
-    unsigned *next_cnt = A.cnt + (r < kMaxTrackedRounds ? r : kMaxTrackedRounds);
+    unsigned *next_cnt = round_counter(A, r);
+    if (gtid == 0) *round_counter(A, r + 1) = 0u;
     int32_t *next = A.wl[cur ^ 1];
     int64_t lim = (len + 31) & ~(int64_t)31;
     for (int64_t i = gtid; i < lim; i += gstride) {
@@ -611,10 +619,6 @@ __global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
     if (threadIdx.x == 0) s_len = ld_acquire_u32(next_cnt);
     __syncthreads();
     len = s_len;
-    if (r >= kMaxTrackedRounds - 1) {  // keep per-round counters reusable
-      A.bar.sync(nb);
-      if (gtid == 0) *next_cnt = 0;
-    }
     cur ^= 1;
     ++r;
     if (len == 0) {
@@ -623,10 +627,11 @@ __global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
     }
     if (len <= kSoloThreshold) break;
   }
-  // ---- small residual: CTA 0 alone, block barriers only
+  // ---- small residual: CTA 0 alone, block barriers only (same counter rotation)
   if (blockIdx.x != 0) return;
   while (true) {
-    unsigned *next_cnt = A.cnt + (r < kMaxTrackedRounds ? r : kMaxTrackedRounds);
+    unsigned *next_cnt = round_counter(A, r);
+    if (threadIdx.x == 0) *round_counter(A, r + 1) = 0u;
     int32_t *next = A.wl[cur ^ 1];
     int64_t lim = (len + 31) & ~(int64_t)31;
     for (int64_t i = threadIdx.x; i < lim; i += blockDim.x) {
@@ -643,11 +648,6 @@ __global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
     if (threadIdx.x == 0) s_len = *(volatile unsigned *)next_cnt;
     __syncthreads();
     len = s_len;
-    if (r >= kMaxTrackedRounds - 1) {
-      __syncthreads();
-      if (threadIdx.x == 0) *next_cnt = 0;
-      __syncthreads();
-    }
     cur ^= 1;
     ++r;
     if (len == 0) break;
@@ -671,10 +671,16 @@ struct RootLabelOut {
   }
 };
 
-// M[u] for u in [u0, u1): the label of the first root on u's H-path.
+// M[u] for u in [u0, u1): the label of the first root on u's H-path (Alg 3
+// l.14 inherit, Alg 5 l.17-21 pointer jumping).
+// Active chains strictly decrease in priority, so with R3's hashed priorities
+// they are a few steps long; a walk is cut after kAssignWalk steps and the
+// vertex is left to the pointer-jumping passes below (adversarial explicit
+// priorities, e.g. a path visited in id order: one chain of length n).
+constexpr int kAssignWalk = 64;
 __global__ void k_assign(int64_t u0, int64_t u1, const int32_t *__restrict__ H,
                          const uint8_t *__restrict__ status, const int32_t *__restrict__ lab,
-                         int32_t *__restrict__ M) {
+                         int32_t *__restrict__ M, int32_t *__restrict__ jump, int *__restrict__ long_chain) {
   int64_t u = u0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (u >= u1) return;
   if (status[u] == ROOT) {
@@ -682,8 +688,38 @@ __global__ void k_assign(int64_t u0, int64_t u1, const int32_t *__restrict__ H,
     return;
   }
   int32_t x = H[u];
-  while (status[x] != ROOT) x = H[x];
-  M[u] = lab[x];
+  for (int s = 0; s < kAssignWalk; ++s) {
+    if (status[x] == ROOT) {
+      M[u] = lab[x];
+      return;
+    }
+    x = H[x];
+  }
+  jump[u] = x;  // resumed by k_jump
+  *long_chain = 1;
+}
+
+// Pointer jumping over all vertices: jump[u] = first root on u's H-path for
+// roots' predecessors.  Init: jump[u] = u (root) or H[u]; each pass replaces
+// jump[u] by jump[jump[u]] (concurrent updates only move further along the
+// same path, so every interleaving converges), ceil(log2 n) passes suffice.
+__global__ void k_jump_init(int64_t n, const int32_t *__restrict__ H, const uint8_t *__restrict__ status,
+                            int32_t *__restrict__ jump) {
+  int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u < n) jump[u] = status[u] == ROOT ? (int32_t)u : H[u];
+}
+__global__ void k_jump(int64_t n, const uint8_t *__restrict__ status, int32_t *__restrict__ jump) {
+  int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u >= n) return;
+  const int32_t x = jump[u];
+  if (status[x] != ROOT) jump[u] = jump[x];
+}
+__global__ void k_assign_jumped(int64_t u0, int64_t u1, const uint8_t *__restrict__ status,
+                                const int32_t *__restrict__ jump, const int32_t *__restrict__ lab,
+                                int32_t *__restrict__ M) {
+  int64_t u = u0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u >= u1 || status[u] == ROOT) return;
+  M[u] = lab[jump[u]];
 }
 
 int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes) {
@@ -692,7 +728,7 @@ int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes) {
   b += ws_bytes(n, 1) * 2;      // status, rootflag
   b += ws_bytes(n, 4);          // blocked
   b += 2 * ws_bytes(n, 4);      // worklists
-  b += ws_bytes(kMaxTrackedRounds + 2, 4) + ws_bytes(4, 4) + ws_bytes(4, 8);
+  b += ws_bytes(4, 4) + ws_bytes(4, 4) + ws_bytes(4, 8);
   b += heavy_ws(n, nnz);
   b += scan_ws_bytes(n);
   b += ws_bytes(n, 4);          // labels (partial-range mapping)
@@ -712,9 +748,9 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   int32_t *blocked = ws_take<int32_t>(ctx, n);
   int32_t *wl0 = ws_take<int32_t>(ctx, n);
   int32_t *wl1 = ws_take<int32_t>(ctx, n);
-  unsigned *cnt = ws_take<unsigned>(ctx, kMaxTrackedRounds + 2);
+  unsigned *cnt = ws_take<unsigned>(ctx, 4);
   unsigned *bar = ws_take<unsigned>(ctx, 4);
-  int64_t *scal = ws_take<int64_t>(ctx, 4);  // [0] n_c, [1] rounds (int32 in low word)
+  int64_t *scal = ws_take<int64_t>(ctx, 4);  // [0] n_c, [1] rounds (int32 in low word), [2] long chain
   const bool full = u0 == 0 && u1 == n;
   int32_t *lab = full ? M : ws_take<int32_t>(ctx, n);
   if (!status || !rootflag || !blocked || !wl0 || !wl1 || !cnt || !bar || !scal || !lab) {
@@ -725,7 +761,7 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   int ph = phase_begin(ctx, "rounds", 5.0 * dn);
   HEC_CUDA_TRY(cudaMemsetAsync(rootflag, 0, n, s));
   HEC_CUDA_TRY(cudaMemsetAsync(blocked, 0, sizeof(int32_t) * n, s));
-  HEC_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(unsigned) * (kMaxTrackedRounds + 2), s));
+  HEC_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(unsigned) * 4, s));
   HEC_CUDA_TRY(cudaMemsetAsync(bar, 0, sizeof(unsigned) * 4, s));
   HEC_CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(int64_t) * 4, s));
   k_round_init<<<nblk(n, 256), 256, 0, s>>>(n, H, prio, status, blocked);
@@ -753,13 +789,24 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   ScanTiles st = take_scan_tiles(ctx, n);
   if (!st.desc || !st.ticket) { set_error("workspace under-reserved (scan)"); return HEC_EINVAL; }
   HEC_TRY(chained_scan(ctx, n, RootFlagIn{status}, RootLabelOut{status, lab, root_out}, st, scal));
-  if (u1 > u0) {
-    k_assign<<<nblk(u1 - u0, 256), 256, 0, s>>>(u0, u1, H, status, lab, M);
+  int *long_chain = reinterpret_cast<int *>(scal + 2);
+  if (u1 > u0) {  // wl0 is free after the rounds: jump targets of cut walks
+    k_assign<<<nblk(u1 - u0, 256), 256, 0, s>>>(u0, u1, H, status, lab, M, wl0, long_chain);
+    HEC_LAUNCH_CHECK();
+  }
+  int64_t h[3];
+  HEC_TRY(read_scalars(ctx, scal, 3, h));
+  if ((int32_t)(h[2] & 0xffffffff)) {  // some H-chain is longer than kAssignWalk
+    k_jump_init<<<nblk(n, 256), 256, 0, s>>>(n, H, status, wl0);
+    HEC_LAUNCH_CHECK();
+    for (int64_t reach = 1; reach < n; reach *= 2) {
+      k_jump<<<nblk(n, 256), 256, 0, s>>>(n, status, wl0);
+      HEC_LAUNCH_CHECK();
+    }
+    k_assign_jumped<<<nblk(u1 - u0, 256), 256, 0, s>>>(u0, u1, status, wl0, lab, M);
     HEC_LAUNCH_CHECK();
   }
   phase_end(ctx, ph);
-  int64_t h[2];
-  HEC_TRY(read_scalars(ctx, scal, 2, h));
   res->n_c = h[0];
   res->rounds = (int)(int32_t)(h[1] & 0xffffffff);
   return HEC_OK;

@@ -116,14 +116,22 @@ class Context:
     def profile_reset(self):
         check(load().hec_ctx_profile_reset(self.h), "hec_ctx_profile_reset")
 
-    def profile(self) -> dict:
-        """{phase: {"ms": summed device ms, "calls": n, "bytes": algorithmic bytes}}"""
+    def profile(self, by_level: bool = False) -> dict:
+        """{phase: {"ms": summed device ms, "calls": n, "bytes": algorithmic bytes}}
+        (summed over levels), or with by_level {(phase, level): {...}}."""
         L = load()
-        arr = (_lib.HecPhaseTime * 32)()
+        cap = 512
+        arr = (_lib.HecPhaseTime * cap)()
         cnt = ctypes.c_int()
-        check(L.hec_ctx_profile(self.h, arr, 32, ctypes.byref(cnt)), "hec_ctx_profile")
-        return {arr[i].name.decode(): {"ms": arr[i].ms, "calls": arr[i].calls, "bytes": arr[i].bytes}
-                for i in range(min(cnt.value, 32))}
+        check(L.hec_ctx_profile(self.h, arr, cap, ctypes.byref(cnt)), "hec_ctx_profile")
+        out: dict = {}
+        for i in range(min(cnt.value, cap)):
+            key = (arr[i].name.decode(), int(arr[i].level)) if by_level else arr[i].name.decode()
+            d = out.setdefault(key, {"ms": 0.0, "calls": 0, "bytes": 0.0})
+            d["ms"] += arr[i].ms
+            d["calls"] += arr[i].calls
+            d["bytes"] += arr[i].bytes
+        return out
 
     def launches(self) -> int:
         return int(load().hec_ctx_launches(self.h))

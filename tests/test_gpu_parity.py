@@ -188,6 +188,40 @@ def test_mapping_adversarial_path(P, ctx):
         assert nc == nco and np.array_equal(M.cpu().numpy(), Mo)
 
 
+def path_csr(n):
+    """Path 0-1-...-(n-1), unit weights, as a CSR (numpy; from_edges is too slow at 2M)."""
+    deg = np.full(n, 2, np.int64)
+    deg[0] = deg[-1] = 1
+    rp = np.zeros(n + 1, np.int64)
+    rp[1:] = np.cumsum(deg)
+    col = np.empty(rp[-1], np.int32)
+    mid = rp[1:n - 1]                                 # rows 1 .. n-2: (u-1, u+1)
+    col[mid] = np.arange(0, n - 2, dtype=np.int32)
+    col[mid + 1] = np.arange(2, n, dtype=np.int32)
+    col[0] = 1                                        # row 0: (1)
+    col[-1] = n - 2                                   # row n-1: (n-2)
+    return gg.Graph(rp, col, np.ones(rp[-1], np.int32), np.ones(n, np.int32))
+
+
+def test_mapping_long_chain_identity_path(P, ctx):
+    """Identity visit order on a 2M-vertex path: one aggregate (SURVEY §8(c) M1
+    closed form, n_c = 1) reached through a single H-chain of length n -- the
+    inherit step must not walk it per vertex (pointer jumping, Alg 5 l.17-21)."""
+    import time
+    n = 2_000_000
+    g = path_csr(n)
+    assert np.array_equal(o.heavy(g)[:5], [1, 0, 1, 2, 3])
+    pr = np.arange(n, dtype=np.uint64)
+    dg, pt = dev(P, g), prio_tensor(pr)
+    P.hec_find_mapping_prio(ctx, dg, pt)  # warm-up
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    M, nc = P.hec_find_mapping_prio(ctx, dg, pt)
+    dt = time.perf_counter() - t0
+    assert nc == 1 and int(M.max()) == 0 and int(M.min()) == 0
+    assert dt < 1.0, f"{dt:.3f} s"
+
+
 @pytest.mark.parametrize("which", ["c1", "c2", "rmat16", "random"])
 def test_mapping_parity_seeded(P, ctx, which):
     rng = np.random.default_rng(13)

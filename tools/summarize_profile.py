@@ -8,7 +8,8 @@ Writes
                                 cold-cache serialised launches: compare shares)
   profiles/<tag>_launches.csv   the raw launch list
   profiles/<tag>_full.txt       key --set full metrics + warp-stall breakdown
-  profiles/ncu_traffic.json     DRAM bytes per step per bench phase (read by bench.py)
+  profiles/ncu_traffic.json     DRAM bytes per level of mapping / construction, stamped
+                                with the CUDA sources' hash (read by bench.py)
 """
 import collections
 import csv
@@ -21,28 +22,14 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 PROF = os.path.join(ROOT, "profiles")
 
-# libhec kernel -> bench.py phase (hec_ctx_profile names)
-PHASE = {
-    "k_tile_coords": "heavy", "k_heavy": "heavy", "k_heavy_fixup": "heavy", "k_fill_identity": "heavy",
-    "k_round_init": "rounds", "k_rounds": "rounds",
-    "RootFlagIn": "relabel", "k_assign": "relabel",
-    "k_member_count": "bucket", "k_member_fill": "bucket", "k_big_rows": "bucket", "CountIn": "bucket",
-    "DegIn": "bucket", "RowWeightIn": "bucket", "BlockCountIn": "bucket",
-    "UnitsIn": "rows_skew", "BucketsIn": "rows_skew", "k_part_count": "rows_skew", "k_part_write": "rows_skew",
-    "k_fb_jobs": "rows_skew", "k_bucket_fallback": "rows_skew", "k_dense_accum": "rows_skew",
-    "k_block_desc": "rows", "k_block_ends": "rows", "k_rows": "rows", "BlkCntIn": "rows",
-    "k_pieces": "rows", "k_tiers": "rows", "k_wide_list": "rows", "k_expand": "expand",
-    "k_bucket_blocks": "rows_skew",
-    "k_place": "place", "k_hrank": "rows", "k_rbm": "rows", "k_span_coords": "heavy",
-    "k_row_bins": "rows_skew", "k_part_warp": "rows_skew", "k_seg_fill": "rows_skew", "RowUIn": "rows_skew",
-}
+# kernels of the mapping (a1-a5); every other libhec kernel belongs to the construction
+MAPPING = ("k_span_coords", "k_heavy", "k_fill_identity", "k_tile_coords", "k_round_init", "k_rounds",
+           "RootFlagIn", "k_assign", "k_jump")
+LEVEL_START = ("k_span_coords", "k_tile_coords", "k_fill_identity")  # first launch of each level's mapping
 
 
-def phase_of(name):
-    for k, v in PHASE.items():
-        if k in name:
-            return v
-    return "other"
+def part_of(name):
+    return "mapping" if any(k in name for k in MAPPING) else "construction"
 
 
 def launches(path):
@@ -65,11 +52,11 @@ def main():
     per = launches(lc)
     shutil.copy(lc, os.path.join(PROF, f"{tag}_launches.csv"))
     tot = sum(v.get("gpu__time_duration.sum", 0) for v in per.values())
-    kern, ph = collections.OrderedDict(), collections.OrderedDict()
+    kern = collections.OrderedDict()
     for (i, k), v in per.items():
         t = v.get("gpu__time_duration.sum", 0)
         b = v.get("dram__bytes_read.sum", 0) + v.get("dram__bytes_write.sum", 0)
-        for agg, key in ((kern, k), (ph, phase_of(k))):
+        for agg, key in ((kern, k),):
             a = agg.setdefault(key, [0, 0.0, 0.0])
             a[0] += 1
             a[1] += t
@@ -79,19 +66,33 @@ def main():
     for k, (n, t, b) in sorted(kern.items(), key=lambda kv: -kv[1][1]):
         lines.append(f"{k[:58]:58s} n={n:4d} {t / 1e6:9.3f} ms {100 * t / tot:5.1f}%  DRAM {b / 1e9:8.3f} GB "
                      f"{b / max(t, 1):7.1f} GB/s")
-    lines += ["", "## per bench phase"]
-    traffic = {}
-    for k, (n, t, b) in sorted(ph.items(), key=lambda kv: -kv[1][1]):
-        lines.append(f"{k:12s} {t / 1e6:9.3f} ms {100 * t / tot:5.1f}%  DRAM {b / 1e9:8.3f} GB")
-        traffic[k] = b
+    # per level (a level starts at its mapping's first launch): mapping / construction
+    levels = []
+    for (i, k), v in per.items():
+        if any(k.startswith(x) for x in LEVEL_START) or not levels:
+            levels.append({"mapping_ms": 0.0, "mapping_dram": 0.0, "construction_ms": 0.0,
+                           "construction_dram": 0.0, "launches": 0})
+        t = v.get("gpu__time_duration.sum", 0)
+        b = v.get("dram__bytes_read.sum", 0) + v.get("dram__bytes_write.sum", 0)
+        pt = part_of(k)
+        levels[-1][pt + "_ms"] += t / 1e6
+        levels[-1][pt + "_dram"] += b
+        levels[-1]["launches"] += 1
+    lines += ["", "## per level (ncu, cold-cache)"]
+    for l, lv in enumerate(levels):
+        lines.append(f"L{l}: mapping {lv['mapping_ms']:8.3f} ms DRAM {lv['mapping_dram'] / 1e9:7.3f} GB | "
+                     f"construction {lv['construction_ms']:8.3f} ms DRAM {lv['construction_dram'] / 1e9:7.3f} GB "
+                     f"({lv['launches']} launches)")
     open(os.path.join(PROF, f"{tag}_launches.txt"), "w").write("\n".join(lines) + "\n")
-    # per workload (tag r1_c4_... -> "C4"): bench.py reads the entry of its own config
+    # per workload (tag r2_c4_... -> "C4"): bench.py reads the entry of its own config
     cfg = next(("C" + p[1:] for p in tag.split("_") if p[:1] == "c" and p[1:].isdigit()), tag)
     tp = os.path.join(PROF, "ncu_traffic.json")
     allt = json.load(open(tp)) if os.path.exists(tp) else {}
-    if "tag" in allt:  # old single-workload layout
-        allt = {}
-    allt[cfg] = {"tag": tag, "source": f"profiles/{tag}_launches.csv", "unit": "bytes per step", **traffic}
+    allt = {k: v for k, v in allt.items() if isinstance(v, dict) and "levels" in v}
+    sys.path.insert(0, ROOT)
+    from bench import source_stamp
+    allt[cfg] = {"tag": tag, "source": f"profiles/{tag}_launches.csv", "source_stamp": source_stamp(),
+                 "unit": "DRAM bytes (read + write) per hierarchy, ncu cold-cache", "levels": levels}
     json.dump(allt, open(tp, "w"), indent=1)
     print("\n".join(lines))
     if len(sys.argv) > 3:
