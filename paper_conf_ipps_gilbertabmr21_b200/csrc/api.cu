@@ -221,9 +221,6 @@ HEC_API void hec_ctx_destroy(hec_ctx *ctx) {
   dev_free(ctx, ctx->ws2.base);
   cudaStreamSynchronize(ctx->stream);
   if (ctx->h_pinned) cudaFreeHost(ctx->h_pinned);
-  if (ctx->aux) { cudaStreamSynchronize(ctx->aux); cudaStreamDestroy(ctx->aux); }
-  if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
-  if (ctx->ev_join) cudaEventDestroy(ctx->ev_join);
   resolve_profile(ctx);
   for (auto e : ctx->prof_pool) cudaEventDestroy(e);
   delete ctx;

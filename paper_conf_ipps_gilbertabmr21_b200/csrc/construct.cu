@@ -263,232 +263,9 @@ __global__ void k_seg_fill(int64_t nseg, const int64_t *__restrict__ ptr, int32_
 constexpr int kXT = 256;       // threads per CTA
 constexpr int kXChunk = 4096;  // positions per warp task
 
-// Member table [tb, tb + 128) of the warp: member-edge starts (mpre) and source
-// row starts (mstart).  Reloaded only when the walk leaves it, so a window of
-// 128 positions inside a long member row costs no metadata traffic.
-__device__ __forceinline__ void exp_table_load(const Layout &L, const int64_t *__restrict__ mstart, int64_t mend,
-                                               int64_t tb, WarpExpTab &W) {
-  const int lane = threadIdx.x & 31;
-  const int64_t pend_m = L.mpre[mend];
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    const int64_t j = tb + lane + 32 * t;
-    W.mp[lane + 32 * t] = j < mend ? L.mpre[j] : pend_m;
-    W.ms[lane + 32 * t] = j < mend ? mstart[j] : 0;
-  }
-  if (lane == 0) W.mp[128] = tb + 128 < mend ? L.mpre[tb + 128] : pend_m;
-  __syncwarp();
-}
-
-// Plan the window of positions [q, q + n) (n <= 128) whose first position lies
-// in member i0: e[t] = source entry of position q + lane + 32 t (or -1).
-// Advances i0 to the member containing q + n; may reload the table.
-__device__ __forceinline__ int exp_plan(const Layout &L, const int64_t *__restrict__ mstart, int64_t mend, int64_t q,
-                                        int64_t Pend, int64_t &i0, int64_t &tb, WarpExpTab &W, int64_t (&e)[4]) {
-  const int lane = threadIdx.x & 31;
-  const int64_t want = q + 128 < Pend ? q + 128 : Pend;
-  if (i0 >= tb + 128 || (W.mp[128] < want && i0 != tb)) {
-    __syncwarp();
-    tb = i0;
-    exp_table_load(L, mstart, mend, tb, W);
-  }
-  const int64_t limit = W.mp[128] < want ? W.mp[128] : want;
-  const int n = (int)(limit - q);
-#pragma unroll
-  for (int t = 0; t < 4; ++t) W.mk[lane + 32 * t] = -1;
-  __syncwarp();
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {  // member k starts inside the window and is non-empty
-    const int k = lane + 32 * t;
-    const int64_t rs = W.mp[k] - q;
-    if (rs >= 0 && rs < n && W.mp[k + 1] > W.mp[k]) W.mk[rs] = k;
-  }
-  __syncwarp();
-  // inclusive max-scan over positions (blocked: lane owns 4 consecutive ones)
-  const int base = (int)(i0 - tb);  // member containing q, relative to the table
-  int m[4], run = base;
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    run = max(run, W.mk[4 * lane + t]);
-    m[t] = run;
-  }
-  int x = run;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const int y = __shfl_up_sync(0xffffffffu, x, o);
-    if (lane >= o) x = max(x, y);
-  }
-  int before = __shfl_up_sync(0xffffffffu, x, 1);
-  if (lane == 0) before = base;
-  __syncwarp();
-#pragma unroll
-  for (int t = 0; t < 4; ++t) W.mk[4 * lane + t] = max(before, m[t]);
-  __syncwarp();
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    const int r = lane + 32 * t;
-    e[t] = -1;
-    if (r < n) {
-      const int k = W.mk[r];
-      e[t] = W.ms[k] + (q + r - W.mp[k]);
-    }
-  }
-  i0 = tb + last_le(W.mp, 0, 129, limit);
-  __syncwarp();
-  return n;
-}
-
-// Every member-edge position p in [P_lo, P_hi) (the active rows) gets its
-// fine entry's (b = M[v], w): Sb/Sw[p - P_lo].  One streaming pass with warp-level
-// member walks (no CTA barriers); all later construction kernels read these
-// arrays with coalesced loads.  Self entries are kept (b == own row): the
-// consumers know their row and drop them.  Two windows are in flight per warp:
-// the next window's col/wgt loads are issued before this window's M gathers.
-__global__ void __launch_bounds__(kXT) k_expand(Layout L, const int64_t *__restrict__ mstart,
-                                              int32_t *__restrict__ Sb, int32_t *__restrict__ Sw) {
-  __shared__ WarpExpTab W[kXT / 32];
-  const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
-  const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const int64_t gw = (int64_t)blockIdx.x * (kXT / 32) + wid;
-  const int64_t nw = (int64_t)gridDim.x * (kXT / 32);
-  for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
-    const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
-    int64_t i0 = warp_find_member(L, m_lo, m_hi, P);
-    int64_t tb = i0;
-    exp_table_load(L, mstart, m_hi, tb, W[wid]);
-    int64_t q = P, e[4];
-    int32_t b0[4], w0[4];
-    int n0 = exp_plan(L, mstart, m_hi, q, Pend, i0, tb, W[wid], e);
-    int64_t q0 = q;
-    q += n0;
-#pragma unroll
-    for (int t = 0; t < 4; ++t)
-      if (e[t] >= 0) { b0[t] = __ldcs(L.col + e[t]); w0[t] = __ldcs(L.wgt + e[t]); }
-    while (n0 > 0) {
-      int32_t b1[4], w1[4];
-      int n1 = 0;
-      const int64_t q1 = q;
-      if (q < Pend) {
-        n1 = exp_plan(L, mstart, m_hi, q, Pend, i0, tb, W[wid], e);
-        q += n1;
-#pragma unroll
-        for (int t = 0; t < 4; ++t)
-          if (e[t] >= 0) { b1[t] = __ldcs(L.col + e[t]); w1[t] = __ldcs(L.wgt + e[t]); }
-      }
-#pragma unroll
-      for (int t = 0; t < 4; ++t)
-        if (lane + 32 * t < n0) b0[t] = __ldg(L.M + b0[t]);
-#pragma unroll
-      for (int t = 0; t < 4; ++t) {
-        const int off = lane + 32 * t;
-        if (off < n0) {  // streaming stores: keep M (gathered) resident in L2
-          __stcs(Sb + q0 + off - P_lo, b0[t]);
-          __stcs(Sw + q0 + off - P_lo, w0[t]);
-        }
-      }
-#pragma unroll
-      for (int t = 0; t < 4; ++t) { b0[t] = b1[t]; w0[t] = w1[t]; }
-      n0 = n1;
-      q0 = q1;
-    }
-  }
-}
-
-// Expansion v2: a warp walks the members of its 4096-position chunk 32 at a
-// time (one coalesced load of their metadata per window).  Members with more
-// than kXBig positions in the chunk are streamed one by one by the whole warp;
-// the others are packed: a warp scan of their lengths gives every position of
-// the window a (member, offset) by a 5-step shuffle search, so short rows fill
-// all 32 lanes.  Four positions per lane are in flight per step (col, wgt,
-// then the M gathers).  No shared memory, no CTA barriers.
-constexpr int kXBig = 64;
-
-// Walk the member-edge positions [P, Pend) (all inside members [.., m_hi)):
-// sink(e[4], p[4], ok) receives, per step, up to four positions per lane (e:
-// source entry in col/wgt, p: position).  With skip != nullptr, members whose
-// coarse row has skip[M[member]] >= 0 are passed over (DENSE rows, expanded by
-// their accumulation kernel instead).
-template <int kLong, typename Sink, int kShort = 4, typename IdxT = int64_t>
-__device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restrict__ mstart, int64_t m_lo,
-                                        int64_t m_hi, int64_t P, int64_t Pend, const int32_t *__restrict__ skip,
-                                        Sink &sink) {
-  const int lane = threadIdx.x & 31;
-  int64_t i = warp_find_member(L, m_lo, m_hi, P);
-  while (true) {
-    const int64_t j = i + lane;
-    int64_t mp0 = L.mpre[m_hi], mp1 = mp0, rs = 0;
-    bool skipped = false;
-    if (j < m_hi) {
-      mp0 = L.mpre[j];
-      mp1 = L.mpre[j + 1];
-      rs = mstart[j];
-      if (skip) skipped = skip[L.M[L.members[j]]] >= 0;
-    }
-    const int64_t ps = mp0 > P ? mp0 : P;
-    const int64_t pe = mp1 < Pend ? mp1 : Pend;
-    const int d = (pe > ps && !skipped) ? (int)(pe - ps) : 0;
-    rs += ps - mp0;  // source entry of position ps
-    const bool big = d > kXBig;
-    // ---- packed short members
-    const int ds = big ? 0 : d;
-    int incl = ds;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int y = __shfl_up_sync(0xffffffffu, incl, o);
-      if (lane >= o) incl += y;
-    }
-    const int excl = incl - ds;
-    const int T = __shfl_sync(0xffffffffu, incl, 31);
-    for (int base = 0; base < T; base += 32 * kShort) {
-      IdxT e[kShort], p[kShort];
-      unsigned ok = 0;
-#pragma unroll
-      for (int u = 0; u < kShort; ++u) {
-        const int t = base + lane + 32 * u;
-        int lo = 0;  // largest lane with excl <= t
-#pragma unroll
-        for (int st = 16; st > 0; st >>= 1) {
-          const int c = lo + st;
-          const int v = __shfl_sync(0xffffffffu, excl, c & 31);
-          if (c < 32 && v <= t) lo = c;
-        }
-        const int64_t ors = __shfl_sync(0xffffffffu, rs, lo);
-        const int64_t ops = __shfl_sync(0xffffffffu, ps, lo);
-        const int oex = __shfl_sync(0xffffffffu, excl, lo);
-        e[u] = (IdxT)(ors + (t - oex));
-        p[u] = (IdxT)(ops + (t - oex));
-        if (t < T) ok |= 1u << u;
-      }
-      sink(e, p, ok);
-    }
-    // ---- long members, one at a time
-    unsigned bm = __ballot_sync(0xffffffffu, big);
-    while (bm) {
-      const int src = __ffs(bm) - 1;
-      bm &= bm - 1;
-      const int bd = __shfl_sync(0xffffffffu, d, src);
-      const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
-      const int64_t bps = __shfl_sync(0xffffffffu, ps, src);
-      for (int base = 0; base < bd; base += 32 * kLong) {  // kLong positions per lane in flight
-        IdxT e[kLong], p[kLong];
-        unsigned ok = 0;
-#pragma unroll
-        for (int u = 0; u < kLong; ++u) {
-          const int t = base + lane + 32 * u;
-          e[u] = (IdxT)(brs + t);
-          p[u] = (IdxT)(bps + t);
-          if (t < bd) ok |= 1u << u;
-        }
-        sink(e, p, ok);
-      }
-    }
-    // the window reaches the chunk end (or the last member): done
-    if (__any_sync(0xffffffffu, mp1 >= Pend)) break;
-    i += 32;
-  }
-}
-
+// Expansion (k_expand2): the rows no other kernel walks itself (warp pieces,
+// the SMALL / bin-piece blocks of the HEC_NO_RBM path) are staged once in
+// member-edge space by x2_walk (construct_common.cuh).
 // sink of the expansion: (M[v], w) to the staging at position - P_lo
 struct StageSink {
   const Layout &L;
@@ -513,7 +290,7 @@ struct StageSink {
 template <typename IdxT, int kPer>
 __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
                                                int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
-                                               const int32_t *__restrict__ skip) {
+                                               const int32_t *__restrict__ skip, int64_t skip_thr) {
   const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
   const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
   const int64_t gw = ((int64_t)blockIdx.x * kXT + threadIdx.x) >> 5;
@@ -521,7 +298,7 @@ __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__rest
   StageSink sink{L, Sb, Sw, P_lo};
   for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
     const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
-    x2_walk<kPer, StageSink, kPer, IdxT>(L, mstart, m_lo, m_hi, P, Pend, skip, sink);
+    x2_walk<kPer, StageSink, kPer, IdxT>(L, mstart, m_lo, m_hi, P, Pend, skip, sink, skip_thr);
   }
 }
 
@@ -543,7 +320,8 @@ struct PartArgs {
   const int64_t *unit_ptr;  // units of kUnit positions
   const int32_t *unit_row;  // unit -> big row index
   const int64_t *bkt_ptr;
-  const int32_t *Sb, *Sw;   // expanded entries, indexed from upos(a_lo)
+  const int32_t *Sb, *Sw;   // expanded entries, indexed from upos(a_lo) (k_part_warp rows only)
+  const int64_t *mstart;    // row_ptr[members[i]] (unit passes walk the member rows)
 };
 
 struct UnitInfo {
@@ -590,68 +368,108 @@ __device__ __forceinline__ int entry_bucket(const UnitInfo &u, int32_t b) {
 // passes are bound by per-unit latency, not by same-address replays.)
 __device__ __forceinline__ int agg_add(int32_t *ctr, int bk) { return bk < 0 ? -1 : atomicAdd(ctr + bk, 1); }
 
-// histogram of the unit's entries (self entries dropped) into S.hist
-__device__ __forceinline__ void unit_hist(const PartArgs &A, const UnitInfo &u, PartSmem &S) {
-  for (int i = threadIdx.x; i < u.nb; i += kT) S.hist[i] = 0;
-  __syncthreads();
-  const int32_t *Sb = A.Sb + u.p0;
-  const int cnt = (int)(u.p1 - u.p0);  // <= kUnit
-  // warp-uniform trip count: agg_add's __match_any_sync needs every lane
-  for (int p = threadIdx.x; p - (int)(threadIdx.x & 31) < cnt; p += kPartU * kT) {
-    int32_t b[kPartU];
-#pragma unroll
-    for (int j = 0; j < kPartU; ++j) b[j] = p + j * kT < cnt ? __ldcs(Sb + p + j * kT) : u.a;
-#pragma unroll
-    for (int j = 0; j < kPartU; ++j) agg_add(S.hist, entry_bucket(u, b[j]));
-  }
-  __syncthreads();
+// The unit passes read the member rows themselves (col / wgt streamed once per
+// pass, b = M[v] gathered): a CTA's 16 warps each walk 1/16 of the unit's
+// member-edge positions with x2_walk (no expansion staging for these rows).
+constexpr int kPartSlice = kUnit / (kT / 32);
+
+__device__ __forceinline__ void unit_slice(const UnitInfo &u, int64_t P_lo, int64_t &Pw, int64_t &Pwe) {
+  const int wid = threadIdx.x >> 5;
+  Pw = P_lo + u.p0 + (int64_t)wid * kPartSlice;
+  Pwe = P_lo + u.p1;
+  if (Pw + kPartSlice < Pwe) Pwe = Pw + kPartSlice;
 }
+
+// count pass: bucket of every entry (self entries dropped) into hist
+struct PartCountSink {
+  const Layout &L;
+  const UnitInfo &u;
+  int32_t *hist;
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
+    (void)p;
+    int32_t b[N];
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) b[q] = __ldcs(L.col + e[q]);
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) b[q] = __ldg(L.M + b[q]);
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) agg_add(hist, entry_bucket(u, b[q]));
+  }
+};
+
+// write pass: (b, w) to the entry's slot of its bin (shared-memory cursors)
+struct PartWriteSink {
+  const Layout &L;
+  const UnitInfo &u;
+  int32_t *cursor;
+  int32_t *__restrict__ pbr, *__restrict__ pwr;
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
+    (void)p;
+    int32_t b[N], w[N];
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) { b[q] = __ldcs(L.col + e[q]); w[q] = __ldcs(L.wgt + e[q]); }
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) b[q] = __ldg(L.M + b[q]);
+#pragma unroll
+    for (int q = 0; q < N; ++q) {
+      if (!(ok & (1u << q))) continue;
+      const int slot = agg_add(cursor, entry_bucket(u, b[q]));
+      if (slot >= 0) {
+        pbr[slot] = b[q];
+        pwr[slot] = w[q];
+      }
+    }
+  }
+};
 
 // The unit's slice of each bin is reserved here: the returned running count
 // is the unit's offset inside the bin (ubase), so the write pass needs no
 // second histogram.
+template <typename IdxT>
 __global__ void __launch_bounds__(kT) k_part_count(PartArgs A, unsigned *__restrict__ bkt_cnt,
                                                    int32_t *__restrict__ ubase) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   const UnitInfo u = unit_info(A, blockIdx.x);
-  unit_hist(A, u, S);
+  const Layout &L = A.L;
+  for (int i = threadIdx.x; i < u.nb; i += kT) S.hist[i] = 0;
+  __syncthreads();
+  int64_t Pw, Pwe;
+  unit_slice(u, L.upos(L.a_lo), Pw, Pwe);
+  PartCountSink sink{L, u, S.hist};
+  if (Pw < Pwe) x2_walk<8, PartCountSink, 4, IdxT>(L, A.mstart, L.member_ptr[u.a], L.member_ptr[u.a + 1], Pw, Pwe,
+                                                  nullptr, sink);
+  __syncthreads();
   int32_t *ub = ubase + (int64_t)blockIdx.x * kPartHist;
   for (int i = threadIdx.x; i < u.nb; i += kT)
     if (S.hist[i]) ub[i] = (int32_t)atomicAdd(bkt_cnt + u.b0 + i, (unsigned)S.hist[i]);
 }
 
+template <typename IdxT>
 __global__ void __launch_bounds__(kT) k_part_write(PartArgs A, const int64_t *__restrict__ bkt_off,
                                                    const int32_t *__restrict__ ubase, int32_t *__restrict__ pb,
                                                    int32_t *__restrict__ pw) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   const UnitInfo u = unit_info(A, blockIdx.x);
+  const Layout &L = A.L;
   const int64_t off0 = bkt_off[u.b0];
   const int32_t *ub = ubase + (int64_t)blockIdx.x * kPartHist;
   for (int i = threadIdx.x; i < u.nb; i += kT)  // (slots of bins the unit never hits stay unused)
     S.base[i] = (int32_t)(bkt_off[u.b0 + i] - off0) + ub[i];
   __syncthreads();
-  const int32_t *Sb = A.Sb + u.p0, *Sw = A.Sw + u.p0;
-  int32_t *pbr = pb + off0, *pwr = pw + off0;
-  const int cnt = (int)(u.p1 - u.p0);
-  for (int p = threadIdx.x; p - (int)(threadIdx.x & 31) < cnt; p += kPartU * kT) {
-    int32_t b[kPartU], w[kPartU];
-#pragma unroll
-    for (int j = 0; j < kPartU; ++j) {
-      const bool in = p + j * kT < cnt;
-      b[j] = in ? __ldcs(Sb + p + j * kT) : u.a;
-      w[j] = in ? __ldcs(Sw + p + j * kT) : 0;
-    }
-#pragma unroll
-    for (int j = 0; j < kPartU; ++j) {
-      const int q = agg_add(S.base, entry_bucket(u, b[j]));
-      if (q >= 0) {
-        pbr[q] = b[j];
-        pwr[q] = w[j];
-      }
-    }
-  }
+  int64_t Pw, Pwe;
+  unit_slice(u, L.upos(L.a_lo), Pw, Pwe);
+  PartWriteSink sink{L, u, S.base, pb + off0, pw + off0};
+  if (Pw < Pwe) x2_walk<8, PartWriteSink, 4, IdxT>(L, A.mstart, L.member_ptr[u.a], L.member_ptr[u.a + 1], Pw, Pwe,
+                                                  nullptr, sink);
 }
 
 // Skewed rows with U <= kWarpRowMax (<= kWarpBins bins): one warp counts the
@@ -1043,89 +861,13 @@ struct DenseArgs {
   int64_t nunits;
   unsigned *ticket;
   unsigned long long *dense;  // [nbig][n_c] (zeroed)
-  const int32_t *Sb, *Sw;     // expanded entries, indexed from upos(a_lo)
 };
 
-// A dense unit is kDenseIt entries per thread: all of a unit's loads are issued
-// before its atomics, so each CTA keeps 16 KB x 2 of staging reads in flight
-// (one 4096-entry unit per round trip left the kernel latency-bound).
-constexpr int kDenseIt = 16;
-constexpr int kDenseUnit = kT * kDenseIt;
-constexpr int kDenseUnit2 = 4 * kDenseUnit;  // fused DENSE units: 2048 positions per warp, one barrier
-
-__global__ void __launch_bounds__(kT) k_dense_accum(DenseArgs A) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  int32_t *acc = reinterpret_cast<int32_t *>(smem_raw);
-  __shared__ int64_t s_unit;
-  __shared__ long long s_w[kT / 32];
-  const Layout &L = A.L;
-  const int nc = (int)L.n_c;
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (int b = threadIdx.x; b < nc; b += kT) acc[b] = 0;
-  const int64_t P_lo = L.upos(L.a_lo);
-  int64_t cur_h = -1;
-  long long running = 0;  // weight accumulated since the last merge
-  while (true) {
-    if (threadIdx.x == 0) s_unit = (int64_t)atomicAdd(A.ticket, 1u);
-    __syncthreads();
-    const int64_t unit = s_unit;
-    const int64_t h = unit < A.nunits ? A.unit_row[unit] : -1;
-    int32_t kb[kDenseIt], kw[kDenseIt];
-    long long usum = 0;  // exact weight of this thread's slots
-#pragma unroll
-    for (int k = 0; k < kDenseIt; ++k) { kb[k] = -1; kw[k] = 0; }
-    if (h >= 0) {
-      const int32_t a = A.big_list[h];
-      const int64_t P0 = L.upos(a) + (unit - A.unit_ptr[h]) * kDenseUnit;
-      const int cnt = (int)min((int64_t)kDenseUnit, L.upos(a + 1) - P0);
-      const int32_t *Sb = A.Sb + (P0 - P_lo), *Sw = A.Sw + (P0 - P_lo);
-#pragma unroll
-      for (int k = 0; k < kDenseIt; ++k) {
-        const int p = threadIdx.x + kT * k;
-        if (p < cnt) { kb[k] = __ldcs(Sb + p); kw[k] = __ldcs(Sw + p); }
-      }
-#pragma unroll
-      for (int k = 0; k < kDenseIt; ++k) {
-        if (kb[k] == a) kb[k] = -1;  // self entry (L280)
-        if (kb[k] >= 0) usum += kw[k];
-      }
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) usum += __shfl_xor_sync(0xffffffffu, usum, o);
-    if (lane == 0) s_w[wid] = usum;
-    __syncthreads();
-    long long unit_w = 0;
-    for (int w = 0; w < kT / 32; ++w) unit_w += s_w[w];
-    if (cur_h >= 0 && (h != cur_h || running + unit_w > 0x7fffffffLL)) {  // merge the accumulator
-      unsigned long long *dst = A.dense + cur_h * (int64_t)nc;
-      for (int b = threadIdx.x; b < nc; b += kT) {
-        int32_t v = acc[b];
-        if (v) { atomicAdd(dst + b, (unsigned long long)(uint32_t)v); acc[b] = 0; }
-      }
-      running = 0;
-      __syncthreads();
-    }
-    if (h < 0) return;
-    cur_h = h;
-    if (unit_w > 0x7fffffffLL) {  // the unit alone could overflow int32: exact 64-bit sums in global
-      unsigned long long *dst = A.dense + h * (int64_t)nc;
-#pragma unroll
-      for (int k = 0; k < kDenseIt; ++k)
-        if (kb[k] >= 0) atomicAdd(dst + kb[k], (unsigned long long)(uint32_t)kw[k]);
-      __syncthreads();
-      continue;
-    }
-    running += unit_w;
-#pragma unroll
-    for (int k = 0; k < kDenseIt; ++k)
-      if (kb[k] >= 0) atomicAdd(acc + kb[k], kw[k]);
-    __syncthreads();
-  }
-}
+constexpr int kDenseUnit2 = 32768;  // DENSE units: 2048 positions per warp, one barrier per unit
 
 // DENSE rows fused with their expansion: a persistent CTA takes units of
-// kDenseUnit member-edge positions of one big row; each warp walks its
-// kDenseUnit/16 positions of the row's member rows (x2_walk), gathers M[v] and
+// kDenseUnit2 member-edge positions of one big row; each warp walks its
+// kDenseUnit2/16 positions of the row's member rows (x2_walk), gathers M[v] and
 // adds w into the shared-memory accumulator of the row (uint32: a partial sum
 // above INT32_MAX or a wrap means the coarse weight overflows -- ERR_OVERFLOW
 // here or in k_rows); the accumulator is merged into dense[h] when the CTA
@@ -1280,10 +1022,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     return HEC_EINVAL;
   }
   const int64_t n_out = a_hi - a_lo;  // rows produced by this call
+  // 32-bit entry / position indices in the member walks when nnz < 2^32
+  // (HEC_FORCE_WIDE_INDEX: test hook for the 64-bit instantiation)
+  const bool idx32 = g->nnz < ((int64_t)1 << 32) && getenv("HEC_FORCE_WIDE_INDEX") == nullptr;
   Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi};
   const bool dense = n_c <= kDenseMax;
-  // DENSE rows expanded inside their accumulation (HEC_DENSE_STAGED: staged v1, test hook)
-  const bool fused_dense = dense && getenv("HEC_DENSE_STAGED") == nullptr;
   // bitmap-rank items replace the bin pieces when the key range fits the
   // shared-memory bitmap (HEC_NO_RBM: test / tuning hook for the bin-piece path)
   // rank items for every level (DENSE levels: the small rows); bins are kept
@@ -1306,7 +1049,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t small_vol = r0[1], big_vol = r0[2];
   const int64_t nbig = r0[4] & 0xffffffffLL;
   if (nbig > 0) {
-    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)(fused_dense ? kDenseUnit2 : kDenseUnit) : (int64_t)kUnit,
+    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)kDenseUnit2 : (int64_t)kUnit,
                                              dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
                          st[4], unit_ptr + nbig));
     if (!dense) HEC_TRY(chained_scan(ctx, nbig, BucketsIn{L, big_list, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + nbig));
@@ -1366,12 +1109,16 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     int64_t grid = (warps + kXT / 32 - 1) / (kXT / 32);
     const int64_t cap = (int64_t)ctx->num_sms * 8;
     if (grid > cap) grid = cap;
+    // rank items (rbm: every row above kPieceMax), rows partitioned by CTA
+    // units (U > kWarpRowMax) and fused DENSE rows are walked by their own
+    // kernels: the staging covers the other rows only
+    const int32_t *skip = rbm ? nullptr : big_idx;
+    const int64_t skip_thr = rbm ? (int64_t)kPieceMax : dense ? 0 : kWarpRowMax;
     if (grid > 0) {
-      if (getenv("HEC_EXPAND_V1")) k_expand<<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt);
-      else if (g->nnz < ((int64_t)1 << 32) && getenv("HEC_EXPAND_W64") == nullptr)  // 32-bit entry / position indices
-        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, fused_dense ? big_idx : nullptr);
+      if (idx32)
+        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr);
       else
-        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, fused_dense ? big_idx : nullptr);
+        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr);
       HEC_LAUNCH_CHECK();
     }
     phase_end(ctx, phx);
@@ -1395,90 +1142,31 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   A.bkt_ptr = bkt_ptr;
   A.grp_end = grp_end;
   A.err = err;
+  A.mstart = mstart;
+  A.idx32 = idx32;
 
   static bool attr = false;
   if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(PartSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)sizeof(PartSmem)));
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count<int64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)sizeof(PartSmem)));
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write<int64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(PartSmem)));
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_bucket_fallback, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(FbSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_dense_accum, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)(4 * kDenseMax)));
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_dense_accum2, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)(4 * kDenseMax)));
     attr = true;
   }
 
-  // ---- overlap: whole rows (pieces, rank items) on the aux stream while the
-  // skewed rows are partitioned on the main stream; they share no data but
-  // the staging, which both only read (rank items rewrite their own rows)
-  const bool direct = getenv("HEC_NO_DRANK") == nullptr;
-  // (opt-in, HEC_OVERLAP=1: measured 4 % slower on C4 -- the partition and the
-  // rank kernels compete for shared memory and both are latency-bound)
-  const bool overlap = rbm && !dense && nbig > 0 && nblocks > 0 && getenv("HEC_OVERLAP") != nullptr;
-  RbmItem *list_rb = nullptr, *list_rb2 = nullptr, *list_rb3 = nullptr;  // bins' rank items (overlap mode)
-  // an error return between fork and join must not leave aux work touching the workspace
-  struct AuxGuard {
-    hec_ctx *c = nullptr;
-    ~AuxGuard() {
-      if (c) cudaStreamSynchronize(c->aux);
-    }
-  } aux_guard;
+  const bool direct = getenv("HEC_NO_DRANK") == nullptr;  // test hook: bins through the hash-rank kernels
   int ph_rows = -1;
-  if (overlap) {
-    list_rb = arena_take<RbmItem>(W2, nblocks + 1);
-    list_rb2 = arena_take<RbmItem>(W2, nblocks + 1);
-    list_rb3 = arena_take<RbmItem>(W2, nblocks + 1);
-    if (!list_rb3) { set_error("workspace under-reserved (bin lists)"); return HEC_EINVAL; }
-    if (!ctx->aux) {
-      HEC_CUDA_TRY(cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking));
-      HEC_CUDA_TRY(cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming));
-      HEC_CUDA_TRY(cudaEventCreateWithFlags(&ctx->ev_join, cudaEventDisableTiming));
-    }
-    HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
-    HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
-    A.row_ptr_c = out->row_ptr;
-    A.vwgt_c = out->vwgt;
-    // one phase for the overlapped partition + dedup (their times cannot be split)
-    ph_rows = phase_begin(ctx, "rows", 8.0 * (double)(small_vol + big_vol) + 8.0 * (double)big_vol);
-    k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
-    HEC_LAUNCH_CHECK();
-    HEC_CUDA_TRY(cudaEventRecord(ctx->ev_fork, s));
-    HEC_CUDA_TRY(cudaStreamWaitEvent(ctx->aux, ctx->ev_fork, 0));
-    aux_guard.c = ctx;
-    cudaStream_t main_s = ctx->stream;
-    ctx->stream = ctx->aux;
-    int rc = HEC_OK;
-    k_tiers<<<nblk(nblocks, 256), 256, 0, ctx->aux>>>(L, nblocks, blk, big_idx, bkt_ptr, nullptr, nullptr, nullptr, blk_cnt,
-                                                     grp_end, list_w, list_c, list_r, list_r2, list_d, list_r3, counts + 10,
-                                                     rbm, direct, 1, vw64, err);
-    ctx->launches++;
-    if (cudaGetLastError() != cudaSuccess) rc = HEC_ECUDA;
-    RowsArgs B = A;
-    B.items = list_w;
-    B.nlist = counts + 10;
-    if (rc == HEC_OK) rc = launch_pieces(ctx, B, counts + 5);
-    B.rcap = nblocks + 1;
-    const struct { RbmItem *items; unsigned *n; int dir; } wcls[4] = {
-        {list_r3, counts + 13, 1}, {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}};
-    for (int c = 0; c < 4 && rc == HEC_OK; ++c) {
-      B.ritems = wcls[c].items;
-      B.nlist = wcls[c].n;
-      B.rdir = wcls[c].dir;
-      rc = launch_hrank(ctx, B, c - 1);
-    }
-    if (rc == HEC_OK && cudaEventRecord(ctx->ev_join, ctx->aux) != cudaSuccess) rc = HEC_ECUDA;
-    ctx->stream = main_s;
-    if (rc != HEC_OK) {
-      cudaStreamSynchronize(ctx->aux);
-      return rc;
-    }
-  }
 
   // ---- a9 skewed rows
-  const int ph_skew = overlap ? -1 : phase_begin(ctx, "rows_skew", 8.0 * (double)big_vol);
+  const int ph_skew = phase_begin(ctx, "rows_skew", 8.0 * (double)big_vol);
   int32_t *unit_row = nullptr;
   if (nbig > 0) {
     unit_row = arena_take<int32_t>(W2, nunits + 1);
@@ -1489,13 +1177,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (nbig > 0 && dense) {
     unsigned long long *dn_arr = arena_take<unsigned long long>(W2, (size_t)nbig * n_c);
     HEC_CUDA_TRY(cudaMemsetAsync(dn_arr, 0, sizeof(unsigned long long) * nbig * n_c, s));
-    DenseArgs D{L, big_list, nbig, unit_ptr, unit_row, nunits, counts + 2, dn_arr, sc_col, sc_wgt};
+    DenseArgs D{L, big_list, nbig, unit_ptr, unit_row, nunits, counts + 2, dn_arr};
     int occ = 1;
-    if (fused_dense) HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum2, kT, 4 * (size_t)n_c));
-    else HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum, kT, 4 * (size_t)n_c));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum2, kT, 4 * (size_t)n_c));
     if (occ < 1) occ = 1;
-    if (fused_dense) k_dense_accum2<<<ctx->num_sms * occ, kT, 4 * (size_t)n_c, s>>>(D, mstart, err);
-    else k_dense_accum<<<ctx->num_sms * occ, kT, 4 * (size_t)n_c, s>>>(D);
+    k_dense_accum2<<<ctx->num_sms * occ, kT, 4 * (size_t)n_c, s>>>(D, mstart, err);
     HEC_LAUNCH_CHECK();
     A.dense = dn_arr;
   } else if (nbig > 0) {
@@ -1515,13 +1201,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     int64_t *prow = arena_take<int64_t>(W2, nbig + 1);
     if (!prow) { set_error("workspace under-reserved (prow)"); return HEC_EINVAL; }
     HEC_TRY(chained_scan(ctx, nbig, RowUIn{L, big_list}, PtrOut{prow}, stb, prow + nbig));
-    PartArgs PA{L, big_list, nbig, unit_ptr, unit_row, bkt_ptr, sc_col, sc_wgt};
+    PartArgs PA{L, big_list, nbig, unit_ptr, unit_row, bkt_ptr, sc_col, sc_wgt, mstart};
     if (nunits > 0) {  // rows above kWarpRowMax: CTA units count, per-row scan, scatter
-      k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
+      if (idx32) k_part_count<uint32_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
+      else k_part_count<int64_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
       HEC_LAUNCH_CHECK();
       k_row_bins<<<nblk(nbig * 32, 256), 256, 0, s>>>(PA, prow, bkt_cnt, bkt_off);
       HEC_LAUNCH_CHECK();
-      k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, ubase, pb, pw);
+      if (idx32) k_part_write<uint32_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, ubase, pb, pw);
+      else k_part_write<int64_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, ubase, pb, pw);
       HEC_LAUNCH_CHECK();
     }
     k_part_warp<<<nblk(nbig * 32, kPWT), kPWT, 0, s>>>(PA, prow, bkt_off, bkt_cnt, pb, pw);
@@ -1561,75 +1249,43 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (ph_skew >= 0) phase_end(ctx, ph_skew);
   // counts: [5] pieces ticket [8] wide list [10] warp list [11] CTA list [12] bitmap-rank list
   //         [13] bitmap-rank ticket
-  if (nblocks > 0 && !overlap) {
+  if (nblocks > 0) {
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
                                               list_c, list_r, list_r2, list_d, list_r3, counts + 10, rbm, direct, 0, vw64, err);
     HEC_LAUNCH_CHECK();
-  } else if (nblocks > 0) {  // the whole rows are already in flight on the aux stream: bins now
-    k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, list_rb, list_rb2, list_d, list_rb3, counts + 20, rbm, direct, 2, vw64, err);
-    HEC_LAUNCH_CHECK();
   }
 
   // ---- work blocks (a8/a9 output), then placement (a10)
-  if (!overlap) {
-    HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
-    HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
-  }
+  HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
+  HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
   out->n_c = n_out;
   A.row_ptr_c = out->row_ptr;
   A.vwgt_c = out->vwgt;
-  long long *trace = nullptr;
-  if (getenv("HEC_TRACE_ROWS")) {
-    HEC_TRY(dev_alloc(ctx, (void **)&trace, sizeof(long long) * 4 * (nblocks + 1)));
-    A.trace = trace;
-  }
-  if (!overlap) ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
+  ph_rows = phase_begin(ctx, "rows", 8.0 * (double)small_vol);
   A.items = list_w;
   A.nlist = counts + 10;
-  unsigned long long *pstats = nullptr;
-  if (getenv("HEC_PIECE_STATS")) {
-    HEC_TRY(dev_alloc(ctx, (void **)&pstats, 16 * sizeof(unsigned long long)));
-    HEC_CUDA_TRY(cudaMemsetAsync(pstats, 0, 16 * sizeof(unsigned long long), s));
-    A.pstats = pstats;
-  }
-  if (!overlap) HEC_TRY(launch_pieces(ctx, A, counts + 5));
-  if (pstats) {
-    unsigned long long h[16];
-    HEC_CUDA_TRY(cudaMemcpyAsync(h, pstats, sizeof h, cudaMemcpyDeviceToHost, s));
-    HEC_CUDA_TRY(cudaStreamSynchronize(s));
-    fprintf(stderr, "[pieces n_c=%lld]", (long long)n_c);
-    for (int c = 0; c < 8; ++c) fprintf(stderr, " %s%d:%llu/%llu", c < 4 ? "bin" : "row", 32 << (c & 3), h[2 * c], h[2 * c + 1]);
-    fprintf(stderr, "\n");
-    dev_free(ctx, pstats);
-    A.pstats = nullptr;
-  }
-  if (!overlap) {
-    A.list = list_c;
-    A.nlist = counts + 11;
-    HEC_TRY(launch_rows(ctx, A, false));
-  }
+  HEC_TRY(launch_pieces(ctx, A, counts + 5));
+  A.list = list_c;
+  A.nlist = counts + 11;
+  HEC_TRY(launch_rows(ctx, A, false));
   if (rbm) {
     A.ticket = counts + 30;  // (unused by the rank kernels)
     A.rcap = nblocks + 1;
-    // hash-rank size classes, then the bitmap-rank items above kHrMax2 entries
-    // (overlap mode: classes 0-2 of the whole rows ran on the aux stream; here the bins)
+    // hash-rank size classes, then the multi-round hash rank above kHrMax2
+    // entries (items with too many distinct keys -> the bitmap rank k_rbm)
     struct RankList { RbmItem *items; unsigned *n; int dir; };
     const RankList cls[5] = {{list_r3, counts + 13, 1},
         {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}, {list_r2, counts + 16, -1}};
-    const RankList bcls[5] = {{list_rb3, counts + 23, 1},
-        {list_rb, counts + 22, 1}, {list_rb, counts + 24, -1}, {list_rb2, counts + 25, 1}, {list_rb2, counts + 26, -1}};
     for (int c = -1; c < 4; ++c) {
-      const RankList &C = overlap ? bcls[c + 1] : cls[c + 1];
+      const RankList &C = cls[c + 1];
       A.ritems = C.items;
       A.nlist = C.n;
       A.rdir = C.dir;
-      if (c < 3) HEC_TRY(launch_hrank(ctx, A, c));
-      else if (getenv("HEC_NO_HRANK_BIG")) HEC_TRY(launch_rbm(ctx, A));
-      else {
-        // multi-round hash rank; items with too many distinct keys -> k_rbm
+      if (c < 3) {
+        HEC_TRY(launch_hrank(ctx, A, c));
+      } else {
         HEC_TRY(launch_hrank_big(ctx, A, list_redo, counts + 17));
         A.ritems = list_redo;
         A.nlist = counts + 17;
@@ -1638,29 +1294,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
       }
     }
     A.ritems = list_d;
-    A.nlist = overlap ? counts + 28 : counts + 18;
+    A.nlist = counts + 18;
     A.rdir = 1;
     HEC_TRY(launch_drank(ctx, A));
     A.ticket = counts + 1;
   }
-  if (overlap) {  // join the whole rows; CTA-tier blocks (if any) after both
-    HEC_CUDA_TRY(cudaStreamWaitEvent(s, ctx->ev_join, 0));
-    aux_guard.c = nullptr;  // main is ordered after the aux work from here on
-    A.list = list_c;
-    A.nlist = counts + 11;
-    HEC_TRY(launch_rows(ctx, A, false));
-  }
   phase_end(ctx, ph_rows);
-  if (trace) {
-    std::vector<long long> h(4 * nblocks);
-    HEC_CUDA_TRY(cudaMemcpyAsync(h.data(), trace, sizeof(long long) * 4 * nblocks, cudaMemcpyDeviceToHost, s));
-    HEC_CUDA_TRY(cudaStreamSynchronize(s));
-    char fn[256];
-    snprintf(fn, sizeof fn, "%s_%lld.bin", getenv("HEC_TRACE_ROWS"), (long long)n_c);
-    FILE *f = fopen(fn, "wb");
-    if (f) { fwrite(h.data(), sizeof(long long), h.size(), f); fclose(f); }
-    dev_free(ctx, trace);
-  }
   HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 12, blk_off + nblocks, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
   int64_t r2[13];
@@ -1698,9 +1337,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   phase_end(ctx, ph_place);
   // rows phase: staged / partitioned entries read (8 B each; DENSE rows were
   // accumulated in rows_skew), distinct entries staged (8 B), row_ptr_c + vwgt_c
-  // (overlap mode: the partition's pair writes are in this phase too)
-  phase_set_bytes(ctx, ph_rows, 8.0 * (double)(small_vol + (dense ? 0 : big_vol)) + 8.0 * (double)nnz_c + 12.0 * dnc +
-                                    (overlap ? 8.0 * (double)big_vol : 0.0));
+  phase_set_bytes(ctx, ph_rows, 8.0 * (double)(small_vol + (dense ? 0 : big_vol)) + 8.0 * (double)nnz_c + 12.0 * dnc);
   if (nblocks == 0) HEC_CUDA_TRY(cudaMemsetAsync(out->row_ptr, 0, sizeof(int64_t) * (n_out + 1), s));
   ctx->stats.nnz_c = out->nnz_c;
   return HEC_OK;

@@ -117,91 +117,6 @@ struct Layout {
   __device__ __forceinline__ int64_t U(int64_t a) const { return upos(a + 1) - upos(a); }
 };
 
-// ------------------------------------------------------- warp expansion
-// Warp-private member window in shared memory.
-struct WarpExpTab {
-  int64_t mp[129];  // member-edge start of members i0 .. i0+128 (mpre)
-  int64_t ms[128];  // row_ptr[members[i]] (mstart)
-  int32_t mk[128];  // position -> member (relative to i0)
-};
-
-// One warp expands the member-edge positions [P, limit) with limit <=
-// min(P + 128, Pend, start of member i0 + 128) into registers: slot t of lane l
-// is position P + l + 32 t; b = -1 marks empty slots.  Members are [i0, mend)
-// with i0 the member containing P; on return i0 is the member containing limit.
-// mem[t] receives the member index of the slot.  Positions find their member by
-// a mark + warp max-scan (each non-empty member marks its first position).
-// Only __syncwarp is used, so warps of a CTA proceed independently.
-// Returns limit - P.
-__device__ __forceinline__ int warp_expand(const Layout &L, const int64_t *__restrict__ mstart, int64_t mend,
-                                           int64_t P, int64_t Pend, int64_t &i0, WarpExpTab &W,
-                                           int32_t (&b)[4], int32_t (&w)[4], int64_t (&mem)[4]) {
-  const int lane = threadIdx.x & 31;
-  const int64_t pend_m = L.mpre[mend];
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    const int64_t j = i0 + lane + 32 * t;
-    W.mp[lane + 32 * t] = j < mend ? L.mpre[j] : pend_m;
-    W.ms[lane + 32 * t] = j < mend ? mstart[j] : 0;
-    W.mk[lane + 32 * t] = -1;
-  }
-  if (lane == 0) W.mp[128] = (i0 + 128 < mend) ? L.mpre[i0 + 128] : pend_m;
-  __syncwarp();
-  int64_t limit = P + 128;
-  if (Pend < limit) limit = Pend;
-  if (W.mp[128] < limit) limit = W.mp[128];
-  const int n = (int)(limit - P);
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {  // member k starts inside the window and is non-empty
-    const int k = lane + 32 * t;
-    const int64_t rs = W.mp[k] - P;
-    if (rs >= 0 && rs < n && W.mp[k + 1] > W.mp[k]) W.mk[rs] = k;
-  }
-  __syncwarp();
-  // inclusive max-scan over positions (blocked: lane owns 4 consecutive ones)
-  int m[4], run = 0;  // position 0 lies in member 0 (i0 contains P)
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    run = max(run, W.mk[4 * lane + t]);
-    m[t] = run;
-  }
-  int x = run;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const int y = __shfl_up_sync(0xffffffffu, x, o);
-    if (lane >= o) x = max(x, y);
-  }
-  int before = __shfl_up_sync(0xffffffffu, x, 1);
-  if (lane == 0) before = 0;
-  __syncwarp();
-#pragma unroll
-  for (int t = 0; t < 4; ++t) W.mk[4 * lane + t] = max(before, m[t]);
-  __syncwarp();
-  int64_t e[4];
-  unsigned valid = 0;
-#pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    const int r = lane + 32 * t;
-    b[t] = -1;
-    w[t] = 0;
-    if (r < n) {
-      const int k = W.mk[r];
-      e[t] = W.ms[k] + (P + r - W.mp[k]);
-      mem[t] = i0 + k;
-      valid |= 1u << t;
-    }
-  }
-#pragma unroll
-  for (int t = 0; t < 4; ++t)
-    if (valid & (1u << t)) { b[t] = __ldcs(L.col + e[t]); w[t] = __ldcs(L.wgt + e[t]); }  // streamed once
-#pragma unroll
-  for (int t = 0; t < 4; ++t)
-    if (valid & (1u << t)) b[t] = __ldg(L.M + b[t]);
-  i0 += last_le(W.mp, 0, 129, limit);
-  __syncwarp();
-  return n;
-}
-
 // Largest member i in [lo, hi) with mpre[i] <= P (mpre[lo] <= P), by a warp:
 // 32-ary search, one coalesced probe per round.
 __device__ __forceinline__ int64_t warp_find_member(const Layout &L, int64_t lo, int64_t hi, int64_t P) {
@@ -219,6 +134,98 @@ __device__ __forceinline__ int64_t warp_find_member(const Layout &L, int64_t lo,
   const bool le = idx < hi && L.mpre[idx] <= P;
   return lo + __popc(__ballot_sync(0xffffffffu, le)) - 1;
 }
+
+// ------------------------------------------------------- member walk
+constexpr int kXBig = 64;
+
+// Walk the member-edge positions [P, Pend) (all inside members [.., m_hi)):
+// sink(e[4], p[4], ok) receives, per step, up to four positions per lane (e:
+// source entry in col/wgt, p: position).  Members whose coarse row a has
+// U(a) > skip_thr (and skip[a] >= 0 when skip != nullptr) are passed over: rows
+// that their own kernels walk (rank items, DENSE accumulation, unit partition).
+template <int kLong, typename Sink, int kShort = 4, typename IdxT = int64_t>
+__device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restrict__ mstart, int64_t m_lo,
+                                        int64_t m_hi, int64_t P, int64_t Pend, const int32_t *__restrict__ skip,
+                                        Sink &sink, int64_t skip_thr = INT64_MAX) {
+  const int lane = threadIdx.x & 31;
+  int64_t i = warp_find_member(L, m_lo, m_hi, P);
+  while (true) {
+    const int64_t j = i + lane;
+    int64_t mp0 = L.mpre[m_hi], mp1 = mp0, rs = 0;
+    bool skipped = false;
+    if (j < m_hi) {
+      mp0 = L.mpre[j];
+      mp1 = L.mpre[j + 1];
+      rs = mstart[j];
+      if (skip_thr != INT64_MAX) {
+        const int32_t a = L.M[L.members[j]];
+        skipped = L.U(a) > skip_thr && (!skip || skip[a] >= 0);
+      }
+    }
+    const int64_t ps = mp0 > P ? mp0 : P;
+    const int64_t pe = mp1 < Pend ? mp1 : Pend;
+    const int d = (pe > ps && !skipped) ? (int)(pe - ps) : 0;
+    rs += ps - mp0;  // source entry of position ps
+    const bool big = d > kXBig;
+    // ---- packed short members
+    const int ds = big ? 0 : d;
+    int incl = ds;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    const int excl = incl - ds;
+    const int T = __shfl_sync(0xffffffffu, incl, 31);
+    for (int base = 0; base < T; base += 32 * kShort) {
+      IdxT e[kShort], p[kShort];
+      unsigned ok = 0;
+#pragma unroll
+      for (int u = 0; u < kShort; ++u) {
+        const int t = base + lane + 32 * u;
+        int lo = 0;  // largest lane with excl <= t
+#pragma unroll
+        for (int st = 16; st > 0; st >>= 1) {
+          const int c = lo + st;
+          const int v = __shfl_sync(0xffffffffu, excl, c & 31);
+          if (c < 32 && v <= t) lo = c;
+        }
+        const int64_t ors = __shfl_sync(0xffffffffu, rs, lo);
+        const int64_t ops = __shfl_sync(0xffffffffu, ps, lo);
+        const int oex = __shfl_sync(0xffffffffu, excl, lo);
+        e[u] = (IdxT)(ors + (t - oex));
+        p[u] = (IdxT)(ops + (t - oex));
+        if (t < T) ok |= 1u << u;
+      }
+      sink(e, p, ok);
+    }
+    // ---- long members, one at a time
+    unsigned bm = __ballot_sync(0xffffffffu, big);
+    while (bm) {
+      const int src = __ffs(bm) - 1;
+      bm &= bm - 1;
+      const int bd = __shfl_sync(0xffffffffu, d, src);
+      const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
+      const int64_t bps = __shfl_sync(0xffffffffu, ps, src);
+      for (int base = 0; base < bd; base += 32 * kLong) {  // kLong positions per lane in flight
+        IdxT e[kLong], p[kLong];
+        unsigned ok = 0;
+#pragma unroll
+        for (int u = 0; u < kLong; ++u) {
+          const int t = base + lane + 32 * u;
+          e[u] = (IdxT)(brs + t);
+          p[u] = (IdxT)(bps + t);
+          if (t < bd) ok |= 1u << u;
+        }
+        sink(e, p, ok);
+      }
+    }
+    // the window reaches the chunk end (or the last member): done
+    if (__any_sync(0xffffffffu, mp1 >= Pend)) break;
+    i += 32;
+  }
+}
+
 
 // A warp-tier work item, self-contained so a warp goes straight to its data:
 // entries [base, base + n) of the staging (PIECE: sc_col/sc_wgt) or of the
@@ -311,8 +318,8 @@ struct RowsArgs {
   int64_t *row_ptr_c;
   int32_t *col_c, *wgt_c, *vwgt_c;
   int *err;
-  long long *trace;  // debug: per block (compute cycles, 0, kind, T); nullable
-  unsigned long long *pstats;  // debug (HEC_PIECE_STATS): warp items / entries per kind x size class; nullable
+  const int64_t *mstart;  // row_ptr[members[i]]: rank items walk their member rows (x2_walk)
+  bool idx32;             // entry / position indices of the walks fit 32 bits (nnz < 2^32)
   const int32_t *list;    // blocks of this launch (a tier list)
   const WorkItem *items;  // warp tier: the same, as work items
   const RbmItem *ritems;  // bitmap-rank / hash-rank tier (one size class per launch)

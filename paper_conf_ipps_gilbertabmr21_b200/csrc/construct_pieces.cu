@@ -471,11 +471,6 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
       src_b = A.pb_g;
       src_w = A.pw_g;
     }
-    if (A.pstats && lane == 0) {
-      const int c = (R > 0 ? 4 : 0) + (n <= 32 ? 0 : n <= 64 ? 1 : n <= 128 ? 2 : 3);
-      atomicAdd(A.pstats + 2 * c, 1ull);
-      atomicAdd(A.pstats + 2 * c + 1, (unsigned long long)n);
-    }
     int T;
     if (R == 0) {
       if (n <= 32) T = group_run<1>(W, n, src_b, src_w, base);

@@ -45,7 +45,6 @@ struct RowsSmemT {
   float bscale[kMaxRows];
   int32_t tmp[40];
   unsigned long long wtot;
-  long long tx[2];  // trace: expansion / hashing cycles
   int32_t blk;
 };
 
@@ -105,7 +104,6 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
     const int64_t bi = S.blk;
     if (bi < 0) return;
     const BlockDesc d = A.blk[bi];
-    const long long c0 = A.trace ? clock64() : 0;
     int T = 0, R = 1;
     if (d.kind == B_DENSE) {
       // key chunk [k0, k0 + kCap) of a dense row, already in key order
@@ -212,7 +210,6 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
         __syncthreads();
         continue;
       }
-      const long long c_exp = A.trace ? clock64() : 0;
       int32_t ks[kIt];  // owned slot or -1
 #pragma unroll
       for (int k = 0; k < kIt; ++k) {
@@ -241,7 +238,6 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
       }
       __syncthreads();
       T = smem_exclusive_scan(S.ucnt, R, S.tmp);
-      if (A.trace && t == 0) { S.tx[0] = c_exp - c0; S.tx[1] = clock64() - c_exp; }
       if (t == 0) S.ucnt[R] = T;
       // ---- 3. owned keys: key range per row, buckets, ranks
 #pragma unroll
@@ -297,7 +293,6 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
     }
     __syncthreads();
     // ---- 4. stage the block's sorted distinct entries; k_place moves them
-    const long long c1 = A.trace ? clock64() : 0;
     if (rows_kind(d.kind)) {
       const int64_t P0 = S.mptr[0] - L.upos(L.a_lo);  // staging covers the active rows only
       for (int q = t; q < T; q += kT) {
@@ -327,16 +322,7 @@ __global__ void __launch_bounds__(kT, 2) k_rows(RowsArgs A) {
         }
       }
     }
-    if (t == 0) {
-      A.blk_cnt[bi] = T;
-      if (A.trace) {
-        A.trace[4 * bi] = c1 - c0;
-        // expansion cycles << 32 | hashing cycles (0 for DENSE / fallback blocks)
-        A.trace[4 * bi + 1] = d.kind == B_DENSE ? 0 : (S.tx[0] << 32) | (S.tx[1] & 0xffffffff);
-        A.trace[4 * bi + 2] = d.kind * 100000 + (rows_kind(d.kind) ? R : d.sub);
-        A.trace[4 * bi + 3] = T;
-      }
-    }
+    if (t == 0) A.blk_cnt[bi] = T;
     __syncthreads();
   }
 }

@@ -89,9 +89,6 @@ struct hec_ctx {
   hec::Arena ws;   // per-call workspace (reserved up front)
   hec::Arena ws2;  // construction skew-path workspace (sized after classification)
   int64_t *h_pinned = nullptr;  // pinned host scalars for D2H reads
-  // second stream for construction work that overlaps the skewed-row partition
-  cudaStream_t aux = nullptr;
-  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   hec_stats stats{};
   // state carried between hec_build_rows_count and hec_build_rows_write
   struct DistState *dist = nullptr;

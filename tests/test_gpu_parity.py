@@ -255,19 +255,19 @@ def test_construct_random_labels(P, ctx):
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["rbm", "bins", "staged"])
+@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index"])
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
 def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     """R-MAT with random labels into nc aggregates: few labels give huge rows
     (DENSE when nc <= 32768, key-range buckets otherwise), many labels give
     warp-piece and CTA-window rows.  path=bins forces the key-range bin pieces
-    instead of the bitmap-rank items (HEC_NO_RBM test hook)."""
+    instead of the bitmap-rank items (HEC_NO_RBM test hook); path=wide_index
+    runs the member walks with 64-bit entry indices (the nnz >= 2^32 build,
+    HEC_FORCE_WIDE_INDEX test hook)."""
     if path == "bins":  # DENSE levels: small rows through the k_rows blocks instead of rank items
         monkeypatch.setenv("HEC_NO_RBM", "1")
-    if path == "staged":  # DENSE rows through the staging (v1) instead of the fused expansion
-        if nc > 32768:
-            pytest.skip("BUCKET mode: no DENSE rows")
-        monkeypatch.setenv("HEC_DENSE_STAGED", "1")
+    if path == "wide_index":
+        monkeypatch.setenv("HEC_FORCE_WIDE_INDEX", "1")
     rng = np.random.default_rng(15 + nc)
     g = gg.rmat(14 if nc < 20000 else 17, 16)
     g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
@@ -326,7 +326,7 @@ def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
 
 
 @pytest.mark.parametrize("hot", [False, True])
-@pytest.mark.parametrize("path", ["direct", "hash", "overlap"])
+@pytest.mark.parametrize("path", ["direct", "hash"])
 def test_construct_direct_bins(P, ctx, path, hot, monkeypatch):
     """A hub row of 100k entries whose keys fall in [1, 3001): its key-range
     bins are narrow (<= 4096 keys) and hold ~25k entries each, so they take the
@@ -334,8 +334,6 @@ def test_construct_direct_bins(P, ctx, path, hot, monkeypatch):
     the hash-rank kernels (HEC_NO_DRANK test hook)."""
     if path == "hash":
         monkeypatch.setenv("HEC_NO_DRANK", "1")
-    if path == "overlap":  # whole rows on the second stream during the partition (HEC_OVERLAP)
-        monkeypatch.setenv("HEC_OVERLAP", "1")
     rng = np.random.default_rng(24)
     n, nc = 150000, 40000
     # hot: the hub's 100k entries fall on 30 keys (whole warps of equal keys,
@@ -385,12 +383,9 @@ def test_construct_rbm_rank_windows(P, ctx):
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("staged", [False, True])
-def test_construct_dense_row_overflow(P, ctx, staged, monkeypatch):
+def test_construct_dense_row_overflow(P, ctx):
     """A DENSE skewed row (a hub whose 6000 leaves collapse onto one coarse
     vertex): a coarse weight above INT32_MAX is reported, one just below is exact."""
-    if staged:
-        monkeypatch.setenv("HEC_DENSE_STAGED", "1")
     n = 6001
     M = np.ones(n, np.int32)
     M[0] = 0
