@@ -263,9 +263,12 @@ __global__ void k_seg_fill(int64_t nseg, const int64_t *__restrict__ ptr, int32_
 constexpr int kXT = 256;       // threads per CTA
 constexpr int kXChunk = 4096;  // positions per warp task
 
-// Expansion (k_expand2): the rows no other kernel walks itself (warp pieces,
-// the SMALL / bin-piece blocks of the HEC_NO_RBM path) are staged once in
-// member-edge space by x2_walk (construct_common.cuh).
+// Expansion (k_expand2): every entry of the rows not walked by the DENSE
+// accumulation is staged once, as (b = M[v], w), in member-edge space by
+// x2_walk (construct_common.cuh): the partition, rank and piece kernels then
+// read coalesced runs.  (Walking the member rows inside those kernels instead
+// was measured 1.4x slower on C4: the walk's M[v] gathers need this kernel's
+// occupancy to hide their latency.)
 // sink of the expansion: (M[v], w) to the staging at position - P_lo
 struct StageSink {
   const Layout &L;
@@ -320,8 +323,7 @@ struct PartArgs {
   const int64_t *unit_ptr;  // units of kUnit positions
   const int32_t *unit_row;  // unit -> big row index
   const int64_t *bkt_ptr;
-  const int32_t *Sb, *Sw;   // expanded entries, indexed from upos(a_lo) (k_part_warp rows only)
-  const int64_t *mstart;    // row_ptr[members[i]] (unit passes walk the member rows)
+  const int32_t *Sb, *Sw;   // expanded entries, indexed from upos(a_lo)
 };
 
 struct UnitInfo {
@@ -368,108 +370,68 @@ __device__ __forceinline__ int entry_bucket(const UnitInfo &u, int32_t b) {
 // passes are bound by per-unit latency, not by same-address replays.)
 __device__ __forceinline__ int agg_add(int32_t *ctr, int bk) { return bk < 0 ? -1 : atomicAdd(ctr + bk, 1); }
 
-// The unit passes read the member rows themselves (col / wgt streamed once per
-// pass, b = M[v] gathered): a CTA's 16 warps each walk 1/16 of the unit's
-// member-edge positions with x2_walk (no expansion staging for these rows).
-constexpr int kPartSlice = kUnit / (kT / 32);
-
-__device__ __forceinline__ void unit_slice(const UnitInfo &u, int64_t P_lo, int64_t &Pw, int64_t &Pwe) {
-  const int wid = threadIdx.x >> 5;
-  Pw = P_lo + u.p0 + (int64_t)wid * kPartSlice;
-  Pwe = P_lo + u.p1;
-  if (Pw + kPartSlice < Pwe) Pwe = Pw + kPartSlice;
+// histogram of the unit's entries (self entries dropped) into S.hist
+__device__ __forceinline__ void unit_hist(const PartArgs &A, const UnitInfo &u, PartSmem &S) {
+  for (int i = threadIdx.x; i < u.nb; i += kT) S.hist[i] = 0;
+  __syncthreads();
+  const int32_t *Sb = A.Sb + u.p0;
+  const int cnt = (int)(u.p1 - u.p0);  // <= kUnit
+  // warp-uniform trip count: agg_add's __match_any_sync needs every lane
+  for (int p = threadIdx.x; p - (int)(threadIdx.x & 31) < cnt; p += kPartU * kT) {
+    int32_t b[kPartU];
+#pragma unroll
+    for (int j = 0; j < kPartU; ++j) b[j] = p + j * kT < cnt ? __ldcs(Sb + p + j * kT) : u.a;
+#pragma unroll
+    for (int j = 0; j < kPartU; ++j) agg_add(S.hist, entry_bucket(u, b[j]));
+  }
+  __syncthreads();
 }
-
-// count pass: bucket of every entry (self entries dropped) into hist
-struct PartCountSink {
-  const Layout &L;
-  const UnitInfo &u;
-  int32_t *hist;
-  template <int N, typename IdxT>
-  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
-    (void)p;
-    int32_t b[N];
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) b[q] = __ldcs(L.col + e[q]);
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) b[q] = __ldg(L.M + b[q]);
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) agg_add(hist, entry_bucket(u, b[q]));
-  }
-};
-
-// write pass: (b, w) to the entry's slot of its bin (shared-memory cursors)
-struct PartWriteSink {
-  const Layout &L;
-  const UnitInfo &u;
-  int32_t *cursor;
-  int32_t *__restrict__ pbr, *__restrict__ pwr;
-  template <int N, typename IdxT>
-  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
-    (void)p;
-    int32_t b[N], w[N];
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) { b[q] = __ldcs(L.col + e[q]); w[q] = __ldcs(L.wgt + e[q]); }
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) b[q] = __ldg(L.M + b[q]);
-#pragma unroll
-    for (int q = 0; q < N; ++q) {
-      if (!(ok & (1u << q))) continue;
-      const int slot = agg_add(cursor, entry_bucket(u, b[q]));
-      if (slot >= 0) {
-        pbr[slot] = b[q];
-        pwr[slot] = w[q];
-      }
-    }
-  }
-};
 
 // The unit's slice of each bin is reserved here: the returned running count
 // is the unit's offset inside the bin (ubase), so the write pass needs no
 // second histogram.
-template <typename IdxT>
 __global__ void __launch_bounds__(kT) k_part_count(PartArgs A, unsigned *__restrict__ bkt_cnt,
                                                    int32_t *__restrict__ ubase) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   const UnitInfo u = unit_info(A, blockIdx.x);
-  const Layout &L = A.L;
-  for (int i = threadIdx.x; i < u.nb; i += kT) S.hist[i] = 0;
-  __syncthreads();
-  int64_t Pw, Pwe;
-  unit_slice(u, L.upos(L.a_lo), Pw, Pwe);
-  PartCountSink sink{L, u, S.hist};
-  if (Pw < Pwe) x2_walk<8, PartCountSink, 4, IdxT>(L, A.mstart, L.member_ptr[u.a], L.member_ptr[u.a + 1], Pw, Pwe,
-                                                  nullptr, sink);
-  __syncthreads();
+  unit_hist(A, u, S);
   int32_t *ub = ubase + (int64_t)blockIdx.x * kPartHist;
   for (int i = threadIdx.x; i < u.nb; i += kT)
     if (S.hist[i]) ub[i] = (int32_t)atomicAdd(bkt_cnt + u.b0 + i, (unsigned)S.hist[i]);
 }
 
-template <typename IdxT>
 __global__ void __launch_bounds__(kT) k_part_write(PartArgs A, const int64_t *__restrict__ bkt_off,
                                                    const int32_t *__restrict__ ubase, int32_t *__restrict__ pb,
                                                    int32_t *__restrict__ pw) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PartSmem &S = *reinterpret_cast<PartSmem *>(smem_raw);
   const UnitInfo u = unit_info(A, blockIdx.x);
-  const Layout &L = A.L;
   const int64_t off0 = bkt_off[u.b0];
   const int32_t *ub = ubase + (int64_t)blockIdx.x * kPartHist;
   for (int i = threadIdx.x; i < u.nb; i += kT)  // (slots of bins the unit never hits stay unused)
     S.base[i] = (int32_t)(bkt_off[u.b0 + i] - off0) + ub[i];
   __syncthreads();
-  int64_t Pw, Pwe;
-  unit_slice(u, L.upos(L.a_lo), Pw, Pwe);
-  PartWriteSink sink{L, u, S.base, pb + off0, pw + off0};
-  if (Pw < Pwe) x2_walk<8, PartWriteSink, 4, IdxT>(L, A.mstart, L.member_ptr[u.a], L.member_ptr[u.a + 1], Pw, Pwe,
-                                                  nullptr, sink);
+  const int32_t *Sb = A.Sb + u.p0, *Sw = A.Sw + u.p0;
+  int32_t *pbr = pb + off0, *pwr = pw + off0;
+  const int cnt = (int)(u.p1 - u.p0);
+  for (int p = threadIdx.x; p - (int)(threadIdx.x & 31) < cnt; p += kPartU * kT) {
+    int32_t b[kPartU], w[kPartU];
+#pragma unroll
+    for (int j = 0; j < kPartU; ++j) {
+      const bool in = p + j * kT < cnt;
+      b[j] = in ? __ldcs(Sb + p + j * kT) : u.a;
+      w[j] = in ? __ldcs(Sw + p + j * kT) : 0;
+    }
+#pragma unroll
+    for (int j = 0; j < kPartU; ++j) {
+      const int q = agg_add(S.base, entry_bucket(u, b[j]));
+      if (q >= 0) {
+        pbr[q] = b[j];
+        pwr[q] = w[j];
+      }
+    }
+  }
 }
 
 // Skewed rows with U <= kWarpRowMax (<= kWarpBins bins): one warp counts the
@@ -1109,11 +1071,10 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     int64_t grid = (warps + kXT / 32 - 1) / (kXT / 32);
     const int64_t cap = (int64_t)ctx->num_sms * 8;
     if (grid > cap) grid = cap;
-    // rank items (rbm: every row above kPieceMax), rows partitioned by CTA
-    // units (U > kWarpRowMax) and fused DENSE rows are walked by their own
-    // kernels: the staging covers the other rows only
-    const int32_t *skip = rbm ? nullptr : big_idx;
-    const int64_t skip_thr = rbm ? (int64_t)kPieceMax : dense ? 0 : kWarpRowMax;
+    // DENSE rows are walked by their accumulation kernel (k_dense_accum2);
+    // everything else is staged once here
+    const int32_t *skip = dense ? big_idx : nullptr;
+    const int64_t skip_thr = dense ? 0 : INT64_MAX;
     if (grid > 0) {
       if (idx32)
         k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr);
@@ -1147,13 +1108,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
 
   static bool attr = false;
   if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(PartSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(PartSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count<int64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(PartSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write<int64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(PartSmem)));
     HEC_CUDA_TRY(cudaFuncSetAttribute(k_bucket_fallback, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)sizeof(FbSmem)));
@@ -1201,15 +1158,13 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     int64_t *prow = arena_take<int64_t>(W2, nbig + 1);
     if (!prow) { set_error("workspace under-reserved (prow)"); return HEC_EINVAL; }
     HEC_TRY(chained_scan(ctx, nbig, RowUIn{L, big_list}, PtrOut{prow}, stb, prow + nbig));
-    PartArgs PA{L, big_list, nbig, unit_ptr, unit_row, bkt_ptr, sc_col, sc_wgt, mstart};
+    PartArgs PA{L, big_list, nbig, unit_ptr, unit_row, bkt_ptr, sc_col, sc_wgt};
     if (nunits > 0) {  // rows above kWarpRowMax: CTA units count, per-row scan, scatter
-      if (idx32) k_part_count<uint32_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
-      else k_part_count<int64_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
+      k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
       HEC_LAUNCH_CHECK();
       k_row_bins<<<nblk(nbig * 32, 256), 256, 0, s>>>(PA, prow, bkt_cnt, bkt_off);
       HEC_LAUNCH_CHECK();
-      if (idx32) k_part_write<uint32_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, ubase, pb, pw);
-      else k_part_write<int64_t><<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, ubase, pb, pw);
+      k_part_write<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_off, ubase, pb, pw);
       HEC_LAUNCH_CHECK();
     }
     k_part_warp<<<nblk(nbig * 32, kPWT), kPWT, 0, s>>>(PA, prow, bkt_off, bkt_cnt, pb, pw);
