@@ -76,8 +76,31 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   return total;
 }
 
-template <int NT, int PER = 8>
-__global__ void __launch_bounds__(NT, PER == 8 ? 1024 / NT : 4) k_hrank(RowsArgs A) {
+// Whole-row items read their member rows themselves: warp w walks the row's
+// member-edge positions [32 PER w, 32 PER (w + 1)) (x2_walk: col / wgt streamed,
+// b = M[v] gathered) into its own slice of the value table, then takes its
+// registers from there -- no expansion staging in HBM for these rows.
+struct SmemStageSink {
+  const Layout &L;
+  int2 *stage;
+  int64_t Pw;
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
+    int32_t b[N], w[N];
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) { b[q] = __ldcs(L.col + e[q]); w[q] = __ldcs(L.wgt + e[q]); }
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) b[q] = __ldg(L.M + b[q]);
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+      if (ok & (1u << q)) stage[(int64_t)p[q] - Pw] = make_int2(b[q], w[q]);
+  }
+};
+
+template <int NT, int PER = 8, typename IdxT = uint32_t>
+__global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4) k_hrank(RowsArgs A) {
   constexpr int kCapE = HrSmem<NT, PER>::kCapE;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   HrSmem<NT, PER> &S = *reinterpret_cast<HrSmem<NT, PER> *>(smem_raw);
@@ -107,57 +130,68 @@ __global__ void __launch_bounds__(NT, PER == 8 ? 1024 / NT : 4) k_hrank(RowsArgs
     // any positive scale keeps the buckets monotone in b (approximate division)
     const float scale = __fdividef((float)NB, (float)(it.hi - lo));
     int32_t kb[PER], kw[PER];
+    if (it.bk >= 0) {  // key-range bin: partitioned pairs
 #pragma unroll
-    for (int k = 0; k < PER; ++k) {
-      const int i = t + NT * k;
-      kb[k] = -1;
-      kw[k] = 0;
-      if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+      for (int k = 0; k < PER; ++k) {
+        const int i = t + NT * k;
+        kb[k] = -1;
+        kw[k] = 0;
+        if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+      }
+    } else {  // whole row: fused member walk into the warp's slice of val
+      const int lane = t & 31, wid = t >> 5;
+      const int base = wid * 32 * PER;
+      int2 *stage = reinterpret_cast<int2 *>(S.val) + base;
+      const int64_t Pw = A.L.upos(A.L.a_lo) + it.src + base;
+      const int64_t Pwe = Pw + (n - base < 32 * PER ? n - base : 32 * PER);
+      if (Pw < Pwe) {
+        SmemStageSink sink{A.L, stage, Pw};
+        x2_walk<4, SmemStageSink, 4, IdxT>(A.L, A.mstart, A.L.member_ptr[a], A.L.member_ptr[a + 1], Pw, Pwe, nullptr,
+                                          sink);
+      }
+      __syncwarp();
+#pragma unroll
+      for (int k = 0; k < PER; ++k) {
+        const int i = lane + 32 * k;
+        kb[k] = -1;
+        kw[k] = 0;
+        if (base + i < n) {
+          const int2 v = stage[i];
+          kb[k] = v.x;
+          kw[k] = v.y;
+        }
+      }
+      __syncwarp();
+#pragma unroll
+      for (int k = 0; k < PER; ++k) stage[lane + 32 * k] = make_int2(0, 0);  // val is zero between items
+      __syncthreads();
     }
     // ---- 1. hash merge; owners count their bucket (keys lie in [lo, hi) by
     // construction of the items: whole rows span [0, n_c), bins their range)
-    // The PER first probes are issued back to back (independent CASes), so a
-    // thread waits for one round trip, not PER; collisions (load <= 1/2) are
-    // then resolved per entry, and the weight / bucket adds are issued
-    // together as well.
     bool wrap = false;
     int slot[PER], bpos[PER];
-    int32_t old[PER];
     unsigned own = 0;
 #pragma unroll
     for (int k = 0; k < PER; ++k) {
       if (kb[k] == a) kb[k] = -1;  // self entry (L280)
-      slot[k] = (int)((hr_hash(kb[k]) >> hshift) & hmask);
-    }
-#pragma unroll
-    for (int k = 0; k < PER; ++k) old[k] = kb[k] >= 0 ? atomicCAS(&S.key[slot[k]], kEmpty, kb[k]) : kEmpty;
-#pragma unroll
-    for (int k = 0; k < PER; ++k) {
       if (kb[k] < 0) continue;
-      uint32_t h = (uint32_t)slot[k];
-      int32_t o = old[k];
-      while (o != kEmpty && o != kb[k]) {
+      uint32_t h = (hr_hash(kb[k]) >> hshift) & hmask;
+      while (true) {
+        const int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
+        if (old == kEmpty) { own |= 1u << k; break; }
+        if (old == kb[k]) break;
         h = (h + 1) & hmask;
-        o = atomicCAS(&S.key[h], kEmpty, kb[k]);
       }
-      if (o == kEmpty) own |= 1u << k;
       slot[k] = (int)h;
+      const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
+      wrap |= o + (uint32_t)kw[k] < o;
+      if (own & (1u << k)) {
+        int bk = (int)__fmul_rz((float)(kb[k] - lo), scale);
+        bk = bk < NB - 1 ? bk : NB - 1;
+        bpos[k] = atomicAdd(&S.cnt[bk], 1);
+        slot[k] |= bk << 16;  // slot < 2^14, bucket < 2^13
+      }
     }
-    uint32_t prev[PER];
-#pragma unroll
-    for (int k = 0; k < PER; ++k)
-      if (kb[k] >= 0) prev[k] = atomicAdd(&S.val[slot[k]], (uint32_t)kw[k]);
-#pragma unroll
-    for (int k = 0; k < PER; ++k) {
-      if (!(own & (1u << k))) continue;
-      int bk = (int)__fmul_rz((float)(kb[k] - lo), scale);
-      bk = bk < NB - 1 ? bk : NB - 1;
-      bpos[k] = atomicAdd(&S.cnt[bk], 1);
-      slot[k] |= bk << 16;  // slot < 2^14, bucket < 2^13
-    }
-#pragma unroll
-    for (int k = 0; k < PER; ++k)
-      if (kb[k] >= 0) wrap |= prev[k] + (uint32_t)kw[k] < prev[k];
     if (wrap) atomicOr(err, ERR_OVERFLOW);
     __syncthreads();
     // ---- 2. bucket offsets; owners place their key in bucket order
@@ -419,19 +453,24 @@ int launch_drank(hec_ctx *ctx, const RowsArgs &A) {
   return HEC_OK;
 }
 
-template <int NT>
+template <int NT, typename IdxT>
 static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
+  static_assert(sizeof(HrSmem<NT>::val) >= sizeof(int2) * HrSmem<NT>::kCapE, "walk staging fits in val");
   const size_t smem = sizeof(HrSmem<NT>);
-  HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank<NT, 8, IdxT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 1;
-  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_hrank<NT>, NT, smem));
+  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_hrank<NT, 8, IdxT>, NT, smem));
   if (occ < 1) occ = 1;
   int64_t grid = (int64_t)ctx->num_sms * occ;
   if (A.nblocks < grid) grid = A.nblocks;
   if (grid < 1) return HEC_OK;
-  k_hrank<NT><<<(unsigned)grid, NT, smem, ctx->stream>>>(A);
+  k_hrank<NT, 8, IdxT><<<(unsigned)grid, NT, smem, ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
+}
+template <int NT>
+static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
+  return A.idx32 ? launch_hrank_t<NT, uint32_t>(ctx, A) : launch_hrank_t<NT, int64_t>(ctx, A);
 }
 
 // One size class of items (the list in A.ritems / A.nlist): cls -1, 0, 1, 2 =
