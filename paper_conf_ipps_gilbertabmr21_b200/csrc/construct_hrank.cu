@@ -76,30 +76,7 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   return total;
 }
 
-// Whole-row items read their member rows themselves: warp w walks the row's
-// member-edge positions [32 PER w, 32 PER (w + 1)) (x2_walk: col / wgt streamed,
-// b = M[v] gathered) into its own slice of the value table, then takes its
-// registers from there -- no expansion staging in HBM for these rows.
-struct SmemStageSink {
-  const Layout &L;
-  int2 *stage;
-  int64_t Pw;
-  template <int N, typename IdxT>
-  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
-    int32_t b[N], w[N];
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) { b[q] = __ldcs(L.col + e[q]); w[q] = __ldcs(L.wgt + e[q]); }
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) b[q] = __ldg(L.M + b[q]);
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-      if (ok & (1u << q)) stage[(int64_t)p[q] - Pw] = make_int2(b[q], w[q]);
-  }
-};
-
-template <int NT, int PER = 8, typename IdxT = uint32_t>
+template <int NT, int PER = 8>
 __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4) k_hrank(RowsArgs A) {
   constexpr int kCapE = HrSmem<NT, PER>::kCapE;
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -130,41 +107,12 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     // any positive scale keeps the buckets monotone in b (approximate division)
     const float scale = __fdividef((float)NB, (float)(it.hi - lo));
     int32_t kb[PER], kw[PER];
-    if (it.bk >= 0) {  // key-range bin: partitioned pairs
 #pragma unroll
-      for (int k = 0; k < PER; ++k) {
-        const int i = t + NT * k;
-        kb[k] = -1;
-        kw[k] = 0;
-        if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
-      }
-    } else {  // whole row: fused member walk into the warp's slice of val
-      const int lane = t & 31, wid = t >> 5;
-      const int base = wid * 32 * PER;
-      int2 *stage = reinterpret_cast<int2 *>(S.val) + base;
-      const int64_t Pw = A.L.upos(A.L.a_lo) + it.src + base;
-      const int64_t Pwe = Pw + (n - base < 32 * PER ? n - base : 32 * PER);
-      if (Pw < Pwe) {
-        SmemStageSink sink{A.L, stage, Pw};
-        x2_walk<4, SmemStageSink, 4, IdxT>(A.L, A.mstart, A.L.member_ptr[a], A.L.member_ptr[a + 1], Pw, Pwe, nullptr,
-                                          sink);
-      }
-      __syncwarp();
-#pragma unroll
-      for (int k = 0; k < PER; ++k) {
-        const int i = lane + 32 * k;
-        kb[k] = -1;
-        kw[k] = 0;
-        if (base + i < n) {
-          const int2 v = stage[i];
-          kb[k] = v.x;
-          kw[k] = v.y;
-        }
-      }
-      __syncwarp();
-#pragma unroll
-      for (int k = 0; k < PER; ++k) stage[lane + 32 * k] = make_int2(0, 0);  // val is zero between items
-      __syncthreads();
+    for (int k = 0; k < PER; ++k) {
+      const int i = t + NT * k;
+      kb[k] = -1;
+      kw[k] = 0;
+      if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
     }
     // ---- 1. hash merge; owners count their bucket (keys lie in [lo, hi) by
     // construction of the items: whole rows span [0, n_c), bins their range)
@@ -453,24 +401,23 @@ int launch_drank(hec_ctx *ctx, const RowsArgs &A) {
   return HEC_OK;
 }
 
-template <int NT, typename IdxT>
+template <int NT, int PER = 8>
 static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
-  static_assert(sizeof(HrSmem<NT>::val) >= sizeof(int2) * HrSmem<NT>::kCapE, "walk staging fits in val");
-  const size_t smem = sizeof(HrSmem<NT>);
-  HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank<NT, 8, IdxT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int occ = 1;
-  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_hrank<NT, 8, IdxT>, NT, smem));
-  if (occ < 1) occ = 1;
+  static bool attr = false;
+  static int occ = 1;
+  const size_t smem = sizeof(HrSmem<NT, PER>);
+  if (!attr) {
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank<NT, PER>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_hrank<NT, PER>, NT, smem));
+    if (occ < 1) occ = 1;
+    attr = true;
+  }
   int64_t grid = (int64_t)ctx->num_sms * occ;
   if (A.nblocks < grid) grid = A.nblocks;
   if (grid < 1) return HEC_OK;
-  k_hrank<NT, 8, IdxT><<<(unsigned)grid, NT, smem, ctx->stream>>>(A);
+  k_hrank<NT, PER><<<(unsigned)grid, NT, smem, ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
-}
-template <int NT>
-static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
-  return A.idx32 ? launch_hrank_t<NT, uint32_t>(ctx, A) : launch_hrank_t<NT, int64_t>(ctx, A);
 }
 
 // One size class of items (the list in A.ritems / A.nlist): cls -1, 0, 1, 2 =
