@@ -35,3 +35,10 @@ clean:
 	rm -rf build graphgen/libgraphgen.so oracle/liboracle.so $(PKG)/libhec.so
 
 .PHONY: all graphgen oracle hec clean
+
+# A/B variants for timing experiments: make variant V=name VFLAGS="-DFOO=1"
+# -> build/variants/<name>/libhec.so (load with HEC_LIB_PATH)
+variant:
+	@mkdir -p build/variants/$(V)
+	$(NVCC) $(NVFLAGS) $(VFLAGS) -shared -o build/variants/$(V)/libhec.so $(CU_SRC) -lcudart
+.PHONY: variant

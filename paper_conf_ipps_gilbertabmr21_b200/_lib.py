@@ -5,7 +5,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhec.so")
+# HEC_LIB_PATH: an alternative build of libhec.so (A/B timing of kernel variants)
+LIB_PATH = os.environ.get("HEC_LIB_PATH") or os.path.join(_HERE, "libhec.so")
 
 HEC_OK, HEC_EINVAL, HEC_ENOMEM, HEC_ECUDA, HEC_EOVERFLOW = 0, -1, -2, -3, -4
 STOP_CUTOFF, STOP_DISCARD, STOP_STALL, STOP_MAX_LEVELS = 0, 1, 2, 3

@@ -151,8 +151,8 @@ __global__ void k_big_rows(Layout L, int64_t big_thr, int32_t *__restrict__ big_
 constexpr int kPartHist = 8192;  // buckets per skewed row (bounds the partition's smem tables)
 constexpr int kUnit = 32768;     // member-edge positions per partition CTA
 
-__host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c, bool rbm = false) {
-  const int64_t avg = rbm ? kRbmBinAvg : kBucketAvg;
+__host__ __device__ __forceinline__ int64_t row_buckets(int64_t U, int64_t n_c, bool rbm, int64_t bin_avg) {
+  const int64_t avg = rbm ? bin_avg : kBucketAvg;
   int64_t nb = (U + avg - 1) / avg;
   // rows holding >= 1/16 of the key range in entries: bins no wider than
   // kDirectR keys (>= 256 entries each on average) for the direct-indexed kernel
@@ -179,7 +179,7 @@ struct BlockCountIn {
     if (!L.active(a)) return 0;
     const int64_t U = L.U(a);
     const int c = cls(U);
-    if (c == 2) return dense ? dense_chunks(L.n_c) : row_buckets(U, L.n_c, rbm);
+    if (c == 2) return dense ? dense_chunks(L.n_c) : row_buckets(U, L.n_c, rbm, L.bin_avg);
     if (c == 1 && rbm) return 1;
     if (a == L.a_lo || cls(L.U(a - 1)) != c) return 1;
     const int64_t win = c == 0 ? kPieceWin : kWin;  // rows of one class are contiguous in S
@@ -242,7 +242,9 @@ struct BucketsIn {
   Layout L;
   const int32_t *big_list;
   bool rbm;
-  __device__ __forceinline__ int64_t operator()(int64_t h) const { return row_buckets(L.U(big_list[h]), L.n_c, rbm); }
+  __device__ __forceinline__ int64_t operator()(int64_t h) const {
+    return row_buckets(L.U(big_list[h]), L.n_c, rbm, L.bin_avg);
+  }
 };
 
 // Segment -> owner table: out[k] = h for k in [ptr[h], ptr[h+1]) (a warp per
@@ -987,7 +989,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // 32-bit entry / position indices in the member walks when nnz < 2^32
   // (HEC_FORCE_WIDE_INDEX: test hook for the 64-bit instantiation)
   const bool idx32 = g->nnz < ((int64_t)1 << 32) && getenv("HEC_FORCE_WIDE_INDEX") == nullptr;
-  Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi};
+  Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi, kRbmBinAvg};
+  if (const char *e = getenv("HEC_TUNE_BINAVG")) L.bin_avg = atoll(e);  // (tuning experiment)
   const bool dense = n_c <= kDenseMax;
   // bitmap-rank items replace the bin pieces when the key range fits the
   // shared-memory bitmap (HEC_NO_RBM: test / tuning hook for the bin-piece path)

@@ -21,14 +21,19 @@
 
 namespace hec {
 
+#ifndef HEC_BUCKET_SHIFT
+#define HEC_BUCKET_SHIFT 0
+#endif
+constexpr int kBucketShift = HEC_BUCKET_SHIFT;  // buckets per item: pow2(n) << kBucketShift
 template <int NT, int PER = 8>
 struct HrSmem {
   static constexpr int kCapE = NT * PER;     // entries per item
   static constexpr int kSlots = 2 * kCapE;   // hash slots (load <= 1/2)
+  static constexpr int kNB = kCapE << kBucketShift;  // max buckets
   int32_t key[kSlots];
   uint32_t val[kSlots];
-  int32_t cnt[kCapE + 1];                    // bucket counts (zeroed by the scan)
-  uint16_t offs[kCapE + 2];                  // bucket offsets (<= kCapE)
+  int32_t cnt[kNB + 1];                      // bucket counts (zeroed by the scan)
+  uint16_t offs[kNB + 2];                    // bucket offsets (<= kCapE)
   int32_t scr[kCapE];                        // distinct keys in bucket order
   int32_t wsum[NT / 32 + 1];
   int32_t nd;                                // distinct keys of the item
@@ -43,10 +48,10 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int per = (nb + NT - 1) / NT;
   const int beg = t * per;
-  int v[PER];
+  int v[PER << kBucketShift];
   int local = 0;
 #pragma unroll
-  for (int i = 0; i < PER; ++i) {
+  for (int i = 0; i < (PER << kBucketShift); ++i) {
     v[i] = 0;
     if (i < per && beg + i < nb) { v[i] = c[beg + i]; c[beg + i] = 0; }
     local += v[i];
@@ -68,7 +73,7 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   }
   int run = before + x - local;
 #pragma unroll
-  for (int i = 0; i < PER; ++i) {
+  for (int i = 0; i < (PER << kBucketShift); ++i) {
     if (i < per && beg + i < nb) o[beg + i] = (uint16_t)run;
     run += v[i];
   }
@@ -87,7 +92,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
   int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
   int *const err = A.err;
   for (int i = t; i < HrSmem<NT, PER>::kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
-  for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
+  for (int i = t; i <= HrSmem<NT, PER>::kNB; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
   __syncthreads();
   RbmItem nx{};
@@ -101,8 +106,8 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     int32_t *const src_w = (it.bk < 0 ? scw : pwg) + it.src;
     // table geometry: NB buckets (power of two >= n), 2 NB hash slots
     const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
-    const int NB = 1 << lg;
-    const uint32_t hmask = 2u * NB - 1u;
+    const int NB = 1 << (lg + kBucketShift);
+    const uint32_t hmask = (2u << lg) - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
     // any positive scale keeps the buckets monotone in b (approximate division)
     const float scale = __fdividef((float)NB, (float)(it.hi - lo));
