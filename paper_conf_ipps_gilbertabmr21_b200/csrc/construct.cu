@@ -1060,6 +1060,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   RbmItem *list_redo = arena_take<RbmItem>(W2, nblocks + 1);  // n > 4096 items left to k_rbm
   RbmItem *list_d = arena_take<RbmItem>(W2, nblocks + 1);     // direct-indexed bins (k_drank)
   RbmItem *list_r3 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n <= kHrMaxS
+  RbmItem *list_mredo = arena_take<RbmItem>(W2, nblocks + 1);  // k_mrank items left to k_hrank
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1123,6 +1124,9 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
 
   const bool direct = getenv("HEC_NO_DRANK") == nullptr;  // test hook: bins through the hash-rank kernels
+  // rank items <= 4096 entries: order-preserving hash rank (HEC_NO_MRANK: the
+  // unordered hash + bucket rank k_hrank for all of them, test hook)
+  const bool use_mrank = getenv("HEC_NO_MRANK") == nullptr;
   int ph_rows = -1;
 
   // ---- a9 skewed rows
@@ -1242,7 +1246,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
       A.nlist = C.n;
       A.rdir = C.dir;
       if (c < 3) {
-        HEC_TRY(launch_hrank(ctx, A, c));
+        if (use_mrank) HEC_TRY(launch_mrank(ctx, A, c, list_mredo, counts + 19));
+        else HEC_TRY(launch_hrank(ctx, A, c));
       } else {
         HEC_TRY(launch_hrank_big(ctx, A, list_redo, counts + 17));
         A.ritems = list_redo;
@@ -1250,6 +1255,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
         A.rdir = 1;
         HEC_TRY(launch_rbm(ctx, A));
       }
+    }
+    if (use_mrank) {  // items whose keys crowded the order-preserving table
+      A.ritems = list_mredo;
+      A.nlist = counts + 19;
+      A.rdir = 1;
+      HEC_TRY(launch_hrank(ctx, A, 2));
     }
     A.ritems = list_d;
     A.nlist = counts + 18;

@@ -337,6 +337,8 @@ int launch_place(hec_ctx *ctx, const RowsArgs &A);
 int launch_rbm(hec_ctx *ctx, const RowsArgs &A);  // construct_rbm.cu
 int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls);  // construct_hrank.cu (cls -1..2: n <= 512/1024/2048/4096)
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo);  // n > 4096
+// order-preserving hash rank, classes as launch_hrank; overflowing items -> redo (k_hrank<512>)
+int launch_mrank(hec_ctx *ctx, const RowsArgs &A, int cls, RbmItem *redo, unsigned *nredo);
 int launch_drank(hec_ctx *ctx, const RowsArgs &A);  // bins with hi - lo <= kDirectR
 
 }  // namespace hec

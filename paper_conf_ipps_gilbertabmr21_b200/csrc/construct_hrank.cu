@@ -21,19 +21,14 @@
 
 namespace hec {
 
-#ifndef HEC_BUCKET_SHIFT
-#define HEC_BUCKET_SHIFT 0
-#endif
-constexpr int kBucketShift = HEC_BUCKET_SHIFT;  // buckets per item: pow2(n) << kBucketShift
 template <int NT, int PER = 8>
 struct HrSmem {
   static constexpr int kCapE = NT * PER;     // entries per item
   static constexpr int kSlots = 2 * kCapE;   // hash slots (load <= 1/2)
-  static constexpr int kNB = kCapE << kBucketShift;  // max buckets
   int32_t key[kSlots];
   uint32_t val[kSlots];
-  int32_t cnt[kNB + 1];                      // bucket counts (zeroed by the scan)
-  uint16_t offs[kNB + 2];                    // bucket offsets (<= kCapE)
+  int32_t cnt[kCapE + 1];                    // bucket counts (zeroed by the scan)
+  uint16_t offs[kCapE + 2];                  // bucket offsets (<= kCapE)
   int32_t scr[kCapE];                        // distinct keys in bucket order
   int32_t wsum[NT / 32 + 1];
   int32_t nd;                                // distinct keys of the item
@@ -48,10 +43,10 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int per = (nb + NT - 1) / NT;
   const int beg = t * per;
-  int v[PER << kBucketShift];
+  int v[PER];
   int local = 0;
 #pragma unroll
-  for (int i = 0; i < (PER << kBucketShift); ++i) {
+  for (int i = 0; i < PER; ++i) {
     v[i] = 0;
     if (i < per && beg + i < nb) { v[i] = c[beg + i]; c[beg + i] = 0; }
     local += v[i];
@@ -73,7 +68,7 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   }
   int run = before + x - local;
 #pragma unroll
-  for (int i = 0; i < (PER << kBucketShift); ++i) {
+  for (int i = 0; i < PER; ++i) {
     if (i < per && beg + i < nb) o[beg + i] = (uint16_t)run;
     run += v[i];
   }
@@ -92,7 +87,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
   int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
   int *const err = A.err;
   for (int i = t; i < HrSmem<NT, PER>::kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
-  for (int i = t; i <= HrSmem<NT, PER>::kNB; i += NT) S.cnt[i] = 0;
+  for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
   __syncthreads();
   RbmItem nx{};
@@ -106,8 +101,8 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     int32_t *const src_w = (it.bk < 0 ? scw : pwg) + it.src;
     // table geometry: NB buckets (power of two >= n), 2 NB hash slots
     const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
-    const int NB = 1 << (lg + kBucketShift);
-    const uint32_t hmask = (2u << lg) - 1u;
+    const int NB = 1 << lg;
+    const uint32_t hmask = 2u * NB - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
     // any positive scale keeps the buckets monotone in b (approximate division)
     const float scale = __fdividef((float)NB, (float)(it.hi - lo));
@@ -293,6 +288,179 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
     }
     __syncthreads();
   }
+}
+
+// ---------------------------------------------------------------------------
+// Order-preserving hash rank (k_mrank).  Same items as k_hrank, but the table
+// is indexed by a MONOTONE function of the key, h(b) = floor((b - lo) * S / W)
+// (W = hi - lo, S = 2 pow2(n) home slots) with linear probing forward, no
+// wrap-around, and probe distances bounded by kMaxProbe.  A key sits at or
+// after its home and at most d = (the item's largest probe distance) after
+// it, so for keys x at slot i and y at slot m:  m < i - d  =>  h(y) <= m <
+// i - d <= h(x)  =>  y < x  (h monotone), and symmetrically m > i + d => y >
+// x.  The output rank of x is therefore
+//   (occupied slots before i) - #{m in [i-d, i): y > x} + #{m in (i, i+d]: y < x},
+// one block scan of per-thread occupancy counts plus <= 2d comparisons per
+// key -- replacing k_hrank's bucket counts, scatter and in-bucket rank loop,
+// which its source profile put at ~45% of its instructions.  Items whose
+// probes exceed kMaxProbe or the table margin (keys crowded in a narrow part of
+// [lo, hi)) are left untouched and appended to a redo list for k_hrank.
+constexpr int kMaxProbe = 48;
+template <int NT, int PER = 8>
+struct MrSmem {
+  static constexpr int kCapE = NT * PER;
+  static constexpr int kQ = 2 * PER + 1;       // slots per thread in the sweep
+  static constexpr int kSlots = kQ * NT;       // 2 pow2(n) home slots + >= NT margin
+  int32_t key[kSlots + kMaxProbe];             // tail: permanently empty (rank window)
+  uint32_t val[kSlots];
+  int32_t wsum[NT / 32];
+  int32_t overflow, dmax;
+};
+
+template <int NT, int PER = 8>
+__global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__restrict__ redo,
+                                                         unsigned *__restrict__ nredo) {
+  using SM = MrSmem<NT, PER>;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  SM &S = *reinterpret_cast<SM *>(smem_raw);
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  const int64_t nitems = *A.nlist;
+  int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
+  for (int i = t; i < SM::kSlots + kMaxProbe; i += NT) S.key[i] = kEmpty;
+  for (int i = t; i < SM::kSlots; i += NT) S.val[i] = 0u;
+  if (t == 0) { S.overflow = 0; S.dmax = 0; }
+  __syncthreads();
+  RbmItem nx{};
+  if (blockIdx.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, blockIdx.x);
+  for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
+    const RbmItem it = nx;  // descriptor prefetched one item ahead
+    if (ii + gridDim.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, ii + gridDim.x);
+    const int n = it.n;
+    const int32_t a = it.row, lo = it.lo;
+    int32_t *const src_b = (it.bk < 0 ? scb : pbg) + it.src;
+    int32_t *const src_w = (it.bk < 0 ? scw : pwg) + it.src;
+    // geometry: Sh = 2 pow2(n) home slots; the sweep covers q slots per thread
+    const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
+    const int Sh = 2 << lg;
+    const int q = Sh / NT + 1;
+    const int Stot = q * NT;             // probes stay below Stot (margin >= 1 slot per thread)
+    const float scale = __fdividef((float)Sh, (float)(it.hi - lo));
+    int32_t kb[PER], kw[PER];
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int i = t + NT * k;
+      kb[k] = -1;
+      kw[k] = 0;
+      if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+    }
+    // ---- 1. insert at the monotone home slot, probing forward
+    bool wrap = false, over = false;
+    int dist = 0;
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      if (kb[k] == a) kb[k] = -1;  // self entry (L280)
+      if (kb[k] < 0) continue;
+      int h = (int)__fmul_rz((float)(kb[k] - lo), scale);
+      h = h < Sh - 1 ? h : Sh - 1;
+      const int home = h;
+      while (true) {
+        const int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
+        if (old == kEmpty || old == kb[k]) break;
+        if (++h >= Stot || h - home > kMaxProbe) { over = true; break; }
+      }
+      if (over) break;
+      dist = max(dist, h - home);
+      const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
+      wrap |= o + (uint32_t)kw[k] < o;
+    }
+    if (over) S.overflow = 1;
+    if (dist > 0) atomicMax(&S.dmax, dist);
+    if (wrap) atomicOr(A.err, ERR_OVERFLOW);
+    __syncthreads();
+    if (S.overflow) {  // crowded keys: clean up, leave the item to k_hrank
+      for (int i = t; i < Stot; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
+      if (t == 0) {
+        redo[atomicAdd(nredo, 1u)] = it;
+        S.overflow = 0;
+        S.dmax = 0;
+      }
+      __syncthreads();
+      continue;
+    }
+    // ---- 2. occupancy of the thread's slots [t q, t q + q), block scan
+    const int j0 = t * q;
+    const int d = S.dmax;
+    unsigned occ = 0;
+    for (int j = 0; j < q; ++j) occ |= (unsigned)(S.key[j0 + j] != kEmpty) << j;
+    const int c = __popc(occ);
+    int x = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) S.wsum[wid] = x;
+    __syncthreads();
+    int base = x - c, D = 0;
+#pragma unroll
+    for (int w = 0; w < NT / 32; ++w) {
+      const int s = S.wsum[w];
+      base += w < wid ? s : 0;
+      D += s;
+    }
+    // ---- 3. rank of every occupied slot of the thread, (b, sum) written at it
+    bool over32 = false;
+    int before = base;
+    for (int j = 0; j < q; ++j) {
+      if (!((occ >> j) & 1u)) continue;
+      const int i = j0 + j;
+      const int32_t b = S.key[i];
+      int r = before++;
+      for (int m = i - d < 0 ? 0 : i - d; m < i; ++m) r -= S.key[m] > b;
+      for (int m = i + 1; m <= i + d; ++m) {
+        const int32_t y = S.key[m];
+        r += y != kEmpty && y < b;
+      }
+      const uint32_t sum = S.val[i];
+      over32 |= sum > 0x7fffffffu;
+      src_b[r] = b;
+      src_w[r] = (int32_t)sum;
+    }
+    if (over32) atomicOr(A.err, ERR_OVERFLOW);
+    __syncthreads();  // every neighbourhood read before the slots are cleared
+    for (int j = 0; j < q; ++j) {
+      if ((occ >> j) & 1u) {
+        S.key[j0 + j] = kEmpty;
+        S.val[j0 + j] = 0u;
+      }
+    }
+    if (t == 0) {
+      A.blk_cnt[it.bi] = D;
+      S.dmax = 0;
+    }
+    __syncthreads();
+  }
+}
+
+int launch_mrank(hec_ctx *ctx, const RowsArgs &A, int cls, RbmItem *redo, unsigned *nredo) {
+#define HEC_MR(NTV)                                                                                          \
+  {                                                                                                          \
+    const size_t smem = sizeof(MrSmem<NTV>);                                                                 \
+    HEC_CUDA_TRY(cudaFuncSetAttribute(k_mrank<NTV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
+    int occ = 1;                                                                                             \
+    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_mrank<NTV>, NTV, smem));              \
+    int64_t grid = (int64_t)ctx->num_sms * (occ < 1 ? 1 : occ);                                             \
+    if (A.nblocks < grid) grid = A.nblocks;                                                                  \
+    if (grid < 1) return HEC_OK;                                                                             \
+    k_mrank<NTV><<<(unsigned)grid, NTV, smem, ctx->stream>>>(A, redo, nredo);                                \
+    HEC_LAUNCH_CHECK();                                                                                      \
+    return HEC_OK;                                                                                           \
+  }
+  if (cls < 0) HEC_MR(64)
+  if (cls == 0) HEC_MR(128)
+  if (cls == 1) HEC_MR(256)
+  HEC_MR(512)
+#undef HEC_MR
 }
 
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo) {

@@ -255,7 +255,7 @@ def test_construct_random_labels(P, ctx):
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index"])
+@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index", "hrank"])
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
 def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     """R-MAT with random labels into nc aggregates: few labels give huge rows
@@ -268,6 +268,8 @@ def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
         monkeypatch.setenv("HEC_NO_RBM", "1")
     if path == "wide_index":
         monkeypatch.setenv("HEC_FORCE_WIDE_INDEX", "1")
+    if path == "hrank":  # rank items through the unordered hash + bucket rank (k_hrank) only
+        monkeypatch.setenv("HEC_NO_MRANK", "1")
     rng = np.random.default_rng(15 + nc)
     g = gg.rmat(14 if nc < 20000 else 17, 16)
     g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
@@ -295,6 +297,38 @@ def test_construct_wide_piece_keys(P, ctx, monkeypatch):
         cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
     check_hierarchy(P, ctx, gg.config(2), 1000)
+
+
+@pytest.mark.parametrize("spread", [600, 6000, 60000])
+def test_construct_crowded_keys(P, ctx, spread):
+    """Whole-row rank items whose keys crowd the low end of [0, n_c): the
+    order-preserving table (k_mrank) sees long probe runs -- spread 600 forces
+    its probe bound and the redo through k_hrank, 6000 gives long runs with a
+    large rank window, 60000 is uniform."""
+    rng = np.random.default_rng(31 + spread)
+    n, nc = 200000, 60000
+    M = rng.integers(0, nc, n).astype(np.int32)
+    M[rng.permutation(n)[:nc]] = np.arange(nc)
+    by_label = [np.flatnonzero((M >= 1) & (M < spread))]
+    edges = {}
+    heads = np.arange(200)  # rows 0..9 of 20 members, each member with ~120 neighbours in the crowded labels
+    M[heads] = heads // 20
+    for u in heads:
+        for v in rng.choice(by_label[0], 120, replace=False):
+            if v != u:
+                edges[(min(u, v), max(u, v))] = int(rng.integers(1, 5))
+    for _ in range(2 * n):
+        u, v = rng.integers(0, n, 2)
+        if u != v:
+            edges[(min(u, v), max(u, v))] = int(rng.integers(1, 9))
+    g = gg.from_edges(n, [(u, v, w) for (u, v), w in edges.items()])
+    present = np.unique(M)
+    remap = np.full(nc, -1, np.int64)
+    remap[present] = np.arange(present.size)
+    M = remap[M].astype(np.int32)
+    nc = int(present.size)
+    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+    assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
 @pytest.mark.parametrize("path", ["rbm", "bins"])
