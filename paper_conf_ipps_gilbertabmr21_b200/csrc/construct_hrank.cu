@@ -298,10 +298,12 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
 // after its home and at most d = (the item's largest probe distance) after
 // it, so for keys x at slot i and y at slot m:  m < i - d  =>  h(y) <= m <
 // i - d <= h(x)  =>  y < x  (h monotone), and symmetrically m > i + d => y >
-// x.  The output rank of x is therefore
-//   (occupied slots before i) - #{m in [i-d, i): y > x} + #{m in (i, i+d]: y < x},
-// one block scan of per-thread occupancy counts plus <= 2d comparisons per
-// key -- replacing k_hrank's bucket counts, scatter and in-bucket rank loop,
+// x; and a key beyond an empty slot is in another run, whose homes lie on that
+// side of x's home.  The output rank of x is therefore
+//   (occupied slots before i) - #{y > x in its run within [i-d, i)}
+//                             + #{y < x in its run within (i, i+d]},
+// one block scan of per-thread occupancy counts plus a few comparisons per
+// key (runs are ~1-2 slots at load <= 1/2) -- replacing k_hrank's bucket counts, scatter and in-bucket rank loop,
 // which its source profile put at ~45% of its instructions.  Items whose
 // probes exceed kMaxProbe or the table margin (keys crowded in a narrow part of
 // [lo, hi)) are left untouched and appended to a redo list for k_hrank.
@@ -379,6 +381,7 @@ __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__
     __syncthreads();
     if (S.overflow) {  // crowded keys: clean up, leave the item to k_hrank
       for (int i = t; i < Stot; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
+      __syncthreads();  // every thread has read the flag before it is reset
       if (t == 0) {
         redo[atomicAdd(nredo, 1u)] = it;
         S.overflow = 0;
@@ -415,11 +418,19 @@ __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__
       if (!((occ >> j) & 1u)) continue;
       const int i = j0 + j;
       const int32_t b = S.key[i];
+      // only keys of the same run within distance d can be out of order (a
+      // key beyond an empty slot lies in another run, whose homes are all on
+      // that side of x's home)
       int r = before++;
-      for (int m = i - d < 0 ? 0 : i - d; m < i; ++m) r -= S.key[m] > b;
+      for (int m = i - 1; m >= i - d && m >= 0; --m) {
+        const int32_t y = S.key[m];
+        if (y == kEmpty) break;
+        r -= y > b;
+      }
       for (int m = i + 1; m <= i + d; ++m) {
         const int32_t y = S.key[m];
-        r += y != kEmpty && y < b;
+        if (y == kEmpty) break;
+        r += y < b;
       }
       const uint32_t sum = S.val[i];
       over32 |= sum > 0x7fffffffu;
