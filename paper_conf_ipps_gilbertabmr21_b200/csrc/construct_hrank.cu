@@ -307,6 +307,14 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
 // which its source profile put at ~45% of its instructions.  Items whose
 // probes exceed kMaxProbe or the table margin (keys crowded in a narrow part of
 // [lo, hi)) are left untouched and appended to a redo list for k_hrank.
+//
+// Keys are not uniform in [0, n_c): with unit weights the heavy-neighbour
+// tie-break (smallest id, L116) grows large aggregates at low ids, so low
+// coarse ids carry ~5x the volume (R-MAT).  Items wider than n_c / 64 keys
+// map keys through F, the level's volume CDF (upos(b) / P, kept as a
+// kCdfK-interval piecewise-linear table in shared memory): homes stay
+// monotone and are close to uniform (an R-MAT s20 simulation: largest probe
+// distance 5-20 slots, against 50-300 for the linear map).
 constexpr int kMaxProbe = 48;
 template <int NT, int PER = 8>
 struct MrSmem {
@@ -315,9 +323,20 @@ struct MrSmem {
   static constexpr int kSlots = kQ * NT;       // 2 pow2(n) home slots + >= NT margin
   int32_t key[kSlots + kMaxProbe];             // tail: permanently empty (rank window)
   uint32_t val[kSlots];
+  uint32_t cdf[kCdfK + 1];                     // F at i n_c / kCdfK, fixed point (2^31 = all volume)
   int32_t wsum[NT / 32];
   int32_t overflow, dmax;
 };
+
+// F(b): piecewise-linear interpolation of the CDF table (monotone in b).
+__device__ __forceinline__ uint32_t cdf_at(const uint32_t *cdf, float kscale, int32_t b) {
+  const float x = (float)b * kscale;
+  int k = (int)x;
+  if (k >= kCdfK) return cdf[kCdfK];
+  const float frac = x - (float)k;
+  const uint32_t base = cdf[k];
+  return base + (uint32_t)__fmul_rz((float)(cdf[k + 1] - base), frac);
+}
 
 template <int NT, int PER = 8>
 __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__restrict__ redo,
@@ -330,8 +349,10 @@ __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__
   int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
   for (int i = t; i < SM::kSlots + kMaxProbe; i += NT) S.key[i] = kEmpty;
   for (int i = t; i < SM::kSlots; i += NT) S.val[i] = 0u;
+  for (int i = t; i <= kCdfK; i += NT) S.cdf[i] = A.cdf[i];
   if (t == 0) { S.overflow = 0; S.dmax = 0; }
   __syncthreads();
+  const float kscale = (float)kCdfK / (float)A.L.n_c;
   RbmItem nx{};
   if (blockIdx.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, blockIdx.x);
   for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
@@ -346,7 +367,12 @@ __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__
     const int Sh = 2 << lg;
     const int q = Sh / NT + 1;
     const int Stot = q * NT;             // probes stay below Stot (margin >= 1 slot per thread)
-    const float scale = __fdividef((float)Sh, (float)(it.hi - lo));
+    // home(b) = (G(b) - G(lo)) * Sh / (G(hi) - G(lo)), G = F, or the identity
+    // when F's fixed point cannot resolve Sh homes inside [lo, hi)
+    const uint32_t g0 = cdf_at(S.cdf, kscale, lo);
+    const uint32_t g1 = cdf_at(S.cdf, kscale, it.hi);
+    const bool use_cdf = g1 - g0 >= (uint32_t)Sh;
+    const float scale = __fdividef((float)Sh, use_cdf ? (float)(g1 - g0) : (float)(it.hi - lo));
     int32_t kb[PER], kw[PER];
 #pragma unroll
     for (int k = 0; k < PER; ++k) {
@@ -362,7 +388,8 @@ __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__
     for (int k = 0; k < PER; ++k) {
       if (kb[k] == a) kb[k] = -1;  // self entry (L280)
       if (kb[k] < 0) continue;
-      int h = (int)__fmul_rz((float)(kb[k] - lo), scale);
+      const uint32_t g = use_cdf ? cdf_at(S.cdf, kscale, kb[k]) - g0 : (uint32_t)(kb[k] - lo);
+      int h = (int)__fmul_rz((float)g, scale);
       h = h < Sh - 1 ? h : Sh - 1;
       const int home = h;
       while (true) {
