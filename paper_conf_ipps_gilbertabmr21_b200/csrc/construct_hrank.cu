@@ -381,26 +381,32 @@ __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__
       kw[k] = 0;
       if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
     }
-    // ---- 1. insert at the monotone home slot, probing forward
+    // ---- 1. insert at the monotone home slot, probing forward (the warp
+    // reconverges after every entry: a divergent exit here made the later
+    // entries run once per divergent lane group)
     bool wrap = false, over = false;
     int dist = 0;
 #pragma unroll
     for (int k = 0; k < PER; ++k) {
       if (kb[k] == a) kb[k] = -1;  // self entry (L280)
-      if (kb[k] < 0) continue;
-      const uint32_t g = use_cdf ? cdf_at(S.cdf, kscale, kb[k]) - g0 : (uint32_t)(kb[k] - lo);
-      int h = (int)__fmul_rz((float)g, scale);
-      h = h < Sh - 1 ? h : Sh - 1;
-      const int home = h;
-      while (true) {
-        const int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
-        if (old == kEmpty || old == kb[k]) break;
-        if (++h >= Stot || h - home > kMaxProbe) { over = true; break; }
+      if (kb[k] >= 0 && !over) {
+        const uint32_t g = use_cdf ? cdf_at(S.cdf, kscale, kb[k]) - g0 : (uint32_t)(kb[k] - lo);
+        int h = (int)__fmul_rz((float)g, scale);
+        h = h < Sh - 1 ? h : Sh - 1;
+        const int home = h;
+        int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
+        while (old != kEmpty && old != kb[k] && !over) {
+          ++h;
+          if (h >= Stot || h - home > kMaxProbe) over = true;
+          else old = atomicCAS(&S.key[h], kEmpty, kb[k]);
+        }
+        if (!over) {
+          dist = max(dist, h - home);
+          const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
+          wrap |= o + (uint32_t)kw[k] < o;
+        }
       }
-      if (over) break;
-      dist = max(dist, h - home);
-      const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
-      wrap |= o + (uint32_t)kw[k] < o;
+      __syncwarp();
     }
     if (over) S.overflow = 1;
     if (dist > 0) atomicMax(&S.dmax, dist);
@@ -442,27 +448,31 @@ __global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__
     bool over32 = false;
     int before = base;
     for (int j = 0; j < q; ++j) {
-      if (!((occ >> j) & 1u)) continue;
-      const int i = j0 + j;
-      const int32_t b = S.key[i];
-      // only keys of the same run within distance d can be out of order (a
-      // key beyond an empty slot lies in another run, whose homes are all on
-      // that side of x's home)
-      int r = before++;
-      for (int m = i - 1; m >= i - d && m >= 0; --m) {
-        const int32_t y = S.key[m];
-        if (y == kEmpty) break;
-        r -= y > b;
+      if ((occ >> j) & 1u) {
+        const int i = j0 + j;
+        const int32_t b = S.key[i];
+        // only keys of the same run within distance d can be out of order (a
+        // key beyond an empty slot lies in another run, whose homes are all on
+        // that side of x's home)
+        int r = before++;
+        int32_t y = i > 0 && d > 0 ? S.key[i - 1] : kEmpty;
+        for (int m = i - 1; y != kEmpty;) {
+          r -= y > b;
+          --m;
+          y = m >= i - d && m >= 0 ? S.key[m] : kEmpty;
+        }
+        y = d > 0 ? S.key[i + 1] : kEmpty;
+        for (int m = i + 1; y != kEmpty;) {
+          r += y < b;
+          ++m;
+          y = m <= i + d ? S.key[m] : kEmpty;
+        }
+        const uint32_t sum = S.val[i];
+        over32 |= sum > 0x7fffffffu;
+        src_b[r] = b;
+        src_w[r] = (int32_t)sum;
       }
-      for (int m = i + 1; m <= i + d; ++m) {
-        const int32_t y = S.key[m];
-        if (y == kEmpty) break;
-        r += y < b;
-      }
-      const uint32_t sum = S.val[i];
-      over32 |= sum > 0x7fffffffu;
-      src_b[r] = b;
-      src_w[r] = (int32_t)sum;
+      __syncwarp();
     }
     if (over32) atomicOr(A.err, ERR_OVERFLOW);
     __syncthreads();  // every neighbourhood read before the slots are cleared
