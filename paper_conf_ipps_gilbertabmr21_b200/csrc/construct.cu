@@ -214,7 +214,8 @@ __global__ void k_block_ends(int64_t nblocks, int64_t a_hi, BlockDesc *__restric
 }
 
 // Volume CDF of the coarse ids: cdf[i] = upos(floor(i n_c / kCdfK)) / upos(n_c)
-// in 2^31 fixed point (upos(a) = member-edge volume of the rows below a).
+// in 2^31 fixed point (upos(a) = member-edge volume of the rows below a);
+// the hash-rank kernels balance their key-range buckets with it.
 __global__ void k_cdf_table(Layout L, uint32_t *__restrict__ cdf) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i > kCdfK) return;
@@ -1073,7 +1074,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   RbmItem *list_redo = arena_take<RbmItem>(W2, nblocks + 1);  // n > 4096 items left to k_rbm
   RbmItem *list_d = arena_take<RbmItem>(W2, nblocks + 1);     // direct-indexed bins (k_drank)
   RbmItem *list_r3 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n <= kHrMaxS
-  RbmItem *list_mredo = arena_take<RbmItem>(W2, nblocks + 1);  // k_mrank items left to k_hrank
   uint32_t *cdf = arena_take<uint32_t>(W2, kCdfK + 1);
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
@@ -1141,9 +1141,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
 
   const bool direct = getenv("HEC_NO_DRANK") == nullptr;  // test hook: bins through the hash-rank kernels
-  // rank items <= 4096 entries: order-preserving hash rank (HEC_NO_MRANK: the
-  // unordered hash + bucket rank k_hrank for all of them, test hook)
-  const bool use_mrank = getenv("HEC_NO_MRANK") == nullptr;
   int ph_rows = -1;
 
   // ---- a9 skewed rows
@@ -1263,8 +1260,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
       A.nlist = C.n;
       A.rdir = C.dir;
       if (c < 3) {
-        if (use_mrank) HEC_TRY(launch_mrank(ctx, A, c, list_mredo, counts + 19));
-        else HEC_TRY(launch_hrank(ctx, A, c));
+        HEC_TRY(launch_hrank(ctx, A, c));
       } else {
         HEC_TRY(launch_hrank_big(ctx, A, list_redo, counts + 17));
         A.ritems = list_redo;
@@ -1272,12 +1268,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
         A.rdir = 1;
         HEC_TRY(launch_rbm(ctx, A));
       }
-    }
-    if (use_mrank) {  // items whose keys crowded the order-preserving table
-      A.ritems = list_mredo;
-      A.nlist = counts + 19;
-      A.rdir = 1;
-      HEC_TRY(launch_hrank(ctx, A, 2));
     }
     A.ritems = list_d;
     A.nlist = counts + 18;

@@ -76,6 +76,16 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   return total;
 }
 
+// F(b): piecewise-linear interpolation of the coarse-id volume CDF table
+// (construct.cu k_cdf_table; 2^31 fixed point), monotone in b.
+__device__ __forceinline__ uint32_t cdf_at(const uint32_t *__restrict__ cdf, float kscale, int32_t b) {
+  const float x = (float)b * kscale;
+  const int k = (int)x;
+  if (k >= kCdfK) return __ldg(cdf + kCdfK);
+  const uint32_t base = __ldg(cdf + k);
+  return base + (uint32_t)__fmul_rz((float)(__ldg(cdf + k + 1) - base), x - (float)k);
+}
+
 template <int NT, int PER = 8>
 __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4) k_hrank(RowsArgs A) {
   constexpr int kCapE = HrSmem<NT, PER>::kCapE;
@@ -86,6 +96,8 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
   // kernel-argument pointers held in registers (not re-read per slot)
   int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
   int *const err = A.err;
+  const uint32_t *const cdf = A.cdf;
+  const float kscale = (float)kCdfK / (float)A.L.n_c;
   for (int i = t; i < HrSmem<NT, PER>::kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
   for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
@@ -104,8 +116,15 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     const int NB = 1 << lg;
     const uint32_t hmask = 2u * NB - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
-    // any positive scale keeps the buckets monotone in b (approximate division)
-    const float scale = __fdividef((float)NB, (float)(it.hi - lo));
+    // Buckets must be monotone in b; any positive scale does.  Coarse keys are
+    // far from uniform (with unit weights the smallest-id tie-break, L116,
+    // grows large aggregates at low ids: ~5x the volume at the low end on
+    // R-MAT), so b is first mapped through F, the level's coarse-id volume
+    // CDF (piecewise linear, kCdfK intervals): buckets then hold ~equal shares
+    // of the distinct keys and the in-bucket rank below stays short.
+    const uint32_t g0 = cdf_at(cdf, kscale, lo), g1 = cdf_at(cdf, kscale, it.hi);
+    const bool use_cdf = g1 - g0 >= (uint32_t)NB;
+    const float scale = __fdividef((float)NB, use_cdf ? (float)(g1 - g0) : (float)(it.hi - lo));
     int32_t kb[PER], kw[PER];
 #pragma unroll
     for (int k = 0; k < PER; ++k) {
@@ -134,7 +153,8 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
       const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
       wrap |= o + (uint32_t)kw[k] < o;
       if (own & (1u << k)) {
-        int bk = (int)__fmul_rz((float)(kb[k] - lo), scale);
+        const uint32_t g = use_cdf ? cdf_at(cdf, kscale, kb[k]) - g0 : (uint32_t)(kb[k] - lo);
+        int bk = (int)__fmul_rz((float)g, scale);
         bk = bk < NB - 1 ? bk : NB - 1;
         bpos[k] = atomicAdd(&S.cnt[bk], 1);
         slot[k] |= bk << 16;  // slot < 2^14, bucket < 2^13
@@ -288,227 +308,6 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
     }
     __syncthreads();
   }
-}
-
-// ---------------------------------------------------------------------------
-// Order-preserving hash rank (k_mrank).  Same items as k_hrank, but the table
-// is indexed by a MONOTONE function of the key, h(b) = floor((b - lo) * S / W)
-// (W = hi - lo, S = 2 pow2(n) home slots) with linear probing forward, no
-// wrap-around, and probe distances bounded by kMaxProbe.  A key sits at or
-// after its home and at most d = (the item's largest probe distance) after
-// it, so for keys x at slot i and y at slot m:  m < i - d  =>  h(y) <= m <
-// i - d <= h(x)  =>  y < x  (h monotone), and symmetrically m > i + d => y >
-// x; and a key beyond an empty slot is in another run, whose homes lie on that
-// side of x's home.  The output rank of x is therefore
-//   (occupied slots before i) - #{y > x in its run within [i-d, i)}
-//                             + #{y < x in its run within (i, i+d]},
-// one block scan of per-thread occupancy counts plus a few comparisons per
-// key (runs are ~1-2 slots at load <= 1/2) -- replacing k_hrank's bucket counts, scatter and in-bucket rank loop,
-// which its source profile put at ~45% of its instructions.  Items whose
-// probes exceed kMaxProbe or the table margin (keys crowded in a narrow part of
-// [lo, hi)) are left untouched and appended to a redo list for k_hrank.
-//
-// Keys are not uniform in [0, n_c): with unit weights the heavy-neighbour
-// tie-break (smallest id, L116) grows large aggregates at low ids, so low
-// coarse ids carry ~5x the volume (R-MAT).  Items wider than n_c / 64 keys
-// map keys through F, the level's volume CDF (upos(b) / P, kept as a
-// kCdfK-interval piecewise-linear table in shared memory): homes stay
-// monotone and are close to uniform (an R-MAT s20 simulation: largest probe
-// distance 5-20 slots, against 50-300 for the linear map).
-constexpr int kMaxProbe = 48;
-template <int NT, int PER = 8>
-struct MrSmem {
-  static constexpr int kCapE = NT * PER;
-  static constexpr int kQ = 2 * PER + 1;       // slots per thread in the sweep
-  static constexpr int kSlots = kQ * NT;       // 2 pow2(n) home slots + >= NT margin
-  int32_t key[kSlots + kMaxProbe];             // tail: permanently empty (rank window)
-  uint32_t val[kSlots];
-  uint32_t cdf[kCdfK + 1];                     // F at i n_c / kCdfK, fixed point (2^31 = all volume)
-  int32_t wsum[NT / 32];
-  int32_t overflow, dmax;
-};
-
-// F(b): piecewise-linear interpolation of the CDF table (monotone in b).
-__device__ __forceinline__ uint32_t cdf_at(const uint32_t *cdf, float kscale, int32_t b) {
-  const float x = (float)b * kscale;
-  int k = (int)x;
-  if (k >= kCdfK) return cdf[kCdfK];
-  const float frac = x - (float)k;
-  const uint32_t base = cdf[k];
-  return base + (uint32_t)__fmul_rz((float)(cdf[k + 1] - base), frac);
-}
-
-template <int NT, int PER = 8>
-__global__ void __launch_bounds__(NT, 1536 / NT) k_mrank(RowsArgs A, RbmItem *__restrict__ redo,
-                                                         unsigned *__restrict__ nredo) {
-  using SM = MrSmem<NT, PER>;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  SM &S = *reinterpret_cast<SM *>(smem_raw);
-  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
-  const int64_t nitems = *A.nlist;
-  int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
-  for (int i = t; i < SM::kSlots + kMaxProbe; i += NT) S.key[i] = kEmpty;
-  for (int i = t; i < SM::kSlots; i += NT) S.val[i] = 0u;
-  for (int i = t; i <= kCdfK; i += NT) S.cdf[i] = A.cdf[i];
-  if (t == 0) { S.overflow = 0; S.dmax = 0; }
-  __syncthreads();
-  const float kscale = (float)kCdfK / (float)A.L.n_c;
-  RbmItem nx{};
-  if (blockIdx.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, blockIdx.x);
-  for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
-    const RbmItem it = nx;  // descriptor prefetched one item ahead
-    if (ii + gridDim.x < nitems) nx = rbm_at(A.ritems, A.rdir, A.rcap, ii + gridDim.x);
-    const int n = it.n;
-    const int32_t a = it.row, lo = it.lo;
-    int32_t *const src_b = (it.bk < 0 ? scb : pbg) + it.src;
-    int32_t *const src_w = (it.bk < 0 ? scw : pwg) + it.src;
-    // geometry: Sh = 2 pow2(n) home slots; the sweep covers q slots per thread
-    const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
-    const int Sh = 2 << lg;
-    const int q = Sh / NT + 1;
-    const int Stot = q * NT;             // probes stay below Stot (margin >= 1 slot per thread)
-    // home(b) = (G(b) - G(lo)) * Sh / (G(hi) - G(lo)), G = F, or the identity
-    // when F's fixed point cannot resolve Sh homes inside [lo, hi)
-    const uint32_t g0 = cdf_at(S.cdf, kscale, lo);
-    const uint32_t g1 = cdf_at(S.cdf, kscale, it.hi);
-    const bool use_cdf = g1 - g0 >= (uint32_t)Sh;
-    const float scale = __fdividef((float)Sh, use_cdf ? (float)(g1 - g0) : (float)(it.hi - lo));
-    int32_t kb[PER], kw[PER];
-#pragma unroll
-    for (int k = 0; k < PER; ++k) {
-      const int i = t + NT * k;
-      kb[k] = -1;
-      kw[k] = 0;
-      if (i < n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
-    }
-    // ---- 1. insert at the monotone home slot, probing forward (the warp
-    // reconverges after every entry: a divergent exit here made the later
-    // entries run once per divergent lane group)
-    bool wrap = false, over = false;
-    int dist = 0;
-#pragma unroll
-    for (int k = 0; k < PER; ++k) {
-      if (kb[k] == a) kb[k] = -1;  // self entry (L280)
-      if (kb[k] >= 0 && !over) {
-        const uint32_t g = use_cdf ? cdf_at(S.cdf, kscale, kb[k]) - g0 : (uint32_t)(kb[k] - lo);
-        int h = (int)__fmul_rz((float)g, scale);
-        h = h < Sh - 1 ? h : Sh - 1;
-        const int home = h;
-        int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
-        while (old != kEmpty && old != kb[k] && !over) {
-          ++h;
-          if (h >= Stot || h - home > kMaxProbe) over = true;
-          else old = atomicCAS(&S.key[h], kEmpty, kb[k]);
-        }
-        if (!over) {
-          dist = max(dist, h - home);
-          const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
-          wrap |= o + (uint32_t)kw[k] < o;
-        }
-      }
-      __syncwarp();
-    }
-    if (over) S.overflow = 1;
-    if (dist > 0) atomicMax(&S.dmax, dist);
-    if (wrap) atomicOr(A.err, ERR_OVERFLOW);
-    __syncthreads();
-    if (S.overflow) {  // crowded keys: clean up, leave the item to k_hrank
-      for (int i = t; i < Stot; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
-      __syncthreads();  // every thread has read the flag before it is reset
-      if (t == 0) {
-        redo[atomicAdd(nredo, 1u)] = it;
-        S.overflow = 0;
-        S.dmax = 0;
-      }
-      __syncthreads();
-      continue;
-    }
-    // ---- 2. occupancy of the thread's slots [t q, t q + q), block scan
-    const int j0 = t * q;
-    const int d = S.dmax;
-    unsigned occ = 0;
-    for (int j = 0; j < q; ++j) occ |= (unsigned)(S.key[j0 + j] != kEmpty) << j;
-    const int c = __popc(occ);
-    int x = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) S.wsum[wid] = x;
-    __syncthreads();
-    int base = x - c, D = 0;
-#pragma unroll
-    for (int w = 0; w < NT / 32; ++w) {
-      const int s = S.wsum[w];
-      base += w < wid ? s : 0;
-      D += s;
-    }
-    // ---- 3. rank of every occupied slot of the thread, (b, sum) written at it
-    bool over32 = false;
-    int before = base;
-    for (int j = 0; j < q; ++j) {
-      if ((occ >> j) & 1u) {
-        const int i = j0 + j;
-        const int32_t b = S.key[i];
-        // only keys of the same run within distance d can be out of order (a
-        // key beyond an empty slot lies in another run, whose homes are all on
-        // that side of x's home)
-        int r = before++;
-        int32_t y = i > 0 && d > 0 ? S.key[i - 1] : kEmpty;
-        for (int m = i - 1; y != kEmpty;) {
-          r -= y > b;
-          --m;
-          y = m >= i - d && m >= 0 ? S.key[m] : kEmpty;
-        }
-        y = d > 0 ? S.key[i + 1] : kEmpty;
-        for (int m = i + 1; y != kEmpty;) {
-          r += y < b;
-          ++m;
-          y = m <= i + d ? S.key[m] : kEmpty;
-        }
-        const uint32_t sum = S.val[i];
-        over32 |= sum > 0x7fffffffu;
-        src_b[r] = b;
-        src_w[r] = (int32_t)sum;
-      }
-      __syncwarp();
-    }
-    if (over32) atomicOr(A.err, ERR_OVERFLOW);
-    __syncthreads();  // every neighbourhood read before the slots are cleared
-    for (int j = 0; j < q; ++j) {
-      if ((occ >> j) & 1u) {
-        S.key[j0 + j] = kEmpty;
-        S.val[j0 + j] = 0u;
-      }
-    }
-    if (t == 0) {
-      A.blk_cnt[it.bi] = D;
-      S.dmax = 0;
-    }
-    __syncthreads();
-  }
-}
-
-int launch_mrank(hec_ctx *ctx, const RowsArgs &A, int cls, RbmItem *redo, unsigned *nredo) {
-#define HEC_MR(NTV)                                                                                          \
-  {                                                                                                          \
-    const size_t smem = sizeof(MrSmem<NTV>);                                                                 \
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_mrank<NTV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
-    int occ = 1;                                                                                             \
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_mrank<NTV>, NTV, smem));              \
-    int64_t grid = (int64_t)ctx->num_sms * (occ < 1 ? 1 : occ);                                             \
-    if (A.nblocks < grid) grid = A.nblocks;                                                                  \
-    if (grid < 1) return HEC_OK;                                                                             \
-    k_mrank<NTV><<<(unsigned)grid, NTV, smem, ctx->stream>>>(A, redo, nredo);                                \
-    HEC_LAUNCH_CHECK();                                                                                      \
-    return HEC_OK;                                                                                           \
-  }
-  if (cls < 0) HEC_MR(64)
-  if (cls == 0) HEC_MR(128)
-  if (cls == 1) HEC_MR(256)
-  HEC_MR(512)
-#undef HEC_MR
 }
 
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo) {

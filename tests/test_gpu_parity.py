@@ -255,7 +255,7 @@ def test_construct_random_labels(P, ctx):
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index", "hrank"])
+@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index"])
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
 def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     """R-MAT with random labels into nc aggregates: few labels give huge rows
@@ -268,8 +268,6 @@ def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
         monkeypatch.setenv("HEC_NO_RBM", "1")
     if path == "wide_index":
         monkeypatch.setenv("HEC_FORCE_WIDE_INDEX", "1")
-    if path == "hrank":  # rank items through the unordered hash + bucket rank (k_hrank) only
-        monkeypatch.setenv("HEC_NO_MRANK", "1")
     rng = np.random.default_rng(15 + nc)
     g = gg.rmat(14 if nc < 20000 else 17, 16)
     g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
@@ -301,10 +299,9 @@ def test_construct_wide_piece_keys(P, ctx, monkeypatch):
 
 @pytest.mark.parametrize("spread", [600, 6000, 60000])
 def test_construct_crowded_keys(P, ctx, spread):
-    """Whole-row rank items whose keys crowd the low end of [0, n_c): the
-    order-preserving table (k_mrank) sees long probe runs -- spread 600 forces
-    its probe bound and the redo through k_hrank, 6000 gives long runs with a
-    large rank window, 60000 is uniform."""
+    """Whole-row rank items whose keys crowd the low end of [0, n_c) (spread
+    600 / 6000) or spread uniformly (60000): the hash-rank buckets, balanced by
+    the level's volume CDF, see very uneven key densities."""
     rng = np.random.default_rng(31 + spread)
     n, nc = 200000, 60000
     M = rng.integers(0, nc, n).astype(np.int32)
