@@ -213,19 +213,6 @@ __global__ void k_block_ends(int64_t nblocks, int64_t a_hi, BlockDesc *__restric
   if (rows_kind(blk[k].kind)) blk[k].row1 = (k + 1 < nblocks) ? blk[k + 1].row0 : (int32_t)a_hi;
 }
 
-// Volume CDF of the coarse ids: cdf[i] = upos(floor(i n_c / kCdfK)) / upos(n_c)
-// in 2^31 fixed point (upos(a) = member-edge volume of the rows below a);
-// the hash-rank kernels balance their key-range buckets with it.
-__global__ void k_cdf_table(Layout L, uint32_t *__restrict__ cdf) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i > kCdfK) return;
-  const int64_t P = L.upos(L.n_c);
-  const int64_t a = (int64_t)((double)i * (double)L.n_c / (double)kCdfK);
-  const int64_t v = L.upos(a < L.n_c ? a : L.n_c);
-  cdf[i] = P > 0 ? (uint32_t)((double)v / (double)P * 2147483648.0) : 0u;
-  if (i == kCdfK) cdf[i] = 2147483648u;
-}
-
 // ------------------------------------------------------- a9 BUCKET partition
 // Work units: big row h (list index) split into ceil(U/unit) windows of `unit`
 // member-edge positions (kUnit: partition, kCap: dense accumulation);
@@ -1044,7 +1031,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // ---- second arena: block list, block counts/offsets, staging, skew-path buffers
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
-                ws_bytes(kCdfK + 1, 4) +
                 8 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
@@ -1074,7 +1060,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   RbmItem *list_redo = arena_take<RbmItem>(W2, nblocks + 1);  // n > 4096 items left to k_rbm
   RbmItem *list_d = arena_take<RbmItem>(W2, nblocks + 1);     // direct-indexed bins (k_drank)
   RbmItem *list_r3 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n <= kHrMaxS
-  uint32_t *cdf = arena_take<uint32_t>(W2, kCdfK + 1);
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1123,9 +1108,6 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   A.err = err;
   A.mstart = mstart;
   A.idx32 = idx32;
-  A.cdf = cdf;
-  k_cdf_table<<<nblk(kCdfK + 1, 256), 256, 0, s>>>(L, cdf);
-  HEC_LAUNCH_CHECK();
 
   static bool attr = false;
   if (!attr) {

@@ -243,7 +243,6 @@ struct WorkItem {
 // k_hrank<128/256/512> (construct_hrank.cu), larger ones to k_rbm.
 constexpr int kHrMaxS = 512, kHrMax0 = 1024, kHrMax1 = 2048, kHrMax2 = 4096;
 constexpr int kDirectR = 4096;  // bins with a key range this small: direct-indexed counters (k_drank)
-constexpr int kCdfK = 1024;     // intervals of the coarse-id volume CDF table (hash-rank buckets)
 
 // A bitmap-rank item (construct_rbm.cu), self-contained so a CTA prefetches it:
 // entries [src, src + n) of sc_col/sc_wgt (B_RBM whole row) or pb_g/pw_g (bin),
@@ -320,7 +319,6 @@ struct RowsArgs {
   int64_t *row_ptr_c;
   int32_t *col_c, *wgt_c, *vwgt_c;
   int *err;
-  const uint32_t *cdf;    // [kCdfK + 1] volume CDF of the coarse ids (hash-rank buckets)
   const int64_t *mstart;  // row_ptr[members[i]]: rank items walk their member rows (x2_walk)
   bool idx32;             // entry / position indices of the walks fit 32 bits (nnz < 2^32)
   const int32_t *list;    // blocks of this launch (a tier list)

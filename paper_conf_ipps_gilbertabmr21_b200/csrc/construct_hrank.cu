@@ -76,16 +76,6 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   return total;
 }
 
-// F(b): piecewise-linear interpolation of the coarse-id volume CDF table
-// (construct.cu k_cdf_table; 2^31 fixed point), monotone in b.
-__device__ __forceinline__ uint32_t cdf_at(const uint32_t *__restrict__ cdf, float kscale, int32_t b) {
-  const float x = (float)b * kscale;
-  const int k = (int)x;
-  if (k >= kCdfK) return __ldg(cdf + kCdfK);
-  const uint32_t base = __ldg(cdf + k);
-  return base + (uint32_t)__fmul_rz((float)(__ldg(cdf + k + 1) - base), x - (float)k);
-}
-
 template <int NT, int PER = 8>
 __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4) k_hrank(RowsArgs A) {
   constexpr int kCapE = HrSmem<NT, PER>::kCapE;
@@ -96,8 +86,6 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
   // kernel-argument pointers held in registers (not re-read per slot)
   int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
   int *const err = A.err;
-  const uint32_t *const cdf = A.cdf;
-  const float kscale = (float)kCdfK / (float)A.L.n_c;
   for (int i = t; i < HrSmem<NT, PER>::kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
   for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
@@ -116,15 +104,8 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     const int NB = 1 << lg;
     const uint32_t hmask = 2u * NB - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
-    // Buckets must be monotone in b; any positive scale does.  Coarse keys are
-    // far from uniform (with unit weights the smallest-id tie-break, L116,
-    // grows large aggregates at low ids: ~5x the volume at the low end on
-    // R-MAT), so b is first mapped through F, the level's coarse-id volume
-    // CDF (piecewise linear, kCdfK intervals): buckets then hold ~equal shares
-    // of the distinct keys and the in-bucket rank below stays short.
-    const uint32_t g0 = cdf_at(cdf, kscale, lo), g1 = cdf_at(cdf, kscale, it.hi);
-    const bool use_cdf = g1 - g0 >= (uint32_t)NB;
-    const float scale = __fdividef((float)NB, use_cdf ? (float)(g1 - g0) : (float)(it.hi - lo));
+    // any positive scale keeps the buckets monotone in b (approximate division)
+    const float scale = __fdividef((float)NB, (float)(it.hi - lo));
     int32_t kb[PER], kw[PER];
 #pragma unroll
     for (int k = 0; k < PER; ++k) {
@@ -153,8 +134,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
       const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
       wrap |= o + (uint32_t)kw[k] < o;
       if (own & (1u << k)) {
-        const uint32_t g = use_cdf ? cdf_at(cdf, kscale, kb[k]) - g0 : (uint32_t)(kb[k] - lo);
-        int bk = (int)__fmul_rz((float)g, scale);
+        int bk = (int)__fmul_rz((float)(kb[k] - lo), scale);
         bk = bk < NB - 1 ? bk : NB - 1;
         bpos[k] = atomicAdd(&S.cnt[bk], 1);
         slot[k] |= bk << 16;  // slot < 2^14, bucket < 2^13
