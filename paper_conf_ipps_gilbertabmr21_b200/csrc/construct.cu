@@ -1032,6 +1032,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   {
     size_t b2 = ws_bytes(nblocks + 1, sizeof(BlockDesc)) + 4 * ws_bytes(nblocks + 1, 4) + ws_bytes(nblocks + 1, 8) +
                 8 * ws_bytes(nblocks + 1, sizeof(RbmItem)) +
+                ws_bytes(2 * drank_split_bound(big_vol) + 1, sizeof(RbmItem)) +
+                ws_bytes((size_t)drank_split_bound(big_vol) * kDirectR, 4) + ws_bytes(drank_split_bound(big_vol), 4) +
                 ws_bytes(nblocks + 1, sizeof(WorkItem)) +
                 ws_bytes(nblocks + 1, 8) + scan_ws_bytes(nblocks) +
                 2 * ws_bytes((size_t)(small_vol + big_vol) + 1, 4);
@@ -1059,6 +1061,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   RbmItem *list_r2 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n > 2048 (front / back)
   RbmItem *list_redo = arena_take<RbmItem>(W2, nblocks + 1);  // n > 4096 items left to k_rbm
   RbmItem *list_d = arena_take<RbmItem>(W2, nblocks + 1);     // direct-indexed bins (k_drank)
+  // chunks of the direct-indexed bins above kDrSplit entries, their accumulators and tickets
+  const int64_t nsplit_max = drank_split_bound(big_vol);
+  RbmItem *list_dc = arena_take<RbmItem>(W2, 2 * nsplit_max + 1);
+  uint32_t *drank_acc = arena_take<uint32_t>(W2, (size_t)nsplit_max * kDirectR);
+  unsigned *drank_done = arena_take<unsigned>(W2, nsplit_max);
   RbmItem *list_r3 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n <= kHrMaxS
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
@@ -1254,7 +1261,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.ritems = list_d;
     A.nlist = counts + 18;
     A.rdir = 1;
-    HEC_TRY(launch_drank(ctx, A));
+    HEC_TRY(launch_drank(ctx, A, list_dc, counts + 19, drank_acc, counts + 20, drank_done, counts + 21));
     A.ticket = counts + 1;
   }
   phase_end(ctx, ph_rows);

@@ -250,6 +250,10 @@ constexpr int kDirectR = 4096;  // bins with a key range this small: direct-inde
 struct RbmItem {
   int64_t src;
   int32_t n, row, lo, hi, bi, bk;  // bk: bin index (-1 for a whole row)
+  // chunk c of nchunk of a split direct-indexed bin (k_drank; nchunk = 0 otherwise):
+  // counters accumulate at gacc[acc .. acc + hi - lo), sidx its completion ticket
+  int32_t chunk, nchunk, sidx;
+  int64_t acc;
 };
 
 // smallest b in [0, n_c] whose partition bin floor(b * nb / n_c) (float, clamped
@@ -338,6 +342,11 @@ int launch_rbm(hec_ctx *ctx, const RowsArgs &A);  // construct_rbm.cu
 int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls);  // construct_hrank.cu (cls -1..2: n <= 512/1024/2048/4096)
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo);  // n > 4096
 
-int launch_drank(hec_ctx *ctx, const RowsArgs &A);  // bins with hi - lo <= kDirectR
+// bins with hi - lo <= kDirectR; bins above kDrSplit entries are cut into chunks
+// (list dc, global accumulators gacc / tickets done, sized by drank_split_bound)
+constexpr int kDrSplit = 16384;
+inline int64_t drank_split_bound(int64_t entries) { return entries / kDrSplit + 1; }  // split bins
+int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, uint32_t *gacc,
+                 unsigned *gacc_used, unsigned *done, unsigned *nsplit);
 
 }  // namespace hec

@@ -311,49 +311,123 @@ int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *n
 // b - lo (one shared-memory atomic, no probing); a scan over the range's
 // non-zero counters then gives every distinct key its rank, and each thread
 // writes its slice of keys in order -- already sorted, no hashing, no ranking
-// pass.  Items of any length (rounds of NT*8 entries, no barrier between rounds).
+// pass.
+// Bins above kDrSplit entries (the hub aggregates' bins: on C5 level 1 a few
+// of them held most entries, and one CTA per bin left 79% of the SMs idle at
+// the tail) are cut into chunks of kDrSplit entries: each chunk accumulates in
+// shared memory, adds its non-zero counters to the bin's global accumulator,
+// and the chunk that takes the bin's last completion ticket (after a fence)
+// sweeps the accumulator and writes the bin -- so no CTA holds more than one
+// chunk of work.
 constexpr int kDrT = 256;
 static_assert(kDirectR == kDrT * 16, "16 counters per thread");
-__global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
+
+// chunk items of the split bins (list_d items with n > kDrSplit)
+__global__ void k_drank_split(const RbmItem *__restrict__ items, const unsigned *__restrict__ nitems,
+                              RbmItem *__restrict__ dc, unsigned *__restrict__ ndc,
+                              unsigned *__restrict__ gacc_used, unsigned *__restrict__ nsplit) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= *nitems) return;
+  const RbmItem it = items[i];
+  if (it.n <= kDrSplit) return;
+  const int nch = (it.n + kDrSplit - 1) / kDrSplit;
+  const unsigned base = atomicAdd(ndc, (unsigned)nch);
+  const int64_t acc = (int64_t)atomicAdd(gacc_used, (unsigned)kDirectR);
+  const int32_t sidx = (int32_t)atomicAdd(nsplit, 1u);
+  for (int c = 0; c < nch; ++c) {
+    RbmItem ch = it;
+    ch.src = it.src + (int64_t)c * kDrSplit;
+    ch.n = min(kDrSplit, it.n - c * kDrSplit);
+    ch.chunk = c;
+    ch.nchunk = nch;
+    ch.sidx = sidx;
+    ch.acc = acc;
+    dc[base + c] = ch;
+  }
+}
+
+__global__ void k_zero_u32(uint32_t *__restrict__ p, const unsigned *__restrict__ count) {
+  const int64_t n = *count;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = 0u;
+}
+
+// Items: list_d (unsplit bins; split ones are skipped) then the chunks in dc.
+__global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A, const RbmItem *__restrict__ dc,
+                                                const unsigned *__restrict__ ndc, uint32_t *__restrict__ gacc,
+                                                unsigned *__restrict__ done) {
   __shared__ uint32_t val[kDirectR];
   __shared__ int32_t wsum[kDrT / 32];
+  __shared__ int s_last;
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
-  const int64_t nitems = *A.nlist;
+  const int64_t nd = *A.nlist, nitems = nd + *ndc;
   int32_t *const pbg = A.pb_g, *const pwg = A.pw_g;
   for (int i = t; i < kDirectR; i += kDrT) val[i] = 0u;
   __syncthreads();
   for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
-    const RbmItem it = rbm_at(A.ritems, A.rdir, A.rcap, ii);
+    const RbmItem it = ii < nd ? rbm_at(A.ritems, A.rdir, A.rcap, ii) : dc[ii - nd];
+    if (ii < nd && it.n > kDrSplit) continue;  // done as chunks
     const int32_t a = it.row, lo = it.lo;
-    int32_t *const src_b = pbg + it.src;  // bins only (it.bk >= 0)
-    int32_t *const src_w = pwg + it.src;
     bool wrap = false;
-    for (int64_t r0 = 0; r0 < it.n; r0 += 8 * kDrT) {
-      int32_t kb[8], kw[8];
+    {
+      const int32_t *const src_b = pbg + it.src, *const src_w = pwg + it.src;
+      for (int64_t r0 = 0; r0 < it.n; r0 += 8 * kDrT) {
+        int32_t kb[8], kw[8];
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const int64_t i = r0 + t + kDrT * k;
-        kb[k] = -1;
-        kw[k] = 0;
-        if (i < it.n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+        for (int k = 0; k < 8; ++k) {
+          const int64_t i = r0 + t + kDrT * k;
+          kb[k] = -1;
+          kw[k] = 0;
+          if (i < it.n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+        }
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          if (kb[k] < 0 || kb[k] == a) continue;  // self entry (L280)
+          const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
+          wrap |= o + (uint32_t)kw[k] < o;
+        }
       }
+    }
+    __syncthreads();
+    // thread t owns counters [16 t, 16 t + 16)
+    uint32_t v[16];
+    int64_t out = it.src;  // the bin's entries start here; its sorted row is written over them
+    if (it.nchunk > 0) {
+      // chunk of a split bin: add the counters to the bin's accumulator; the
+      // last chunk to finish sweeps it
+      uint32_t *const g = gacc + it.acc;
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        if (kb[k] < 0 || kb[k] == a) continue;  // self entry (L280)
-        const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
-        wrap |= o + (uint32_t)kw[k] < o;
+      for (int q = 0; q < 16; ++q) {
+        const uint32_t x = val[16 * t + q];
+        if (x) {
+          const uint32_t o = atomicAdd(g + 16 * t + q, x);
+          wrap |= o + x < o;
+          val[16 * t + q] = 0u;
+        }
+      }
+      if (wrap) atomicOr(A.err, ERR_OVERFLOW);
+      __threadfence();
+      __syncthreads();
+      if (t == 0) s_last = atomicAdd(done + it.sidx, 1u) == (unsigned)(it.nchunk - 1);
+      __syncthreads();
+      if (!s_last) continue;
+      __threadfence();
+#pragma unroll
+      for (int q = 0; q < 16; ++q) v[q] = __ldcg(g + 16 * t + q);
+      out = it.src - (int64_t)it.chunk * kDrSplit;
+      wrap = false;
+    } else {
+#pragma unroll
+      for (int q = 0; q < 16; ++q) {
+        v[q] = val[16 * t + q];
+        val[16 * t + q] = 0u;
       }
     }
     if (wrap) atomicOr(A.err, ERR_OVERFLOW);
-    __syncthreads();
-    // thread t owns counters [16 t, 16 t + 16): count, block scan, write in order
-    uint32_t v[16];
+    // count, block scan, write in key order
     int c = 0;
 #pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      v[q] = val[16 * t + q];
-      c += v[q] != 0u;
-    }
+    for (int q = 0; q < 16; ++q) c += v[q] != 0u;
     int x = c;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -371,14 +445,14 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
     }
     int pos = before + x - c;
     bool over = false;
+    int32_t *const dst_b = pbg + out, *const dst_w = pwg + out;
 #pragma unroll
     for (int q = 0; q < 16; ++q) {
       if (v[q] != 0u) {
         over |= v[q] > 0x7fffffffu;
-        src_b[pos] = lo + 16 * t + q;
-        src_w[pos] = (int32_t)v[q];
+        dst_b[pos] = lo + 16 * t + q;
+        dst_w[pos] = (int32_t)v[q];
         ++pos;
-        val[16 * t + q] = 0u;
       }
     }
     if (over) atomicOr(A.err, ERR_OVERFLOW);
@@ -387,16 +461,19 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
   }
 }
 
-int launch_drank(hec_ctx *ctx, const RowsArgs &A) {
-  static int occ = 0;
-  if (!occ) {
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank, kDrT, 0));
-    if (occ < 1) occ = 1;
-  }
-  int64_t grid = (int64_t)ctx->num_sms * occ;
-  if (A.nblocks < grid) grid = A.nblocks;
-  if (grid < 1) return HEC_OK;
-  k_drank<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A);
+int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, uint32_t *gacc, unsigned *gacc_used,
+                 unsigned *done, unsigned *nsplit) {
+  if (A.nblocks < 1) return HEC_OK;
+  k_drank_split<<<nblk(A.nblocks + 1, 256), 256, 0, ctx->stream>>>(A.ritems, A.nlist, dc, ndc, gacc_used, nsplit);
+  HEC_LAUNCH_CHECK();
+  k_zero_u32<<<ctx->num_sms * 4, 256, 0, ctx->stream>>>(gacc, gacc_used);
+  HEC_LAUNCH_CHECK();
+  k_zero_u32<<<ctx->num_sms, 256, 0, ctx->stream>>>(done, nsplit);
+  HEC_LAUNCH_CHECK();
+  int occ = 1;
+  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank, kDrT, 0));
+  int64_t grid = (int64_t)ctx->num_sms * (occ < 1 ? 1 : occ);
+  k_drank<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A, dc, ndc, gacc, done);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }
