@@ -1261,7 +1261,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.ritems = list_d;
     A.nlist = counts + 18;
     A.rdir = 1;
-    HEC_TRY(launch_drank(ctx, A, list_dc, counts + 19, drank_acc, counts + 20, drank_done, counts + 21));
+    HEC_TRY(launch_drank(ctx, A, list_dc, counts + 19, drank_acc, drank_done, counts + 21));
     A.ticket = counts + 1;
   }
   phase_end(ctx, ph_rows);

@@ -247,13 +247,13 @@ constexpr int kDirectR = 4096;  // bins with a key range this small: direct-inde
 // A bitmap-rank item (construct_rbm.cu), self-contained so a CTA prefetches it:
 // entries [src, src + n) of sc_col/sc_wgt (B_RBM whole row) or pb_g/pw_g (bin),
 // keys in [lo, hi); row = the coarse row (its self entries are dropped).
+// Chunk c of nchunk of a split direct-indexed bin (k_drank) reuses the fields
+// k_drank does not read: bk = -2 - s (s: the split bin's index; its counters
+// accumulate at gacc[s kDirectR ...), its completion ticket is done[s]) and
+// hi = c << 16 | nchunk.
 struct RbmItem {
   int64_t src;
-  int32_t n, row, lo, hi, bi, bk;  // bk: bin index (-1 for a whole row)
-  // chunk c of nchunk of a split direct-indexed bin (k_drank; nchunk = 0 otherwise):
-  // counters accumulate at gacc[acc .. acc + hi - lo), sidx its completion ticket
-  int32_t chunk, nchunk, sidx;
-  int64_t acc;
+  int32_t n, row, lo, hi, bi, bk;  // bk: bin index (-1 for a whole row, <= -2 for a drank chunk)
 };
 
 // smallest b in [0, n_c] whose partition bin floor(b * nb / n_c) (float, clamped
@@ -346,7 +346,7 @@ int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *n
 // (list dc, global accumulators gacc / tickets done, sized by drank_split_bound)
 constexpr int kDrSplit = 16384;
 inline int64_t drank_split_bound(int64_t entries) { return entries / kDrSplit + 1; }  // split bins
-int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, uint32_t *gacc,
-                 unsigned *gacc_used, unsigned *done, unsigned *nsplit);
+int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, uint32_t *gacc, unsigned *done,
+                 unsigned *nsplit);
 
 }  // namespace hec

@@ -324,30 +324,27 @@ static_assert(kDirectR == kDrT * 16, "16 counters per thread");
 
 // chunk items of the split bins (list_d items with n > kDrSplit)
 __global__ void k_drank_split(const RbmItem *__restrict__ items, const unsigned *__restrict__ nitems,
-                              RbmItem *__restrict__ dc, unsigned *__restrict__ ndc,
-                              unsigned *__restrict__ gacc_used, unsigned *__restrict__ nsplit) {
+                              RbmItem *__restrict__ dc, unsigned *__restrict__ ndc, unsigned *__restrict__ nsplit) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= *nitems) return;
   const RbmItem it = items[i];
   if (it.n <= kDrSplit) return;
   const int nch = (it.n + kDrSplit - 1) / kDrSplit;
   const unsigned base = atomicAdd(ndc, (unsigned)nch);
-  const int64_t acc = (int64_t)atomicAdd(gacc_used, (unsigned)kDirectR);
   const int32_t sidx = (int32_t)atomicAdd(nsplit, 1u);
   for (int c = 0; c < nch; ++c) {
     RbmItem ch = it;
     ch.src = it.src + (int64_t)c * kDrSplit;
     ch.n = min(kDrSplit, it.n - c * kDrSplit);
-    ch.chunk = c;
-    ch.nchunk = nch;
-    ch.sidx = sidx;
-    ch.acc = acc;
+    ch.hi = c << 16 | nch;
+    ch.bk = -2 - sidx;
     dc[base + c] = ch;
   }
 }
 
-__global__ void k_zero_u32(uint32_t *__restrict__ p, const unsigned *__restrict__ count) {
-  const int64_t n = *count;
+// p[0 .. *count * scale) = 0
+__global__ void k_zero_u32(uint32_t *__restrict__ p, const unsigned *__restrict__ count, int scale) {
+  const int64_t n = (int64_t)*count * scale;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     p[i] = 0u;
 }
@@ -392,10 +389,11 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A, const RbmItem *__res
     // thread t owns counters [16 t, 16 t + 16)
     uint32_t v[16];
     int64_t out = it.src;  // the bin's entries start here; its sorted row is written over them
-    if (it.nchunk > 0) {
+    if (it.bk <= -2) {
       // chunk of a split bin: add the counters to the bin's accumulator; the
       // last chunk to finish sweeps it
-      uint32_t *const g = gacc + it.acc;
+      const int sidx = -2 - it.bk, chunk = it.hi >> 16, nchunk = it.hi & 0xffff;
+      uint32_t *const g = gacc + (int64_t)sidx * kDirectR;
 #pragma unroll
       for (int q = 0; q < 16; ++q) {
         const uint32_t x = val[16 * t + q];
@@ -408,13 +406,13 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A, const RbmItem *__res
       if (wrap) atomicOr(A.err, ERR_OVERFLOW);
       __threadfence();
       __syncthreads();
-      if (t == 0) s_last = atomicAdd(done + it.sidx, 1u) == (unsigned)(it.nchunk - 1);
+      if (t == 0) s_last = atomicAdd(done + sidx, 1u) == (unsigned)(nchunk - 1);
       __syncthreads();
       if (!s_last) continue;
       __threadfence();
 #pragma unroll
       for (int q = 0; q < 16; ++q) v[q] = __ldcg(g + 16 * t + q);
-      out = it.src - (int64_t)it.chunk * kDrSplit;
+      out = it.src - (int64_t)chunk * kDrSplit;
       wrap = false;
     } else {
 #pragma unroll
@@ -461,14 +459,14 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A, const RbmItem *__res
   }
 }
 
-int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, uint32_t *gacc, unsigned *gacc_used,
-                 unsigned *done, unsigned *nsplit) {
+int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, uint32_t *gacc, unsigned *done,
+                 unsigned *nsplit) {
   if (A.nblocks < 1) return HEC_OK;
-  k_drank_split<<<nblk(A.nblocks + 1, 256), 256, 0, ctx->stream>>>(A.ritems, A.nlist, dc, ndc, gacc_used, nsplit);
+  k_drank_split<<<nblk(A.nblocks + 1, 256), 256, 0, ctx->stream>>>(A.ritems, A.nlist, dc, ndc, nsplit);
   HEC_LAUNCH_CHECK();
-  k_zero_u32<<<ctx->num_sms * 4, 256, 0, ctx->stream>>>(gacc, gacc_used);
+  k_zero_u32<<<ctx->num_sms * 4, 256, 0, ctx->stream>>>(gacc, nsplit, kDirectR);
   HEC_LAUNCH_CHECK();
-  k_zero_u32<<<ctx->num_sms, 256, 0, ctx->stream>>>(done, nsplit);
+  k_zero_u32<<<ctx->num_sms, 256, 0, ctx->stream>>>(done, nsplit, 1);
   HEC_LAUNCH_CHECK();
   int occ = 1;
   HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank, kDrT, 0));
