@@ -349,83 +349,47 @@ __global__ void k_zero_u32(uint32_t *__restrict__ p, const unsigned *__restrict_
     p[i] = 0u;
 }
 
-// Items: list_d (unsplit bins; split ones are skipped) then the chunks in dc.
-__global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A, const RbmItem *__restrict__ dc,
-                                                const unsigned *__restrict__ ndc, uint32_t *__restrict__ gacc,
-                                                unsigned *__restrict__ done) {
+__global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
   __shared__ uint32_t val[kDirectR];
   __shared__ int32_t wsum[kDrT / 32];
-  __shared__ int s_last;
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
-  const int64_t nd = *A.nlist, nitems = nd + *ndc;
+  const int64_t nitems = *A.nlist;
   int32_t *const pbg = A.pb_g, *const pwg = A.pw_g;
   for (int i = t; i < kDirectR; i += kDrT) val[i] = 0u;
   __syncthreads();
   for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
-    const RbmItem it = ii < nd ? rbm_at(A.ritems, A.rdir, A.rcap, ii) : dc[ii - nd];
-    if (ii < nd && it.n > kDrSplit) continue;  // done as chunks
+    const RbmItem it = rbm_at(A.ritems, A.rdir, A.rcap, ii);
+    if (it.n > kDrSplit) continue;  // split into chunks: k_drank_chunks
     const int32_t a = it.row, lo = it.lo;
+    int32_t *const src_b = pbg + it.src;  // bins only (it.bk >= 0)
+    int32_t *const src_w = pwg + it.src;
     bool wrap = false;
-    {
-      const int32_t *const src_b = pbg + it.src, *const src_w = pwg + it.src;
-      for (int64_t r0 = 0; r0 < it.n; r0 += 8 * kDrT) {
-        int32_t kb[8], kw[8];
+    for (int64_t r0 = 0; r0 < it.n; r0 += 8 * kDrT) {
+      int32_t kb[8], kw[8];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          const int64_t i = r0 + t + kDrT * k;
-          kb[k] = -1;
-          kw[k] = 0;
-          if (i < it.n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
-        }
-#pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          if (kb[k] < 0 || kb[k] == a) continue;  // self entry (L280)
-          const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
-          wrap |= o + (uint32_t)kw[k] < o;
-        }
+      for (int k = 0; k < 8; ++k) {
+        const int64_t i = r0 + t + kDrT * k;
+        kb[k] = -1;
+        kw[k] = 0;
+        if (i < it.n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
       }
-    }
-    __syncthreads();
-    // thread t owns counters [16 t, 16 t + 16)
-    uint32_t v[16];
-    int64_t out = it.src;  // the bin's entries start here; its sorted row is written over them
-    if (it.bk <= -2) {
-      // chunk of a split bin: add the counters to the bin's accumulator; the
-      // last chunk to finish sweeps it
-      const int sidx = -2 - it.bk, chunk = it.hi >> 16, nchunk = it.hi & 0xffff;
-      uint32_t *const g = gacc + (int64_t)sidx * kDirectR;
 #pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        const uint32_t x = val[16 * t + q];
-        if (x) {
-          const uint32_t o = atomicAdd(g + 16 * t + q, x);
-          wrap |= o + x < o;
-          val[16 * t + q] = 0u;
-        }
-      }
-      if (wrap) atomicOr(A.err, ERR_OVERFLOW);
-      __threadfence();
-      __syncthreads();
-      if (t == 0) s_last = atomicAdd(done + sidx, 1u) == (unsigned)(nchunk - 1);
-      __syncthreads();
-      if (!s_last) continue;
-      __threadfence();
-#pragma unroll
-      for (int q = 0; q < 16; ++q) v[q] = __ldcg(g + 16 * t + q);
-      out = it.src - (int64_t)chunk * kDrSplit;
-      wrap = false;
-    } else {
-#pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        v[q] = val[16 * t + q];
-        val[16 * t + q] = 0u;
+      for (int k = 0; k < 8; ++k) {
+        if (kb[k] < 0 || kb[k] == a) continue;  // self entry (L280)
+        const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
+        wrap |= o + (uint32_t)kw[k] < o;
       }
     }
     if (wrap) atomicOr(A.err, ERR_OVERFLOW);
-    // count, block scan, write in key order
+    __syncthreads();
+    // thread t owns counters [16 t, 16 t + 16): count, block scan, write in order
+    uint32_t v[16];
     int c = 0;
 #pragma unroll
-    for (int q = 0; q < 16; ++q) c += v[q] != 0u;
+    for (int q = 0; q < 16; ++q) {
+      v[q] = val[16 * t + q];
+      c += v[q] != 0u;
+    }
     int x = c;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -443,6 +407,100 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A, const RbmItem *__res
     }
     int pos = before + x - c;
     bool over = false;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      if (v[q] != 0u) {
+        over |= v[q] > 0x7fffffffu;
+        src_b[pos] = lo + 16 * t + q;
+        src_w[pos] = (int32_t)v[q];
+        ++pos;
+        val[16 * t + q] = 0u;
+      }
+    }
+    if (over) atomicOr(A.err, ERR_OVERFLOW);
+    if (t == 0) A.blk_cnt[it.bi] = D;
+    __syncthreads();
+  }
+}
+
+// Chunks of the split bins (dc): accumulate, add to the bin's accumulator,
+// the chunk that takes the bin's last ticket sweeps it and writes the bin.
+__global__ void __launch_bounds__(kDrT) k_drank_chunks(RowsArgs A, const RbmItem *__restrict__ dc,
+                                                       const unsigned *__restrict__ ndc, uint32_t *__restrict__ gacc,
+                                                       unsigned *__restrict__ done) {
+  __shared__ uint32_t val[kDirectR];
+  __shared__ int32_t wsum[kDrT / 32];
+  __shared__ int s_last;
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  const int64_t nitems = *ndc;
+  int32_t *const pbg = A.pb_g, *const pwg = A.pw_g;
+  for (int i = t; i < kDirectR; i += kDrT) val[i] = 0u;
+  __syncthreads();
+  for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
+    const RbmItem it = dc[ii];
+    const int32_t a = it.row, lo = it.lo;
+    const int sidx = -2 - it.bk, chunk = it.hi >> 16, nchunk = it.hi & 0xffff;
+    const int32_t *const src_b = pbg + it.src, *const src_w = pwg + it.src;
+    bool wrap = false;
+    for (int64_t r0 = 0; r0 < it.n; r0 += 8 * kDrT) {
+      int32_t kb[8], kw[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int64_t i = r0 + t + kDrT * k;
+        kb[k] = -1;
+        kw[k] = 0;
+        if (i < it.n) { kb[k] = __ldcs(src_b + i); kw[k] = __ldcs(src_w + i); }
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        if (kb[k] < 0 || kb[k] == a) continue;  // self entry (L280)
+        const uint32_t o = atomicAdd(&val[kb[k] - lo], (uint32_t)kw[k]);
+        wrap |= o + (uint32_t)kw[k] < o;
+      }
+    }
+    __syncthreads();
+    uint32_t *const g = gacc + (int64_t)sidx * kDirectR;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const uint32_t x = val[16 * t + q];
+      if (x) {
+        const uint32_t o = atomicAdd(g + 16 * t + q, x);
+        wrap |= o + x < o;
+        val[16 * t + q] = 0u;
+      }
+    }
+    if (wrap) atomicOr(A.err, ERR_OVERFLOW);
+    __threadfence();
+    __syncthreads();
+    if (t == 0) s_last = atomicAdd(done + sidx, 1u) == (unsigned)(nchunk - 1);
+    __syncthreads();
+    if (!s_last) continue;
+    __threadfence();
+    uint32_t v[16];
+    int c = 0;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      v[q] = __ldcg(g + 16 * t + q);
+      c += v[q] != 0u;
+    }
+    int x = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[wid] = x;
+    __syncthreads();
+    int before = 0, D = 0;
+#pragma unroll
+    for (int w = 0; w < kDrT / 32; ++w) {
+      const int sw = wsum[w];
+      before += w < wid ? sw : 0;
+      D += sw;
+    }
+    int pos = before + x - c;
+    bool over = false;
+    const int64_t out = it.src - (int64_t)chunk * kDrSplit;  // the bin's entries start here
     int32_t *const dst_b = pbg + out, *const dst_w = pwg + out;
 #pragma unroll
     for (int q = 0; q < 16; ++q) {
@@ -471,7 +529,12 @@ int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, ui
   int occ = 1;
   HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank, kDrT, 0));
   int64_t grid = (int64_t)ctx->num_sms * (occ < 1 ? 1 : occ);
-  k_drank<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A, dc, ndc, gacc, done);
+  if (A.nblocks < grid) grid = A.nblocks;
+  k_drank<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A);
+  HEC_LAUNCH_CHECK();
+  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank_chunks, kDrT, 0));
+  grid = (int64_t)ctx->num_sms * (occ < 1 ? 1 : occ);
+  k_drank_chunks<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A, dc, ndc, gacc, done);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }
