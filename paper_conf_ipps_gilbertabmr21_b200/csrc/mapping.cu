@@ -554,9 +554,15 @@ struct RoundArgs {
   unsigned *cnt;      // [3] next-list sizes, rotating by round (zeroed)
   int32_t *rounds_out;
   GridBarrier bar;
+  // residual compression (adversarial visit orders): per-vertex scratch
+  int32_t *child;     // an undecided lower child
+  uint8_t *kind;      // K_ROOT / K_ACT / K_UNARY / K_BRANCH
+  uint32_t *jmp[2];   // (target << 0) | parity << 31, double-buffered pointer jumping
 };
 constexpr int kSoloThreshold = 8192;  // finish small residuals in one CTA
 constexpr int kRoundBlock = 512;
+
+constexpr int kComprEvery = 32;  // rounds between residual compressions
 
 // Round r appends its next worklist to cnt[r % 3] and zeroes cnt[(r + 1) % 3]
 // before its barrier.  That counter was last appended in round r - 2 and read
@@ -592,6 +598,122 @@ __device__ __forceinline__ void append(int32_t *list, unsigned *count, bool keep
   if (keep) list[base + __popc(m & ((1u << lane) - 1))] = (int32_t)u;
 }
 
+// ---- residual compression (SURVEY §8(c) "adversarial inputs")
+// After round r the undecided vertices U form a forest under y -> H[y] (y a
+// lower child of H[y], both undecided), and every decided child of an
+// undecided x is ROOT unless it already flagged x (rootflag: an ACTIVE lower
+// child makes x a ROOT).  Alg 3's outcome on U is the NOR evaluation
+//   ACTIVE(x) = !rootflag[x] && no undecided lower child c of x is ACTIVE,
+// so a vertex with exactly one undecided lower child c is NOT(c): unary chains
+// -- the shape of adversarial orders (a path visited against its H direction
+// needs n/2 rounds) -- are resolved by pointer jumping with parity in
+// O(log |U|) passes; branching vertices are left to the following rounds.
+enum : uint8_t { K_ROOT = 1, K_ACT = 2, K_UNARY = 3, K_BRANCH = 4 };
+
+__device__ __forceinline__ bool is_lower(const RoundArgs &A, uint32_t y, int32_t x) {
+  return x != (int32_t)y && A.prio(y) < A.prio((uint32_t)x);
+}
+
+struct GridSync {
+  GridBarrier bar;
+  unsigned nb;
+  __device__ __forceinline__ void operator()() const { bar.sync(nb); }
+};
+struct BlockSync {
+  __device__ __forceinline__ void operator()() const {
+    __threadfence_block();
+    __syncthreads();
+  }
+};
+
+// Compress the residual list (len vertices in `list`, undecided); the new
+// residual goes to `out` (its size counted in *out_cnt, zeroed by the caller),
+// stamped for round r_next.  Returns the new length.
+template <typename Sync>
+__device__ int64_t compress_residual(const RoundArgs &A, const int32_t *list, int64_t len, int32_t *out,
+                                     unsigned *out_cnt, int r_next, int64_t tid, int64_t stride, Sync sync,
+                                     unsigned *s_len) {
+  int32_t *ucnt = A.blocked;  // blocked stamps are rebuilt at the end
+  for (int64_t i = tid; i < len; i += stride) ucnt[list[i]] = 0;
+  sync();
+  for (int64_t i = tid; i < len; i += stride) {
+    const uint32_t y = (uint32_t)list[i];
+    const int32_t x = A.H[y];
+    if (is_lower(A, y, x) && A.status[x] == UNDEC) {
+      atomicAdd(ucnt + x, 1);
+      A.child[x] = (int32_t)y;
+    }
+  }
+  sync();
+  for (int64_t i = tid; i < len; i += stride) {
+    const int32_t x = list[i];
+    uint8_t k;
+    if (A.rootflag[x]) k = K_ROOT;
+    else if (ucnt[x] == 0) k = K_ACT;
+    else if (ucnt[x] == 1) k = K_UNARY;
+    else k = K_BRANCH;
+    A.kind[x] = k;
+    if (k == K_UNARY) A.jmp[0][x] = (uint32_t)A.child[x] | 0x80000000u;  // one NOT step
+  }
+  sync();
+  int passes = 1;
+  for (int64_t l = 1; l < len; l <<= 1) ++passes;
+  for (int p = 0; p < passes; ++p) {
+    const uint32_t *src = A.jmp[p & 1];
+    uint32_t *dst = A.jmp[(p & 1) ^ 1];
+    for (int64_t i = tid; i < len; i += stride) {
+      const int32_t x = list[i];
+      if (A.kind[x] != K_UNARY) continue;
+      const uint32_t e = src[x];
+      const int32_t y = (int32_t)(e & 0x7fffffffu);
+      if (A.kind[y] == K_UNARY) {
+        const uint32_t f = src[y];
+        dst[x] = (f & 0x7fffffffu) | ((e ^ f) & 0x80000000u);
+      } else {
+        dst[x] = e;
+      }
+    }
+    sync();
+  }
+  const uint32_t *fin = A.jmp[passes & 1];
+  for (int64_t i = tid; i < len; i += stride) {
+    const int32_t x = list[i];
+    const uint8_t k = A.kind[x];
+    int v = -1;  // 1 ACTIVE, 0 ROOT, -1 undecided
+    if (k == K_ROOT) v = 0;
+    else if (k == K_ACT) v = 1;
+    else if (k == K_UNARY) {
+      const uint32_t e = fin[x];
+      const uint8_t ky = A.kind[e & 0x7fffffffu];
+      if (ky == K_ROOT || ky == K_ACT) v = (ky == K_ACT) ^ (int)(e >> 31);
+    }
+    if (v >= 0) {
+      A.status[x] = v ? ACTIVE : ROOT;
+      if (v && is_lower(A, (uint32_t)x, A.H[x])) A.rootflag[A.H[x]] = 1;
+    }
+  }
+  sync();
+  const int64_t lim = (len + 31) & ~(int64_t)31;
+  for (int64_t i = tid; i < lim; i += stride) {
+    const int32_t u = i < len ? list[i] : 0;
+    const bool keep = i < len && A.status[u] == UNDEC;
+    append(out, out_cnt, keep, (uint32_t)u);
+  }
+  sync();
+  if (threadIdx.x == 0) *s_len = *(volatile unsigned *)out_cnt;
+  __syncthreads();
+  const int64_t nlen = *s_len;
+  for (int64_t i = tid; i < nlen; i += stride) A.blocked[out[i]] = 0;
+  sync();
+  for (int64_t i = tid; i < nlen; i += stride) {
+    const uint32_t y = (uint32_t)out[i];
+    const int32_t x = A.H[y];
+    if (is_lower(A, y, x)) A.blocked[x] = r_next;
+  }
+  sync();
+  return nlen;
+}
+
 __global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
   const unsigned nb = gridDim.x;
   const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -625,6 +747,18 @@ __global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
       if (gtid == 0) *A.rounds_out = r - 1;
       return;
     }
+    if (r % kComprEvery == 0) {  // long decision chains: compress the residual (counts as one round)
+      unsigned *cnt_c = round_counter(A, r);
+      if (gtid == 0) *round_counter(A, r + 1) = 0u;
+      len = compress_residual(A, A.wl[cur], len, A.wl[cur ^ 1], cnt_c, r + 1, gtid, gstride, GridSync{A.bar, nb},
+                              &s_len);
+      cur ^= 1;
+      ++r;
+      if (len == 0) {
+        if (gtid == 0) *A.rounds_out = r - 1;
+        return;
+      }
+    }
     if (len <= kSoloThreshold) break;
   }
   // ---- small residual: CTA 0 alone, block barriers only (same counter rotation)
@@ -651,6 +785,16 @@ __global__ void __launch_bounds__(kRoundBlock) k_rounds(RoundArgs A) {
     cur ^= 1;
     ++r;
     if (len == 0) break;
+    if (r % kComprEvery == 0) {
+      unsigned *cnt_c = round_counter(A, r);
+      if (threadIdx.x == 0) *round_counter(A, r + 1) = 0u;
+      __syncthreads();
+      len = compress_residual(A, A.wl[cur], len, A.wl[cur ^ 1], cnt_c, r + 1, threadIdx.x, blockDim.x, BlockSync{},
+                              &s_len);
+      cur ^= 1;
+      ++r;
+      if (len == 0) break;
+    }
   }
   if (threadIdx.x == 0) *A.rounds_out = r - 1;
 }
@@ -728,6 +872,7 @@ int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes) {
   b += ws_bytes(n, 1) * 2;      // status, rootflag
   b += ws_bytes(n, 4);          // blocked
   b += 2 * ws_bytes(n, 4);      // worklists
+  b += 3 * ws_bytes(n, 4) + ws_bytes(n, 1);  // residual compression: child, jmp[2], kind
   b += ws_bytes(4, 4) + ws_bytes(4, 4) + ws_bytes(4, 8);
   b += heavy_ws(n, nnz);
   b += scan_ws_bytes(n);
@@ -748,12 +893,17 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   int32_t *blocked = ws_take<int32_t>(ctx, n);
   int32_t *wl0 = ws_take<int32_t>(ctx, n);
   int32_t *wl1 = ws_take<int32_t>(ctx, n);
+  int32_t *child = ws_take<int32_t>(ctx, n);
+  uint32_t *jmp0 = ws_take<uint32_t>(ctx, n);
+  uint32_t *jmp1 = ws_take<uint32_t>(ctx, n);
+  uint8_t *kind = ws_take<uint8_t>(ctx, n);
   unsigned *cnt = ws_take<unsigned>(ctx, 4);
   unsigned *bar = ws_take<unsigned>(ctx, 4);
   int64_t *scal = ws_take<int64_t>(ctx, 4);  // [0] n_c, [1] rounds (int32 in low word), [2] long chain
   const bool full = u0 == 0 && u1 == n;
   int32_t *lab = full ? M : ws_take<int32_t>(ctx, n);
-  if (!status || !rootflag || !blocked || !wl0 || !wl1 || !cnt || !bar || !scal || !lab) {
+  if (!status || !rootflag || !blocked || !wl0 || !wl1 || !cnt || !bar || !scal || !lab || !child || !jmp0 || !jmp1 ||
+      !kind) {
     set_error("workspace under-reserved (mapping)");
     return HEC_EINVAL;
   }
@@ -771,6 +921,7 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   A.n = n; A.H = H; A.prio = prio; A.status = status; A.rootflag = rootflag; A.blocked = blocked;
   A.wl[0] = wl0; A.wl[1] = wl1; A.cnt = cnt; A.rounds_out = reinterpret_cast<int32_t *>(scal + 1);
   A.bar.count = bar; A.bar.gen = bar + 1;
+  A.child = child; A.kind = kind; A.jmp[0] = jmp0; A.jmp[1] = jmp1;
   static int occ = 0;
   if (!occ) {
     HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rounds, kRoundBlock, 0));

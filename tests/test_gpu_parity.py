@@ -222,6 +222,60 @@ def test_mapping_long_chain_identity_path(P, ctx):
     assert dt < 1.0, f"{dt:.3f} s"
 
 
+def test_mapping_long_rounds_reversed_path(P, ctx):
+    """Reverse visit order on a 2M-vertex path: Alg 3 pairs {2k, 2k+1} (SURVEY
+    §8(c) M1 closed form), but the decision chain is n long -- n/2 plain
+    resolution rounds.  The residual compression (pointer jumping with
+    parity along unary chains) must resolve it in well under a second."""
+    import time
+    n = 2_000_000
+    g = path_csr(n)
+    pr = np.arange(n, dtype=np.uint64)[::-1].copy()
+    dg, pt = dev(P, g), prio_tensor(pr)
+    P.hec_find_mapping_prio(ctx, dg, pt)  # warm-up
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    M, nc = P.hec_find_mapping_prio(ctx, dg, pt)
+    dt = time.perf_counter() - t0
+    assert nc == n // 2
+    assert np.array_equal(M.cpu().numpy(), np.arange(n) // 2)
+    assert dt < 1.0, f"{dt:.3f} s"
+
+
+@pytest.mark.parametrize("shape", ["broom", "caterpillar", "spiders"])
+def test_mapping_adversarial_trees(P, ctx, shape):
+    """Trees whose H-forest has long chains with side branches, visited in
+    adversarial orders (priority = depth from the far end), against the oracle."""
+    rng = np.random.default_rng({"broom": 41, "caterpillar": 42, "spiders": 43}[shape])
+    edges = []
+    if shape == "broom":      # a 30k path with a 2k-leaf fan at one end
+        L = 30000
+        edges += [(i, i + 1, 1) for i in range(L - 1)]
+        edges += [(L - 1, L + j, 1) for j in range(2000)]
+        n = L + 2000
+    elif shape == "caterpillar":  # a 20k spine, a pendant leaf at every third vertex
+        L = 20000
+        edges += [(i, i + 1, 2) for i in range(L - 1)]
+        leaves = list(range(0, L, 3))
+        edges += [(v, L + j, 1) for j, v in enumerate(leaves)]
+        n = L + len(leaves)
+    else:                     # 40 paths of random length hanging off a hub
+        n, nxt = 1, 1
+        for _ in range(40):
+            ln = int(rng.integers(100, 3000))
+            prev = 0
+            for _ in range(ln):
+                edges.append((prev, nxt, 1))
+                prev, nxt = nxt, nxt + 1
+        n = nxt
+    g = gg.from_edges(n, edges)
+    for order in (np.arange(n), np.arange(n)[::-1], rng.permutation(n)):
+        pr = o.prio_from_order(order)
+        M, nc = P.hec_find_mapping_prio(ctx, dev(P, g), prio_tensor(pr))
+        Mo, nco, _ = o.mapping(g, pr)
+        assert nc == nco and np.array_equal(M.cpu().numpy(), Mo)
+
+
 @pytest.mark.parametrize("which", ["c1", "c2", "rmat16", "random"])
 def test_mapping_parity_seeded(P, ctx, which):
     rng = np.random.default_rng(13)
