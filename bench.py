@@ -257,19 +257,24 @@ def main():
         if dist:
             dist.barrier()
 
+    comm = None
+    if world > 1:
+        from paper_conf_ipps_gilbertabmr21_b200 import dist as D
+        comm = D.Comm(None, dev)
+
     def hierarchy(graph):
-        """One full hierarchy: single GPU, or every level partitioned over the
-        ranks (H / M / coarse-row-count all-gathers)."""
+        """One full hierarchy: single GPU, or (N > 1) the levels of >= 64M fine
+        entries partitioned over the ranks inside libhec (coarsen_hierarchy_dist:
+        H / M all-gathers, coarse-row ranges, slices all-gathered so every rank
+        holds G_{l+1}); smaller levels replicated."""
         if world > 1:
-            from paper_conf_ipps_gilbertabmr21_b200.dist import coarsen_hierarchy_dist
-            return coarsen_hierarchy_dist(ctx, graph, cfg["cutoff"], gg.COARSEN_SEED)
+            return D.coarsen_hierarchy_dist(ctx, graph, cfg["cutoff"], gg.COARSEN_SEED, comm=comm)
         return P.coarsen_hierarchy(ctx, graph, cfg["cutoff"], gg.COARSEN_SEED)
 
     def step():
         h = hierarchy(dg)
         sizes = [(lv.graph.n, lv.graph.nnz) for lv in h.levels]
-        if world == 1:
-            h.free()
+        h.free()
         return sizes
 
     for _ in range(args.warmup):
@@ -360,8 +365,7 @@ def main():
                 o.copy_(x, non_blocking=True)
             sizes = torch.tensor([lv.graph.n for lv in h.levels], dtype=torch.int64)
             bo = sum(t.numel() * t.element_size() for t in outs) + sizes.numel() * 8
-            if world == 1:
-                h.free()
+            h.free()
             del hg
         e1.record(stream)
         torch.cuda.synchronize()
@@ -392,8 +396,9 @@ def main():
             "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz, "m0": m0,
                        "cutoff": cfg["cutoff"], "seed": gg.COARSEN_SEED,
-                       "parallelism": (f"partitioned x{world}: fine-vertex slices for heavy/M, "
-                                       "coarse-row ranges for construction, NCCL all-gathers")
+                       "parallelism": (f"partitioned x{world} (levels with >= 64M fine entries): fine-vertex "
+                                       "slices for heavy/M, coarse-row ranges for construction, NCCL all-gathers "
+                                       "through libhec's collective callback (gather_ms: their share)")
                        if world > 1 else "single",
                        "l2": f"inputs {(g.nnz * 8 + g.n * 12) / 1e9:.1f} GB > 126 MB L2 (no flush needed)",
                        "levels": [n for n, _ in levels], "gen_s": round(t_gen, 1)},
@@ -409,6 +414,7 @@ def main():
                                             else f"no ncu capture of these sources ({source_stamp()})"),
                          "peak_source": peak_src},
             "levels": per_level,
+            "gather_ms": prof.get("gather", {}).get("ms", 0.0) / args.steps,
             "phases": phases,
             "cpu_baseline": cpu,
             "e2e": e2e,

@@ -171,7 +171,8 @@ HEC_API void hec_hierarchy_free(hec_hierarchy *h);
  * summed device time, number of calls and the algorithmic bytes (compulsory
  * traffic: each input read once, each output written once).
  * Phases: "heavy" (a1), "rounds" (a3), "relabel" (a4+a5), "bucket" (a7),
- * "expand", "rows_skew", "rows" (a8/a9), "place" (a10), and inside
+ * "expand", "rows_skew", "rows" (a8/a9), "place" (a10), "gather" (the
+ * all-gathers of the multi-GPU calls), and inside
  * coarsen_hierarchy one "level" phase per level l spanning its mapping and
  * construction, with SURVEY §8(d)'s compulsory bytes
  *   B_l = 16 nnz + 8 nnz_c + 28 n + 12 n_c   (built level)
@@ -199,6 +200,59 @@ HEC_API int hec_debug_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H);
  * *rounds (host) receives the number of rounds.  prio NULL => hec_prio(seed, level). */
 HEC_API int hec_debug_roots(hec_ctx *ctx, const hec_graph *g, const uint64_t *prio,
                             uint64_t seed, int level, uint8_t *root, int *rounds);
+
+/* ----------------------------------------------- multi-GPU calls (§8(e)) */
+/* One process per GPU; every rank holds the whole input graph (replicated,
+ * e.g. generated or loaded on each rank) and calls the same function with the
+ * same arguments.  The only exchange step is an all-gather of equal-size byte
+ * blocks, supplied by the caller (NCCL through torch.distributed on a GPU box,
+ * gloo in tests), so the library needs no NCCL link of its own:
+ *   allgather(send, recv, bytes, stream, user): rank r's `bytes` bytes at
+ *   device pointer `send` land at recv + r * bytes on every rank, ordered on
+ *   `stream` (the context's); returns 0, or non-zero on failure (the library
+ *   call then returns HEC_ECUDA).
+ * Uneven pieces are padded to the largest one.  Results are bit-identical to
+ * the single-GPU calls (tests/test_gpu_dist.py). */
+typedef int (*hec_allgather_fn)(const void *send, void *recv, size_t bytes, hec_stream_t stream, void *user);
+typedef struct {
+  int32_t rank, world;          /* 0 <= rank < world */
+  hec_allgather_fn allgather;
+  void *user;
+} hec_comm;
+
+/* hec_find_mapping partitioned over the ranks: heavy neighbours of the rank's
+ * fine-vertex slice (the mapping's only edge stream, a1) -> all-gather H; the
+ * resolution rounds and the relabel (vertex-only, cheap) run on every rank;
+ * M of the slice -> all-gather M.  M (device int32[n]) is complete on every
+ * rank on return. */
+HEC_API int hec_find_mapping_dist(hec_ctx *ctx, const hec_graph *g, uint64_t seed, int level,
+                                  const hec_comm *comm, int32_t *M, int64_t *n_c);
+/* build_coarse_graph partitioned by coarse-row range (
+ * construction input "G, n, m, M, n_c" of Alg 6): the
+ * ranks split the coarse rows into contiguous ranges of about equal
+ * member-edge volume (identical on every rank), each builds its rows, the
+ * slices' entry counts are all-gathered and every rank derives the global row
+ * offsets.  gather_full = 1: the slices (row offsets, columns, weights, vertex
+ * weights) are all-gathered and every rank receives the whole G_c, stitched in
+ * C; gather_full = 0: *out holds the rank's slice only -- a CSR of rows
+ * [row_begin, row_end) with local row offsets -- placed by hec_csr_dist_slice. */
+HEC_API int build_coarse_graph_dist(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
+                                    const hec_comm *comm, int gather_full, hec_csr_owned **out);
+/* Placement of a slice from build_coarse_graph_dist(gather_full = 0): its rows
+ * [*row_begin, *row_end) of G_c, its first entry at global position
+ * *entry_offset, *nnz_total entries in all slices.  A whole graph reports
+ * [0, n_c), 0, nnz_c. */
+HEC_API int hec_csr_dist_slice(const hec_csr_owned *csr, int64_t *row_begin, int64_t *row_end,
+                               int64_t *entry_offset, int64_t *nnz_total);
+/* coarsen_hierarchy with every level whose fine graph has at least
+ * partition_min_nnz entries mapped and built by hec_find_mapping_dist and
+ * build_coarse_graph_dist(gather_full = 1); smaller levels run on every rank
+ * locally (no exchange: the construction of small graphs is launch-bound).
+ * Every rank receives the whole hierarchy, identical to coarsen_hierarchy.
+ * partition_min_nnz <= 0 partitions every level. */
+HEC_API int coarsen_hierarchy_dist(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
+                                   int64_t discard_below, int max_levels, const hec_comm *comm,
+                                   int64_t partition_min_nnz, hec_hierarchy **out);
 
 /* ------------------------------------------- multi-GPU building blocks (§8(e)) */
 /* The partitioned hierarchy level (one process per GPU; the collectives are the

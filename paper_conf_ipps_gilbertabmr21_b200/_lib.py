@@ -21,7 +21,8 @@ EXPORTS = [
     "hec_hierarchy_free", "hec_debug_heavy", "hec_debug_roots", "hec_build_rows_count",
     "hec_build_rows_write", "hec_heavy_range", "hec_mapping_from_heavy", "hec_balance_rows",
     "hec_ctx_set_profiling", "hec_ctx_profile_reset", "hec_ctx_profile",
-    "hec_ctx_launches",
+    "hec_ctx_launches", "hec_find_mapping_dist", "build_coarse_graph_dist", "hec_csr_dist_slice",
+    "coarsen_hierarchy_dist",
 ]
 
 
@@ -43,6 +44,14 @@ class HecPhaseTime(ctypes.Structure):
 
 
 ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+# int allgather(const void *send, void *recv, size_t bytes, stream, void *user)
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p,
+                                ctypes.c_void_p)
+
+
+class HecComm(ctypes.Structure):
+    _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("allgather", ALLGATHER_FN),
+                ("user", ctypes.c_void_p)]
 FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 
 _L = None
@@ -90,6 +99,11 @@ def load():
         "hec_ctx_profile_reset": (i32, [p]),
         "hec_ctx_profile": (i32, [p, ctypes.POINTER(HecPhaseTime), i32, ctypes.POINTER(i32)]),
         "hec_ctx_launches": (i64, [p]),
+        "hec_find_mapping_dist": (i32, [p, G, u64, i32, ctypes.POINTER(HecComm), p, ctypes.POINTER(i64)]),
+        "build_coarse_graph_dist": (i32, [p, G, p, i64, ctypes.POINTER(HecComm), i32, ctypes.POINTER(p)]),
+        "hec_csr_dist_slice": (i32, [p, ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i64),
+                                     ctypes.POINTER(i64)]),
+        "coarsen_hierarchy_dist": (i32, [p, G, i64, u64, i64, i32, ctypes.POINTER(HecComm), i64, ctypes.POINTER(p)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

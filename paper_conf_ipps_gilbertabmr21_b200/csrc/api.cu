@@ -145,31 +145,15 @@ static int begin_call(hec_ctx *ctx, size_t ws) {
 
 using namespace hec;
 
-struct hec_csr_owned {
-  hec_ctx *ctx;
-  CoarseOut c;
-};
-
-struct hec_hierarchy {
-  hec_ctx *ctx;
-  struct Level {
-    CoarseOut g;
-    int32_t *M;
-    int64_t n_fine;
-    int rounds;
-  };
-  std::vector<Level> levels;
-  int stop_reason = HEC_STOP_CUTOFF;
-  int64_t discarded_n_c = -1;
-};
-
-static void free_coarse(hec_ctx *ctx, CoarseOut &c) {
+namespace hec {
+void free_coarse(hec_ctx *ctx, CoarseOut &c) {
   dev_free(ctx, c.row_ptr);
   dev_free(ctx, c.col);
   dev_free(ctx, c.wgt);
   dev_free(ctx, c.vwgt);
   c = CoarseOut{};
 }
+}  // namespace hec
 
 extern "C" {
 
@@ -351,12 +335,68 @@ HEC_API int build_coarse_graph(hec_ctx *ctx, const hec_graph *g, const int32_t *
   if (!o) { set_error("out of host memory"); return HEC_ENOMEM; }
   o->ctx = ctx;
   int rc = build_coarse_impl(ctx, g, M, n_c, &o->c);
+  o->slice = DistSlice{0, n_c, 0, o->c.nnz_c};
   if (rc != HEC_OK) {
     free_coarse(ctx, o->c);
     delete o;
     return rc;
   }
   *out = o;
+  return HEC_OK;
+}
+
+HEC_API int hec_csr_dist_slice(const hec_csr_owned *csr, int64_t *row_begin, int64_t *row_end, int64_t *entry_offset,
+                               int64_t *nnz_total) {
+  if (!csr) { set_error("NULL argument"); return HEC_EINVAL; }
+  if (row_begin) *row_begin = csr->slice.row_begin;
+  if (row_end) *row_end = csr->slice.row_end;
+  if (entry_offset) *entry_offset = csr->slice.entry_offset;
+  if (nnz_total) *nnz_total = csr->slice.nnz_total;
+  return HEC_OK;
+}
+
+HEC_API int build_coarse_graph_dist(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
+                                    const hec_comm *comm, int gather_full, hec_csr_owned **out) {
+  if (!out) { set_error("out is NULL"); return HEC_EINVAL; }
+  *out = nullptr;
+  HEC_TRY(check_graph(g));
+  if (g->n > 0 && !M) { set_error("M is NULL"); return HEC_EINVAL; }
+  if (!comm || comm->world < 1 || comm->rank < 0 || comm->rank >= comm->world || !comm->allgather) {
+    set_error("build_coarse_graph_dist: invalid comm");
+    return HEC_EINVAL;
+  }
+  HEC_TRY(begin_call(ctx, ws_bytes_construct(g->n, g->nnz, n_c)));
+  if (ctx->validate) HEC_TRY(validate_graph(ctx, g));
+  hec_csr_owned *o = new (std::nothrow) hec_csr_owned();
+  if (!o) { set_error("out of host memory"); return HEC_ENOMEM; }
+  o->ctx = ctx;
+  int rc = build_coarse_dist_impl(ctx, g, M, n_c, comm, gather_full, &o->c, &o->slice);
+  if (rc != HEC_OK) {
+    free_coarse(ctx, o->c);
+    delete o;
+    return rc;
+  }
+  *out = o;
+  return HEC_OK;
+}
+
+HEC_API int hec_find_mapping_dist(hec_ctx *ctx, const hec_graph *g, uint64_t seed, int level, const hec_comm *comm,
+                                  int32_t *M, int64_t *n_c) {
+  HEC_TRY(check_graph(g));
+  if ((g->n > 0 && !M) || !n_c) { set_error("M / n_c is NULL"); return HEC_EINVAL; }
+  if (!comm || comm->world < 1 || comm->rank < 0 || comm->rank >= comm->world || !comm->allgather) {
+    set_error("hec_find_mapping_dist: invalid comm");
+    return HEC_EINVAL;
+  }
+  size_t ws = 0;
+  ws_bytes_mapping(g->n, g->nnz, &ws);
+  HEC_TRY(begin_call(ctx, ws));
+  if (ctx->validate) HEC_TRY(validate_graph(ctx, g));
+  MapResult r;
+  HEC_TRY(find_mapping_dist_impl(ctx, g, Prio{nullptr, splitmix64(seed + (uint64_t)level)}, comm, M, &r));
+  *n_c = r.n_c;
+  ctx->stats.rounds = r.rounds;
+  ctx->stats.n_c = r.n_c;
   return HEC_OK;
 }
 
@@ -377,8 +417,26 @@ HEC_API void hec_csr_free(hec_csr_owned *csr) {
   delete csr;
 }
 
+static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed, int64_t discard_below,
+                          int max_levels, const hec_comm *comm, int64_t min_nnz, hec_hierarchy **out);
+
 HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
                               int64_t discard_below, int max_levels, hec_hierarchy **out) {
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, out);
+}
+
+HEC_API int coarsen_hierarchy_dist(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
+                                   int64_t discard_below, int max_levels, const hec_comm *comm,
+                                   int64_t partition_min_nnz, hec_hierarchy **out) {
+  if (!comm || comm->world < 1 || comm->rank < 0 || comm->rank >= comm->world || !comm->allgather) {
+    set_error("coarsen_hierarchy_dist: invalid comm");
+    return HEC_EINVAL;
+  }
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, comm, partition_min_nnz, out);
+}
+
+static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed, int64_t discard_below,
+                          int max_levels, const hec_comm *comm, int64_t min_nnz, hec_hierarchy **out) {
   if (!out) { set_error("out is NULL"); return HEC_EINVAL; }
   *out = nullptr;
   HEC_TRY(check_graph(g0));
@@ -411,8 +469,12 @@ HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff,
     rc = ws_reserve(ctx, ws);
     ctx->ws.used = 0;
     MapResult r;
-    if (rc == HEC_OK) rc = find_mapping_impl(ctx, &cur, Prio{nullptr, splitmix64(seed + (uint64_t)level)}, M,
-                                             nullptr, nullptr, &r);
+    // multi-GPU: only levels with at least min_nnz fine entries are partitioned
+    const bool part = comm && comm->world > 1 && cur.nnz >= min_nnz;
+    const Prio prio{nullptr, splitmix64(seed + (uint64_t)level)};
+    if (rc == HEC_OK)
+      rc = part ? find_mapping_dist_impl(ctx, &cur, prio, comm, M, &r)
+                : find_mapping_impl(ctx, &cur, prio, M, nullptr, nullptr, &r);
     if (rc != HEC_OK) { dev_free(ctx, M); break; }
     ctx->stats.rounds = r.rounds;
     ctx->stats.n_c = r.n_c;
@@ -434,7 +496,14 @@ HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff,
     L.M = M;
     L.n_fine = cur.n;
     L.rounds = r.rounds;
-    if (rc == HEC_OK) rc = build_coarse_impl(ctx, &cur, M, r.n_c, &L.g);
+    if (rc == HEC_OK) {
+      if (part) {
+        DistSlice sl;
+        rc = build_coarse_dist_impl(ctx, &cur, M, r.n_c, comm, 1, &L.g, &sl);
+      } else {
+        rc = build_coarse_impl(ctx, &cur, M, r.n_c, &L.g);
+      }
+    }
     if (rc != HEC_OK) {
       free_coarse(ctx, L.g);
       dev_free(ctx, M);

@@ -371,6 +371,7 @@ struct CoarseOut {
   int32_t *col = nullptr, *wgt = nullptr, *vwgt = nullptr;
 };
 size_t ws_bytes_construct(int64_t n, int64_t nnz, int64_t n_c);
+void free_coarse(hec_ctx *ctx, CoarseOut &c);
 // Coarse rows [a_lo, a_hi) only (a_hi < 0: all rows); out->n_c = a_hi - a_lo and
 // row_ptr/vwgt are indexed from a_lo, row_ptr[0] = 0 (range partition, §8(e)).
 int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
@@ -383,5 +384,36 @@ int mapping_from_heavy_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, 
 // Member-edge volume U(a) of every coarse row (int64, device) for range balancing.
 int row_volume_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, int64_t *U);
 int validate_graph(hec_ctx *ctx, const hec_graph *g);
+// Coarse rows split into `parts` ranges of about equal member-edge volume (host bounds[parts+1]).
+int balance_rows_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, int parts, int64_t *bounds);
+// Multi-GPU (dist.cu): mapping with H / M all-gathered; construction by coarse-row range.
+int find_mapping_dist_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, const hec_comm *comm, int32_t *M,
+                           MapResult *res);
+constexpr int kMaxWorld = 64;  // ranks of the multi-GPU calls
+struct DistSlice {
+  int64_t row_begin = 0, row_end = 0, entry_offset = 0, nnz_total = 0;
+};
+int build_coarse_dist_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, const hec_comm *comm,
+                           int gather_full, CoarseOut *out, DistSlice *slice);
 
 }  // namespace hec
+
+// Owned results (opaque in hec.h).
+struct hec_csr_owned {
+  hec_ctx *ctx;
+  hec::CoarseOut c;
+  hec::DistSlice slice;  // rows / entries this result holds (the whole graph unless a dist slice)
+};
+
+struct hec_hierarchy {
+  hec_ctx *ctx;
+  struct Level {
+    hec::CoarseOut g;
+    int32_t *M;
+    int64_t n_fine;
+    int rounds;
+  };
+  std::vector<Level> levels;
+  int stop_reason = HEC_STOP_CUTOFF;
+  int64_t discarded_n_c = -1;
+};

@@ -1,6 +1,11 @@
-"""Host-side logic of the multi-GPU path on CPU: world_size 2,
-gloo backend, 127.0.0.1.  The collectives and range arithmetic used by
-paper_conf_ipps_gilbertabmr21_b200.dist, without a GPU."""
+"""Host side of the multi-GPU path on CPU: world_size 2, gloo,
+127.0.0.1.  libhec's dist calls exchange data only through the all-gather
+callback of paper_conf_ipps_gilbertabmr21_b200.dist; here that callback (byte
+views of raw pointers, equal-block all-gather, rank order) is checked without a
+GPU, together with the fine-vertex slice arithmetic."""
+import ctypes
+
+import numpy as np
 import torch
 import torch.multiprocessing as mp
 
@@ -20,35 +25,40 @@ def test_even_ranges():
 
 def _worker(rank, world, port, q):
     import torch.distributed as dist
-    from paper_conf_ipps_gilbertabmr21_b200.dist import all_gather_scalars, all_gather_uneven, even_ranges
+    from paper_conf_ipps_gilbertabmr21_b200 import _lib
+    from paper_conf_ipps_gilbertabmr21_b200.dist import allgather_bytes
     init(rank, world, port)
     try:
-        n = 11
-        rng = even_ranges(n, world)
-        lo, hi = rng[rank]
-        full = torch.arange(n, dtype=torch.int64) * 3 + 1
-        mine = full[lo:hi].clone()
-        got = all_gather_uneven(mine, [b - a for a, b in rng])
-        assert torch.equal(got, full)
-        # int32 pieces of very different sizes, one empty
-        sizes = [5, 0] if world == 2 else [5] * world
-        piece = torch.full((sizes[rank],), rank + 7, dtype=torch.int32)
-        got = all_gather_uneven(piece, sizes)
-        exp = torch.cat([torch.full((s,), r + 7, dtype=torch.int32) for r, s in enumerate(sizes)])
-        assert torch.equal(got, exp)
-        sc = all_gather_scalars([rank * 10, rank + 1])
-        assert sc == [[r * 10, r + 1] for r in range(world)]
-        # global offsets of slices = exclusive prefix of the gathered totals
-        totals = [v[0] for v in all_gather_scalars([100 + rank])]
-        assert sum(totals[:rank]) == sum(100 + r for r in range(rank))
+        cpu = torch.device("cpu")
+        # equal blocks of raw host bytes, gathered in rank order
+        nb = 13
+        send = np.full(nb, 40 + rank, np.uint8)
+        recv = np.zeros(nb * world, np.uint8)
+        allgather_bytes(send.ctypes.data, recv.ctypes.data, nb, None, cpu)
+        assert np.array_equal(recv, np.repeat(np.arange(40, 40 + world, dtype=np.uint8), nb))
+        # int64 payloads (the slices' entry counts) through the C callback type
+        calls = []
+
+        def cb(s, r, n, stream, user):
+            calls.append(n)
+            allgather_bytes(s, r, int(n), None, cpu)
+            return 0
+        fn = _lib.ALLGATHER_FN(cb)
+        mine = np.array([1000 + rank], np.int64)
+        got = np.zeros(world, np.int64)
+        assert fn(mine.ctypes.data, got.ctypes.data, 8, None, None) == 0
+        assert got.tolist() == [1000 + r for r in range(world)] and calls == [8]
+        # zero-length blocks are legal
+        allgather_bytes(0, 0, 0, None, cpu)
         q.put((rank, "ok"))
     except Exception as e:  # noqa: BLE001
-        q.put((rank, repr(e)))
+        import traceback
+        q.put((rank, traceback.format_exc()))
     finally:
         dist.destroy_process_group()
 
 
-def test_gloo_world2_collectives():
+def test_gloo_world2_allgather_callback():
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = free_port()

@@ -1,6 +1,8 @@
-"""Partitioned hierarchy on the GPU: two ranks (gloo, both on
-cuda:0 — the driver's box has one GPU) run coarsen_hierarchy_dist; every level
-must equal the single-GPU coarsen_hierarchy bit for bit."""
+"""Multi-GPU calls (include/hec.h: hec_find_mapping_dist,
+build_coarse_graph_dist, coarsen_hierarchy_dist) on the GPU: two ranks over
+gloo, both on cuda:0 (the driver's box has one GPU), the all-gather supplied
+by paper_conf_ipps_gilbertabmr21_b200.dist.  Every result must equal the
+single-GPU call bit for bit."""
 import os
 
 import numpy as np
@@ -26,24 +28,35 @@ def _graph(which):
 def _worker(rank, world, port, which, outdir, q):
     import torch.distributed as dist
     import paper_conf_ipps_gilbertabmr21_b200 as P
-    from paper_conf_ipps_gilbertabmr21_b200.dist import coarsen_hierarchy_dist
+    from paper_conf_ipps_gilbertabmr21_b200 import dist as D
     try:
         torch.cuda.set_device(0)
         init(rank, world, port, "gloo")
         g, cutoff = _graph(which)
         ctx = P.Context()
-        H = coarsen_hierarchy_dist(ctx, P.DeviceGraph.from_host(g), cutoff, SEED)
-        if rank == 0:
-            arrs = {"stop": np.array([H.stop_reason, H.discarded_n_c]), "nlev": np.array([len(H.levels)])}
-            for i, lv in enumerate(H.levels):
-                rp, col, wgt, vw = lv.graph.to_host()
-                arrs.update({f"M{i}": lv.M.cpu().numpy(), f"rp{i}": rp, f"col{i}": col, f"wgt{i}": wgt,
-                             f"vw{i}": vw})
-            np.savez(os.path.join(outdir, f"{which}.npz"), **arrs)
+        comm = D.Comm(None, torch.device("cuda", 0))
+        dg = P.DeviceGraph.from_host(g)
+        arrs = {}
+        # whole hierarchy, every level partitioned
+        H = D.coarsen_hierarchy_dist(ctx, dg, cutoff, SEED, comm=comm, partition_min_nnz=0)
+        arrs.update({"stop": np.array([H.stop_reason, H.discarded_n_c]), "nlev": np.array([len(H.levels)])})
+        for i, lv in enumerate(H.levels):
+            rp, col, wgt, vw = lv.graph.to_host()
+            arrs.update({f"M{i}": lv.M.cpu().numpy(), f"rp{i}": rp, f"col{i}": col, f"wgt{i}": wgt, f"vw{i}": vw})
+        # level 0 by the single calls: mapping, then the rank's slice of G_1
+        M, nc = D.hec_find_mapping_dist(ctx, dg, SEED, 0, comm)
+        sl = D.build_coarse_graph_dist(ctx, dg, M, nc, comm, gather_full=False)
+        rp, col, wgt, vw = sl.graph.to_host()
+        arrs.update({"sM": M.cpu().numpy(), "snc": np.array([nc]), "srows": np.array(sl.rows),
+                     "soff": np.array([sl.entry_offset, sl.nnz_total]), "srp": rp, "scol": col, "swgt": wgt,
+                     "svw": vw})
+        np.savez(os.path.join(outdir, f"{which}_{rank}.npz"), **arrs)
         dist.barrier()
+        sl.free()
+        H.free()
         ctx.close()
         q.put((rank, "ok"))
-    except Exception as e:  # noqa: BLE001
+    except Exception:  # noqa: BLE001
         import traceback
         q.put((rank, traceback.format_exc()))
     finally:
@@ -52,7 +65,7 @@ def _worker(rank, world, port, which, outdir, q):
 
 
 @pytest.mark.parametrize("which", ["c1", "rmat14", "mesh27"])
-def test_dist_hierarchy_matches_single_gpu(which, tmp_path):
+def test_dist_matches_single_gpu(which, tmp_path):
     import paper_conf_ipps_gilbertabmr21_b200 as P
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -64,13 +77,29 @@ def test_dist_hierarchy_matches_single_gpu(which, tmp_path):
     for p in procs:
         p.join(timeout=60)
     assert res == {0: "ok", 1: "ok"}, res
-    d = np.load(tmp_path / f"{which}.npz")
     g, cutoff = _graph(which)
     c = P.Context()
-    H = P.coarsen_hierarchy(c, P.DeviceGraph.from_host(g), cutoff, SEED)
-    assert int(d["nlev"][0]) == len(H.levels) and int(d["stop"][0]) == H.stop_reason
-    for i, lv in enumerate(H.levels):
-        rp, col, wgt, vw = lv.graph.to_host()
-        assert np.array_equal(d[f"M{i}"], lv.M.cpu().numpy())
-        assert np.array_equal(d[f"rp{i}"], rp) and np.array_equal(d[f"col{i}"], col)
-        assert np.array_equal(d[f"wgt{i}"], wgt) and np.array_equal(d[f"vw{i}"], vw)
+    dg = P.DeviceGraph.from_host(g)
+    H = P.coarsen_hierarchy(c, dg, cutoff, SEED)
+    M0, nc0 = P.hec_find_mapping(c, dg, SEED, 0)
+    G1 = P.build_coarse_graph(c, dg, M0, nc0)
+    rp1, col1, wgt1, vw1 = G1.graph.to_host()
+    covered = 0
+    for rank in range(2):
+        d = np.load(tmp_path / f"{which}_{rank}.npz")
+        assert int(d["nlev"][0]) == len(H.levels) and int(d["stop"][0]) == H.stop_reason
+        for i, lv in enumerate(H.levels):
+            rp, col, wgt, vw = lv.graph.to_host()
+            assert np.array_equal(d[f"M{i}"], lv.M.cpu().numpy())
+            assert np.array_equal(d[f"rp{i}"], rp) and np.array_equal(d[f"col{i}"], col)
+            assert np.array_equal(d[f"wgt{i}"], wgt) and np.array_equal(d[f"vw{i}"], vw)
+        assert np.array_equal(d["sM"], M0.cpu().numpy()) and int(d["snc"][0]) == nc0
+        a0, a1 = (int(x) for x in d["srows"])
+        off, tot = (int(x) for x in d["soff"])
+        assert tot == G1.graph.nnz and off == rp1[a0]
+        assert np.array_equal(d["srp"] + off, rp1[a0:a1 + 1])
+        k = int(d["srp"][-1])
+        assert np.array_equal(d["scol"][:k], col1[off:off + k]) and np.array_equal(d["swgt"][:k], wgt1[off:off + k])
+        assert np.array_equal(d["svw"][:a1 - a0], vw1[a0:a1])
+        covered += a1 - a0
+    assert covered == nc0
