@@ -310,7 +310,16 @@ __device__ __forceinline__ void seg_load(const SegArgs &A, int64_t k, int (&cc)[
     for (int j = 0; j < 4; ++j) {
       const int64_t e0 = es + 16 * lane + 4 * j;
       int4 c = make_int4(0, 0, 0, 0), w = make_int4(0, 0, 0, 0);
-      if (interior || (e0 + 3 >= elo && e0 < ehi)) { c = __ldcs(c4 + j); w = __ldcs(w4 + j); }
+      if (interior || (e0 >= elo && e0 + 3 < ehi)) {
+        c = __ldcs(c4 + j);
+        w = __ldcs(w4 + j);
+      } else if (e0 + 3 >= elo && e0 < ehi) {  // a group cut by the range: only its in-range entries
+        const int32_t *cs = reinterpret_cast<const int32_t *>(c4 + j), *ws = reinterpret_cast<const int32_t *>(w4 + j);
+        if (e0 >= elo && e0 < ehi) { c.x = __ldcs(cs); w.x = __ldcs(ws); }
+        if (e0 + 1 >= elo && e0 + 1 < ehi) { c.y = __ldcs(cs + 1); w.y = __ldcs(ws + 1); }
+        if (e0 + 2 >= elo && e0 + 2 < ehi) { c.z = __ldcs(cs + 2); w.z = __ldcs(ws + 2); }
+        if (e0 + 3 >= elo && e0 + 3 < ehi) { c.w = __ldcs(cs + 3); w.w = __ldcs(ws + 3); }
+      }
       cc[4 * j] = c.x; cc[4 * j + 1] = c.y; cc[4 * j + 2] = c.z; cc[4 * j + 3] = c.w;
       ww[4 * j] = w.x; ww[4 * j + 1] = w.y; ww[4 * j + 2] = w.z; ww[4 * j + 3] = w.w;
     }
