@@ -1116,18 +1116,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   A.mstart = mstart;
   A.idx32 = idx32;
 
-  static bool attr = false;
-  if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(PartSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_part_write, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(PartSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_bucket_fallback, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(FbSmem)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_dense_accum2, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)(4 * kDenseMax)));
-    attr = true;
-  }
+  int occ_unused = 0;  // dynamic shared-memory opt-ins (cached per context)
+  HEC_TRY(kernel_occupancy(ctx, k_part_count, kT, sizeof(PartSmem), &occ_unused));
+  HEC_TRY(kernel_occupancy(ctx, k_part_write, kT, sizeof(PartSmem), &occ_unused));
+  HEC_TRY(kernel_occupancy(ctx, k_bucket_fallback, kT, sizeof(FbSmem), &occ_unused));
+  HEC_TRY(kernel_occupancy(ctx, k_dense_accum2, kT, 4 * (size_t)kDenseMax, &occ_unused));
 
   const bool direct = getenv("HEC_NO_DRANK") == nullptr;  // test hook: bins through the hash-rank kernels
   int ph_rows = -1;

@@ -292,12 +292,9 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
 
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo) {
   constexpr int NT = 512;
-  static bool attr = false;
   const size_t smem = sizeof(HrSmem<NT>);
-  if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank_big<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    attr = true;
-  }
+  int occ = 1;
+  HEC_TRY(kernel_occupancy(ctx, k_hrank_big<NT>, NT, smem, &occ));
   int64_t grid = (int64_t)ctx->num_sms * 2;
   if (A.nblocks < grid) grid = A.nblocks;
   if (grid < 1) return HEC_OK;
@@ -527,13 +524,13 @@ int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, ui
   k_zero_u32<<<ctx->num_sms, 256, 0, ctx->stream>>>(done, nsplit, 1);
   HEC_LAUNCH_CHECK();
   int occ = 1;
-  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank, kDrT, 0));
-  int64_t grid = (int64_t)ctx->num_sms * (occ < 1 ? 1 : occ);
+  HEC_TRY(kernel_occupancy(ctx, k_drank, kDrT, 0, &occ));
+  int64_t grid = (int64_t)ctx->num_sms * occ;
   if (A.nblocks < grid) grid = A.nblocks;
   k_drank<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();
-  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_drank_chunks, kDrT, 0));
-  grid = (int64_t)ctx->num_sms * (occ < 1 ? 1 : occ);
+  HEC_TRY(kernel_occupancy(ctx, k_drank_chunks, kDrT, 0, &occ));
+  grid = (int64_t)ctx->num_sms * occ;
   k_drank_chunks<<<(unsigned)grid, kDrT, 0, ctx->stream>>>(A, dc, ndc, gacc, done);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
@@ -541,15 +538,9 @@ int launch_drank(hec_ctx *ctx, const RowsArgs &A, RbmItem *dc, unsigned *ndc, ui
 
 template <int NT, int PER = 8>
 static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
-  static bool attr = false;
-  static int occ = 1;
   const size_t smem = sizeof(HrSmem<NT, PER>);
-  if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_hrank<NT, PER>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_hrank<NT, PER>, NT, smem));
-    if (occ < 1) occ = 1;
-    attr = true;
-  }
+  int occ = 1;
+  HEC_TRY(kernel_occupancy(ctx, k_hrank<NT, PER>, NT, smem, &occ));
   int64_t grid = (int64_t)ctx->num_sms * occ;
   if (A.nblocks < grid) grid = A.nblocks;
   if (grid < 1) return HEC_OK;

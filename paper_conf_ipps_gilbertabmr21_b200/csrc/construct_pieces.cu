@@ -502,16 +502,10 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
 // Persistent: one grid of resident CTAs; the list length is read on the device.
 // Keys of row pieces pack (row, b) into 32 bits while n_c <= 2^26.
 int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket) {
-  static int occ[2] = {0, 0};
   constexpr size_t smem = sizeof(WarpTab) * kPW;
-  if (!occ[0]) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_pieces<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_pieces<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_pieces<false>, kPW * 32, smem));
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_pieces<true>, kPW * 32, smem));
-    if (occ[0] < 1) occ[0] = 1;
-    if (occ[1] < 1) occ[1] = 1;
-  }
+  int occ[2] = {1, 1};
+  HEC_TRY(kernel_occupancy(ctx, k_pieces<false>, kPW * 32, smem, &occ[0]));
+  HEC_TRY(kernel_occupancy(ctx, k_pieces<true>, kPW * 32, smem, &occ[1]));
   // (HEC_FORCE_WIDE_KEYS: test hook that exercises the 64-bit key path on small graphs)
   const bool wide_keys = A.L.n_c > (1ll << KeyTraits<uint32_t>::kShift) || getenv("HEC_FORCE_WIDE_KEYS") != nullptr;
   int64_t grid = (int64_t)ctx->num_sms * occ[wide_keys ? 1 : 0];

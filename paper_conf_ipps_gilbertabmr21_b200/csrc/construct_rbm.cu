@@ -205,11 +205,8 @@ __global__ void __launch_bounds__(kRbmT, 1) k_rbm(RowsArgs A) {
 }
 
 int launch_rbm(hec_ctx *ctx, const RowsArgs &A) {
-  static bool attr = false;
-  if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_rbm, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(RbmSmem)));
-    attr = true;
-  }
+  int occ = 1;
+  HEC_TRY(kernel_occupancy(ctx, k_rbm, kRbmT, sizeof(RbmSmem), &occ));
   int64_t grid = ctx->num_sms;  // one CTA per SM (shared-memory bound); items read from *A.nlist
   if (A.nblocks < grid) grid = A.nblocks;
   if (grid < 1) return HEC_OK;

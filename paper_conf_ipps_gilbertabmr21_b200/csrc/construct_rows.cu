@@ -465,19 +465,9 @@ int launch_place(hec_ctx *ctx, const RowsArgs &A) {
 }
 
 int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide) {
-  static int occ[2] = {0, 0};
-  if (!occ[0]) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_rows<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(RowsSmemT<false>)));
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_rows<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(RowsSmemT<true>)));
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_rows<false>, kT,
-                                                               sizeof(RowsSmemT<false>)));
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_rows<true>, kT,
-                                                               sizeof(RowsSmemT<true>)));
-    if (occ[0] < 1) occ[0] = 1;
-    if (occ[1] < 1) occ[1] = 1;
-  }
+  int occ[2] = {1, 1};
+  HEC_TRY(kernel_occupancy(ctx, k_rows<false>, kT, sizeof(RowsSmemT<false>), &occ[0]));
+  HEC_TRY(kernel_occupancy(ctx, k_rows<true>, kT, sizeof(RowsSmemT<true>), &occ[1]));
   // persistent; the list length is read on the device
   int64_t grid = (int64_t)ctx->num_sms * occ[wide ? 1 : 0];
   if (A.nblocks < grid) grid = A.nblocks;

@@ -111,6 +111,9 @@ struct hec_ctx {
     int64_t calls = 0;
   };
   std::vector<PhaseAcc> prof_acc;
+  // launch setup per kernel (hec::kernel_occupancy): a context is bound to one
+  // device, so the cache is per device by construction
+  std::vector<std::pair<const void *, int>> kcache;
 };
 
 namespace hec {
@@ -136,6 +139,28 @@ T *ws_take(hec_ctx *ctx, size_t count) { return arena_take<T>(ctx->ws, count); }
 inline size_t ws_bytes(size_t count, size_t elem) { return align_up(count * elem, 256) + 256; }
 
 int read_scalars(hec_ctx *ctx, const int64_t *dev, int count, int64_t *host_out);
+
+// Launch setup of a kernel on the context's device, cached in the context:
+// the dynamic shared-memory opt-in (when smem > 48 KB) and the resident CTAs
+// per SM for (threads, smem).  Each kernel is always launched with the same
+// (threads, smem) at its call site.
+template <typename K>
+int kernel_occupancy(hec_ctx *ctx, K kernel, int threads, size_t smem, int *occ) {
+  const void *key = reinterpret_cast<const void *>(kernel);
+  for (const auto &e : ctx->kcache)
+    if (e.first == key) {
+      *occ = e.second;
+      return HEC_OK;
+    }
+  if (smem > 48 * 1024)
+    HEC_CUDA_TRY(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int o = 0;
+  HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kernel, threads, smem));
+  if (o < 1) o = 1;
+  ctx->kcache.emplace_back(key, o);
+  *occ = o;
+  return HEC_OK;
+}
 
 // Phase timing: returns a handle for phase_end (-1 when profiling is off).
 int phase_begin(hec_ctx *ctx, const char *name, double bytes);

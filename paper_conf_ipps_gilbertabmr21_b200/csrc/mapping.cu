@@ -500,12 +500,9 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
     k_span_coords<<<nblk(nspans + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, x0, off, nspans, cx);
     HEC_LAUNCH_CHECK();
     SegArgs SA{n, nnz, rp, ebase, u0, x0, off, nspans, g->col - off, g->wgt - off, cx, H, head, mid};
-    static int occ[2] = {0, 0};
-    if (!occ[vec]) {
-      if (vec) HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], k_heavy_seg<true>, 32 * kSegWarps, 0));
-      else HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], k_heavy_seg<false>, 32 * kSegWarps, 0));
-      if (occ[vec] < 1) occ[vec] = 1;
-    }
+    int occ[2] = {1, 1};
+    if (vec) HEC_TRY(kernel_occupancy(ctx, k_heavy_seg<true>, 32 * kSegWarps, 0, &occ[1]));
+    else HEC_TRY(kernel_occupancy(ctx, k_heavy_seg<false>, 32 * kSegWarps, 0, &occ[0]));
     int64_t grid = (int64_t)ctx->num_sms * occ[vec];
     const int64_t want = (nspans + kSegWarps - 1) / kSegWarps;
     if (want < grid) grid = want;
@@ -523,12 +520,8 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
   if (!cx || !head || !mid) { set_error("workspace under-reserved (heavy)"); return HEC_EINVAL; }
   k_tile_coords<<<nblk(ntiles + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, ntiles, cx);
   HEC_LAUNCH_CHECK();
-  static bool attr = false;
-  if (!attr) {
-    HEC_CUDA_TRY(cudaFuncSetAttribute(k_heavy, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)sizeof(HeavySmem)));
-    attr = true;
-  }
+  int occ_tiles = 1;
+  HEC_TRY(kernel_occupancy(ctx, k_heavy, kHvBlock, sizeof(HeavySmem), &occ_tiles));
   k_heavy<<<(unsigned)ntiles, kHvBlock, sizeof(HeavySmem), ctx->stream>>>(
       n, nnz, rp, ebase, u0, ebase & 3, g->col + (ebase & ~(int64_t)3), g->wgt + (ebase & ~(int64_t)3), cx, H,
       head, mid);
@@ -931,11 +924,8 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   A.wl[0] = wl0; A.wl[1] = wl1; A.cnt = cnt; A.rounds_out = reinterpret_cast<int32_t *>(scal + 1);
   A.bar.count = bar; A.bar.gen = bar + 1;
   A.child = child; A.kind = kind; A.jmp[0] = jmp0; A.jmp[1] = jmp1;
-  static int occ = 0;
-  if (!occ) {
-    HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rounds, kRoundBlock, 0));
-    if (occ < 1) occ = 1;
-  }
+  int occ = 1;
+  HEC_TRY(kernel_occupancy(ctx, k_rounds, kRoundBlock, 0, &occ));
   int64_t want = (n + kRoundBlock - 1) / kRoundBlock;
   int64_t grid = (int64_t)ctx->num_sms * occ;
   if (want < grid) grid = want < 1 ? 1 : want;
