@@ -41,6 +41,24 @@ int oracle_mapping(int64_t n, const int64_t *row_ptr, const int32_t *col,
                    const int32_t *wgt, const uint64_t *prio, int32_t *M,
                    int64_t *n_c, uint8_t *root);
 
+/* HEC3 (Alg 5): the order-free second phase of HEC.
+ * Mutual heavy neighbours collapse onto the smaller id (l.5-8), every heavy
+ * neighbour not yet mapped becomes its own root (l.9-12), the remaining
+ * vertices inherit their heavy neighbour's (l.13-16), pointer jumping to the
+ * root (l.17-21), FINDUNIQANDRELABEL by ascending root id (l.22, reading Z3).
+ * P is the identity (reading Z17: Alg 5's O only renames vertices).
+ * M (out, n), *n_c (out), root (out, optional, n bytes). */
+int oracle_mapping_hec3(int64_t n, const int64_t *row_ptr, const int32_t *col,
+                        const int32_t *wgt, int32_t *M, int64_t *n_c, uint8_t *root);
+
+/* HEM (Alg 2) verbatim: vertices visited in ascending prio;
+ * an unmatched u takes its heaviest unmatched neighbour (strict ">" from 0:
+ * the smallest id among equal maxima) or stays a singleton.  Coarse ids by
+ * ascending root id, the root being the visiting vertex u (reading Z3). */
+int oracle_mapping_hem(int64_t n, const int64_t *row_ptr, const int32_t *col,
+                       const int32_t *wgt, const uint64_t *prio, int32_t *M,
+                       int64_t *n_c, uint8_t *root);
+
 /* Output arrays are caller-allocated with the upper bounds row_ptr_c[n_c+1],
  * col_c[nnz], wgt_c[nnz], vwgt_c[n_c]; *nnz_c receives the coarse entry count.
  * *intra receives the directed weight of dropped self-loops (conservation). */
