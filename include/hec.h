@@ -128,6 +128,25 @@ HEC_API int hec_find_mapping(hec_ctx *ctx, const hec_graph *g, uint64_t seed, in
 HEC_API int hec_find_mapping_prio(hec_ctx *ctx, const hec_graph *g, const uint64_t *prio,
                                   int32_t *M, int64_t *n_c);
 
+/* The paper's other FINDCOARSEMAPPING methods, same
+ * contract as hec_find_mapping (M device int32[n], *n_c host, one sync):
+ *   HEC_MAP_HEC   Alg 3 (the default of every other call)
+ *   HEC_MAP_HEC3  Alg 5 (L248-273): mutual heavy neighbours collapse onto the
+ *                 smaller id, vertices with in-degree > 0 in the heavy-neighbour
+ *                 pseudoforest are roots, the others inherit; order-free (seed
+ *                 and level are ignored)
+ *   HEC_MAP_HEM   Alg 2 (L73-97): heavy-edge matching in the hec_prio visit
+ *                 order, the heaviest *unmatched* neighbour (ties -> smallest
+ *                 id), identical to the sequential algorithm (root = the
+ *                 visiting vertex); coarsening ratio <= 2 (L61)
+ * Coarse ids ascend with the aggregates' roots (FINDUNIQANDRELABEL, reading Z3). */
+enum { HEC_MAP_HEC = 0, HEC_MAP_HEC3 = 1, HEC_MAP_HEM = 2 };
+HEC_API int hec_find_mapping_method(hec_ctx *ctx, const hec_graph *g, int method, uint64_t seed, int level,
+                                    int32_t *M, int64_t *n_c);
+/* Same with explicit device priorities (test hook, as hec_find_mapping_prio). */
+HEC_API int hec_find_mapping_method_prio(hec_ctx *ctx, const hec_graph *g, int method, const uint64_t *prio,
+                                         int32_t *M, int64_t *n_c);
+
 /* --------------------------------------------- north-star call 2: construction */
 typedef struct hec_csr_owned hec_csr_owned; /* device CSR owned by the library */
 
@@ -154,6 +173,10 @@ typedef struct hec_hierarchy hec_hierarchy;
  * discard_below <= 0 selects the paper's 10; max_levels <= 0 selects 200. */
 HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
                               int64_t discard_below, int max_levels, hec_hierarchy **out);
+/* coarsen_hierarchy with the mapping method of every level chosen by `method`
+ * (HEC_MAP_*; coarsen_hierarchy == coarsen_hierarchy_ex(..., HEC_MAP_HEC, ...)). */
+HEC_API int coarsen_hierarchy_ex(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
+                                 int64_t discard_below, int max_levels, int method, hec_hierarchy **out);
 HEC_API int hec_hierarchy_levels(const hec_hierarchy *h);
 /* i in [1, levels]: view of G_i, device pointer to M_i (length n_{i-1}), n_{i-1}. */
 HEC_API int hec_hierarchy_level(const hec_hierarchy *h, int i, hec_graph *g_i,

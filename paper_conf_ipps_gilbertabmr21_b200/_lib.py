@@ -10,6 +10,7 @@ LIB_PATH = os.environ.get("HEC_LIB_PATH") or os.path.join(_HERE, "libhec.so")
 
 HEC_OK, HEC_EINVAL, HEC_ENOMEM, HEC_ECUDA, HEC_EOVERFLOW = 0, -1, -2, -3, -4
 STOP_CUTOFF, STOP_DISCARD, STOP_STALL, STOP_MAX_LEVELS = 0, 1, 2, 3
+MAP_METHODS = {"hec": 0, "hec3": 1, "hem": 2}  # HEC_MAP_HEC / HEC_MAP_HEC3 / HEC_MAP_HEM
 
 # Every symbol include/hec.h declares (checked by tests/test_abi.py).
 EXPORTS = [
@@ -22,7 +23,7 @@ EXPORTS = [
     "hec_build_rows_write", "hec_heavy_range", "hec_mapping_from_heavy", "hec_balance_rows",
     "hec_ctx_set_profiling", "hec_ctx_profile_reset", "hec_ctx_profile",
     "hec_ctx_launches", "hec_find_mapping_dist", "build_coarse_graph_dist", "hec_csr_dist_slice",
-    "coarsen_hierarchy_dist",
+    "coarsen_hierarchy_dist", "hec_find_mapping_method", "hec_find_mapping_method_prio", "coarsen_hierarchy_ex",
 ]
 
 
@@ -104,6 +105,9 @@ def load():
         "hec_csr_dist_slice": (i32, [p, ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i64),
                                      ctypes.POINTER(i64)]),
         "coarsen_hierarchy_dist": (i32, [p, G, i64, u64, i64, i32, ctypes.POINTER(HecComm), i64, ctypes.POINTER(p)]),
+        "hec_find_mapping_method": (i32, [p, G, i32, u64, i32, p, ctypes.POINTER(i64)]),
+        "hec_find_mapping_method_prio": (i32, [p, G, i32, p, p, ctypes.POINTER(i64)]),
+        "coarsen_hierarchy_ex": (i32, [p, G, i64, u64, i64, i32, i32, ctypes.POINTER(p)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

@@ -418,11 +418,46 @@ HEC_API void hec_csr_free(hec_csr_owned *csr) {
 }
 
 static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed, int64_t discard_below,
-                          int max_levels, const hec_comm *comm, int64_t min_nnz, hec_hierarchy **out);
+                          int max_levels, const hec_comm *comm, int64_t min_nnz, int method, hec_hierarchy **out);
 
 HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
                               int64_t discard_below, int max_levels, hec_hierarchy **out) {
-  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, out);
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, HEC_MAP_HEC, out);
+}
+
+HEC_API int coarsen_hierarchy_ex(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
+                                 int64_t discard_below, int max_levels, int method, hec_hierarchy **out) {
+  if (method != HEC_MAP_HEC && method != HEC_MAP_HEC3 && method != HEC_MAP_HEM) {
+    set_error("unknown mapping method %d", method);
+    return HEC_EINVAL;
+  }
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, method, out);
+}
+
+static int method_common(hec_ctx *ctx, const hec_graph *g, int method, Prio prio, int32_t *M, int64_t *n_c) {
+  HEC_TRY(check_graph(g));
+  if ((g->n > 0 && !M) || !n_c) { set_error("M / n_c is NULL"); return HEC_EINVAL; }
+  size_t ws = 0;
+  ws_bytes_mapping_variant(g->n, g->nnz, &ws);
+  HEC_TRY(begin_call(ctx, ws));
+  if (ctx->validate) HEC_TRY(validate_graph(ctx, g));
+  MapResult r;
+  HEC_TRY(find_mapping_method_impl(ctx, g, method, prio, M, &r));
+  *n_c = r.n_c;
+  ctx->stats.rounds = r.rounds;
+  ctx->stats.n_c = r.n_c;
+  return HEC_OK;
+}
+
+HEC_API int hec_find_mapping_method(hec_ctx *ctx, const hec_graph *g, int method, uint64_t seed, int level,
+                                    int32_t *M, int64_t *n_c) {
+  return method_common(ctx, g, method, Prio{nullptr, splitmix64(seed + (uint64_t)level)}, M, n_c);
+}
+
+HEC_API int hec_find_mapping_method_prio(hec_ctx *ctx, const hec_graph *g, int method, const uint64_t *prio,
+                                         int32_t *M, int64_t *n_c) {
+  if (!prio && g && g->n > 0) { set_error("prio is NULL"); return HEC_EINVAL; }
+  return method_common(ctx, g, method, Prio{prio, 0}, M, n_c);
 }
 
 HEC_API int coarsen_hierarchy_dist(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
@@ -432,11 +467,11 @@ HEC_API int coarsen_hierarchy_dist(hec_ctx *ctx, const hec_graph *g0, int64_t cu
     set_error("coarsen_hierarchy_dist: invalid comm");
     return HEC_EINVAL;
   }
-  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, comm, partition_min_nnz, out);
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, comm, partition_min_nnz, HEC_MAP_HEC, out);
 }
 
 static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed, int64_t discard_below,
-                          int max_levels, const hec_comm *comm, int64_t min_nnz, hec_hierarchy **out) {
+                          int max_levels, const hec_comm *comm, int64_t min_nnz, int method, hec_hierarchy **out) {
   if (!out) { set_error("out is NULL"); return HEC_EINVAL; }
   *out = nullptr;
   HEC_TRY(check_graph(g0));
@@ -448,7 +483,7 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
   h->ctx = ctx;
   // reserve level-0 sized workspace once; later levels are smaller
   size_t wsm = 0;
-  ws_bytes_mapping(g0->n, g0->nnz, &wsm);
+  ws_bytes_mapping_variant(g0->n, g0->nnz, &wsm);
   size_t wsc = ws_bytes_construct(g0->n, g0->nnz, g0->n / 2 + 1);
   int rc = begin_call(ctx, wsm > wsc ? wsm : wsc);
   if (rc == HEC_OK && ctx->validate) rc = validate_graph(ctx, g0);
@@ -465,7 +500,8 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
     ctx->prof_level = level;
     const int ph_level = phase_begin(ctx, "level", 8.0 * (double)cur.nnz + 12.0 * (double)cur.n);
     size_t ws = 0;
-    ws_bytes_mapping(cur.n, cur.nnz, &ws);
+    if (method == HEC_MAP_HEC) ws_bytes_mapping(cur.n, cur.nnz, &ws);
+    else ws_bytes_mapping_variant(cur.n, cur.nnz, &ws);
     rc = ws_reserve(ctx, ws);
     ctx->ws.used = 0;
     MapResult r;
@@ -474,7 +510,7 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
     const Prio prio{nullptr, splitmix64(seed + (uint64_t)level)};
     if (rc == HEC_OK)
       rc = part ? find_mapping_dist_impl(ctx, &cur, prio, comm, M, &r)
-                : find_mapping_impl(ctx, &cur, prio, M, nullptr, nullptr, &r);
+                : find_mapping_method_impl(ctx, &cur, method, prio, M, &r);
     if (rc != HEC_OK) { dev_free(ctx, M); break; }
     ctx->stats.rounds = r.rounds;
     ctx->stats.n_c = r.n_c;

@@ -389,6 +389,9 @@ int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes);
 int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, uint8_t *root_out,
                       int32_t *H_out, MapResult *res);
 int heavy_only_impl(hec_ctx *ctx, const hec_graph *g, int32_t *H);
+// HEC / HEC3 / HEM (HEC_MAP_*) of one level (mapping_variants.cu).
+int ws_bytes_mapping_variant(int64_t n, int64_t nnz, size_t *bytes);
+int find_mapping_method_impl(hec_ctx *ctx, const hec_graph *g, int method, Prio prio, int32_t *M, MapResult *res);
 
 struct CoarseOut {
   int64_t n_c = 0, nnz_c = 0;

@@ -198,6 +198,25 @@ def hec_find_mapping(ctx: Context, g: DeviceGraph, seed: int, level: int, M: tor
     return M, int(nc.value)
 
 
+def hec_find_mapping_method(ctx: Context, g: DeviceGraph, method: str, seed: int = 0, level: int = 0,
+                            prio: torch.Tensor | None = None):
+    """FINDCOARSEMAPPING by "hec" (Alg 3), "hec3" (Alg 5) or "hem" (Alg 2):
+    (M int32[n] on the device, n_c).  prio: explicit visit order (test hook)."""
+    M = torch.empty(g.n, dtype=torch.int32, device=ctx.device)
+    nc = ctypes.c_int64()
+    gc = g.c()
+    m = _lib.MAP_METHODS[method]
+    L = load()
+    if prio is None:
+        rc = L.hec_find_mapping_method(ctx.h, ctypes.byref(gc), m, seed & 0xFFFFFFFFFFFFFFFF, level,
+                                       M.data_ptr() if g.n else None, ctypes.byref(nc))
+    else:
+        rc = L.hec_find_mapping_method_prio(ctx.h, ctypes.byref(gc), m, prio.data_ptr() if g.n else None,
+                                            M.data_ptr() if g.n else None, ctypes.byref(nc))
+    check(rc, "hec_find_mapping_method")
+    return M, int(nc.value)
+
+
 def hec_find_mapping_prio(ctx: Context, g: DeviceGraph, prio: torch.Tensor, M: torch.Tensor | None = None):
     """Mapping under explicit priorities (uint64 bit patterns in an int64 CUDA tensor)."""
     if M is None:
@@ -308,10 +327,17 @@ class Hierarchy:
 
 
 def coarsen_hierarchy(ctx: Context, g0: DeviceGraph, cutoff: int, seed: int, discard_below: int = 10,
-                      max_levels: int = 200) -> Hierarchy:
-    """Alg 1: G_1..G_l until n_l <= cutoff (discard rule of PAPER.md:L367)."""
+                      max_levels: int = 200, method: str = "hec") -> Hierarchy:
+    """Alg 1: G_1..G_l until n_l <= cutoff (discard rule of PAPER.md:L367), every
+    level mapped by `method` ("hec" Alg 3, "hec3" Alg 5, "hem" Alg 2)."""
     h = ctypes.c_void_p()
     gc = g0.c()
-    check(load().coarsen_hierarchy(ctx.h, ctypes.byref(gc), cutoff, seed & 0xFFFFFFFFFFFFFFFF,
-                                   discard_below, max_levels, ctypes.byref(h)), "coarsen_hierarchy")
+    L = load()
+    if method == "hec":
+        rc = L.coarsen_hierarchy(ctx.h, ctypes.byref(gc), cutoff, seed & 0xFFFFFFFFFFFFFFFF, discard_below,
+                                 max_levels, ctypes.byref(h))
+    else:
+        rc = L.coarsen_hierarchy_ex(ctx.h, ctypes.byref(gc), cutoff, seed & 0xFFFFFFFFFFFFFFFF, discard_below,
+                                    max_levels, _lib.MAP_METHODS[method], ctypes.byref(h))
+    check(rc, "coarsen_hierarchy")
     return Hierarchy(ctx, h)
