@@ -188,6 +188,28 @@ HEC_API int64_t hec_hierarchy_discarded_n_c(const hec_hierarchy *h);
 HEC_API int hec_hierarchy_rounds(const hec_hierarchy *h, int i);
 HEC_API void hec_hierarchy_free(hec_hierarchy *h);
 
+/* ------------------------------------------- consumer: spectral bisection */
+/* Multilevel spectral bisection on a hierarchy (PAPER.md
+ * §III-C): on every level, coarsest first, power iteration for the
+ * Fiedler vector of the graph Laplacian L = D - A (x <- (sigma I - L) x with
+ * sigma = 2 max weighted degree, projected off the constant vector and
+ * normalised; fp64), stopped when ||x_{k+1} - x_k||_2 < tol or after max_iter;
+ * interpolation x_fine[u] = x_coarse[M[u]]; then part 0 = the n/2 vertices with
+ * the smallest (x, id) (no imbalance, L330).  The coarsest start vector is
+ * x0[u] = (splitmix64(seed ^ u) >> 11) 2^-53 - 1/2.
+ *   g0: the hierarchy's input graph; h from coarsen_hierarchy on g0.
+ *   part: device uint8[n0] (0 / 1); x: device double[n0] or NULL (the finest
+ *   iterate); *cut (host): weight of the cut edges; iters (host, optional):
+ *   int64[levels + 1], iterations per level from the coarsest. */
+typedef struct {
+  int64_t max_iter;  /* per level; <= 0 selects 1000 */
+  double tol;        /* < 0 selects 1e-10 (L367); 0 runs max_iter iterations */
+  uint64_t seed;
+} hec_spectral_opts;
+HEC_API int hec_spectral_bisection(hec_ctx *ctx, const hec_graph *g0, const hec_hierarchy *h,
+                                   const hec_spectral_opts *opts, uint8_t *part, double *x, int64_t *cut,
+                                   int64_t *iters);
+
 /* ------------------------------------------------------------ profiling */
 /* When enabled, every phase of the hot path is bracketed by CUDA events on the
  * context stream; hec_ctx_profile() synchronises, then reports per phase the

@@ -9,10 +9,10 @@ from ._lib import (HEC_EINVAL, HEC_ENOMEM, HEC_ECUDA, HEC_EOVERFLOW, HEC_OK, STO
                    STOP_DISCARD, STOP_MAX_LEVELS, STOP_STALL, HecError, load)
 from .hec import (CoarseGraph, Context, DeviceGraph, Hierarchy, Level, build_coarse_graph,  # noqa: F401
                   coarsen_hierarchy, hec_debug_heavy, hec_debug_roots, hec_find_mapping,
-                  hec_find_mapping_method, hec_find_mapping_prio, hec_prio)
+                  hec_find_mapping_method, hec_find_mapping_prio, hec_prio, spectral_bisection)
 
 __all__ = [
     "Context", "DeviceGraph", "CoarseGraph", "Hierarchy", "Level", "hec_find_mapping",
     "hec_find_mapping_prio", "hec_find_mapping_method", "build_coarse_graph", "coarsen_hierarchy", "hec_debug_heavy",
-    "hec_debug_roots", "hec_prio", "HecError", "load",
+    "hec_debug_roots", "hec_prio", "HecError", "load", "spectral_bisection",
 ]

@@ -24,6 +24,7 @@ EXPORTS = [
     "hec_ctx_set_profiling", "hec_ctx_profile_reset", "hec_ctx_profile",
     "hec_ctx_launches", "hec_find_mapping_dist", "build_coarse_graph_dist", "hec_csr_dist_slice",
     "coarsen_hierarchy_dist", "hec_find_mapping_method", "hec_find_mapping_method_prio", "coarsen_hierarchy_ex",
+    "hec_spectral_bisection",
 ]
 
 
@@ -37,6 +38,10 @@ class HecStats(ctypes.Structure):
     _fields_ = [("rounds", ctypes.c_int32), ("fallback", ctypes.c_int32),
                 ("n_c", ctypes.c_int64), ("nnz_c", ctypes.c_int64),
                 ("huge_rows", ctypes.c_int64), ("dense_rows", ctypes.c_int64)]
+
+
+class HecSpectralOpts(ctypes.Structure):
+    _fields_ = [("max_iter", ctypes.c_int64), ("tol", ctypes.c_double), ("seed", ctypes.c_uint64)]
 
 
 class HecPhaseTime(ctypes.Structure):
@@ -108,6 +113,8 @@ def load():
         "hec_find_mapping_method": (i32, [p, G, i32, u64, i32, p, ctypes.POINTER(i64)]),
         "hec_find_mapping_method_prio": (i32, [p, G, i32, p, p, ctypes.POINTER(i64)]),
         "coarsen_hierarchy_ex": (i32, [p, G, i64, u64, i64, i32, i32, ctypes.POINTER(p)]),
+        "hec_spectral_bisection": (i32, [p, G, p, ctypes.POINTER(HecSpectralOpts), p, p, ctypes.POINTER(i64),
+                                         ctypes.POINTER(i64)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

@@ -341,3 +341,20 @@ def coarsen_hierarchy(ctx: Context, g0: DeviceGraph, cutoff: int, seed: int, dis
                                     max_levels, _lib.MAP_METHODS[method], ctypes.byref(h))
     check(rc, "coarsen_hierarchy")
     return Hierarchy(ctx, h)
+
+
+def spectral_bisection(ctx: Context, g0: DeviceGraph, hier: Hierarchy, max_iter: int = 1000, tol: float = 1e-10,
+                       seed: int = 0x5EED):
+    """Multilevel spectral bisection on a hierarchy of g0:
+    (part uint8[n0], x float64[n0] on the device, edge cut, iterations per level
+    from the coarsest)."""
+    part = torch.empty(g0.n, dtype=torch.uint8, device=ctx.device)
+    x = torch.empty(g0.n, dtype=torch.float64, device=ctx.device)
+    cut = ctypes.c_int64()
+    iters = (ctypes.c_int64 * (len(hier.levels) + 1))()
+    opts = _lib.HecSpectralOpts(max_iter, tol, seed & 0xFFFFFFFFFFFFFFFF)
+    gc = g0.c()
+    check(load().hec_spectral_bisection(ctx.h, ctypes.byref(gc), hier.h, ctypes.byref(opts),
+                                        part.data_ptr() if g0.n else None, x.data_ptr() if g0.n else None,
+                                        ctypes.byref(cut), iters), "hec_spectral_bisection")
+    return part, x, int(cut.value), list(iters)
