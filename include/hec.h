@@ -157,6 +157,21 @@ typedef struct hec_csr_owned hec_csr_owned; /* device CSR owned by the library *
  * Returns HEC_EOVERFLOW if a sum exceeds INT32_MAX.  Synchronises once (nnz_c). */
 HEC_API int build_coarse_graph(hec_ctx *ctx, const hec_graph *g, const int32_t *M,
                                int64_t n_c, hec_csr_owned **out);
+/* The construction methods (Alg 6); all
+ * give the same canonical G_c, only the work differs:
+ *   HEC_BUILD_HASH     per-row shared-memory hash merge + order-preserving
+ *                      bucket rank (the default of every other call)
+ *   HEC_BUILD_SORT     sort-based DEDUPWITHWTS (register bitonic pieces,
+ *                      shared-memory bucket sort) for every row
+ *   HEC_BUILD_ONE_END  degree-based one-end storage: an entry is kept only in
+ *                      the row of its end with the smaller C' (the count of a
+ *                      row's non-self fine entries, l.1-5; ties: smaller coarse
+ *                      id, reading Z7), then GraphConsWithTrans (l.22)
+ *   HEC_BUILD_AUTO     ONE_END when max degree / average degree > 10 (L324,
+ *                      reading Z15), else HASH */
+enum { HEC_BUILD_HASH = 0, HEC_BUILD_SORT = 1, HEC_BUILD_ONE_END = 2, HEC_BUILD_AUTO = 3 };
+HEC_API int build_coarse_graph_ex(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, int method,
+                                  hec_csr_owned **out);
 /* Borrow the owned CSR as a hec_graph (valid until hec_csr_free). */
 HEC_API int hec_csr_view(const hec_csr_owned *csr, hec_graph *view);
 HEC_API void hec_csr_free(hec_csr_owned *csr);
@@ -173,10 +188,12 @@ typedef struct hec_hierarchy hec_hierarchy;
  * discard_below <= 0 selects the paper's 10; max_levels <= 0 selects 200. */
 HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
                               int64_t discard_below, int max_levels, hec_hierarchy **out);
-/* coarsen_hierarchy with the mapping method of every level chosen by `method`
- * (HEC_MAP_*; coarsen_hierarchy == coarsen_hierarchy_ex(..., HEC_MAP_HEC, ...)). */
+/* coarsen_hierarchy with the mapping method (HEC_MAP_*) and the construction
+ * method (HEC_BUILD_*) of every level chosen (coarsen_hierarchy ==
+ * coarsen_hierarchy_ex(..., HEC_MAP_HEC, HEC_BUILD_HASH, ...)). */
 HEC_API int coarsen_hierarchy_ex(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
-                                 int64_t discard_below, int max_levels, int method, hec_hierarchy **out);
+                                 int64_t discard_below, int max_levels, int map_method, int build_method,
+                                 hec_hierarchy **out);
 HEC_API int hec_hierarchy_levels(const hec_hierarchy *h);
 /* i in [1, levels]: view of G_i, device pointer to M_i (length n_{i-1}), n_{i-1}. */
 HEC_API int hec_hierarchy_level(const hec_hierarchy *h, int i, hec_graph *g_i,

@@ -11,6 +11,7 @@ LIB_PATH = os.environ.get("HEC_LIB_PATH") or os.path.join(_HERE, "libhec.so")
 HEC_OK, HEC_EINVAL, HEC_ENOMEM, HEC_ECUDA, HEC_EOVERFLOW = 0, -1, -2, -3, -4
 STOP_CUTOFF, STOP_DISCARD, STOP_STALL, STOP_MAX_LEVELS = 0, 1, 2, 3
 MAP_METHODS = {"hec": 0, "hec3": 1, "hem": 2}  # HEC_MAP_HEC / HEC_MAP_HEC3 / HEC_MAP_HEM
+BUILD_METHODS = {"hash": 0, "sort": 1, "one_end": 2, "auto": 3}  # HEC_BUILD_*
 
 # Every symbol include/hec.h declares (checked by tests/test_abi.py).
 EXPORTS = [
@@ -24,7 +25,7 @@ EXPORTS = [
     "hec_ctx_set_profiling", "hec_ctx_profile_reset", "hec_ctx_profile",
     "hec_ctx_launches", "hec_find_mapping_dist", "build_coarse_graph_dist", "hec_csr_dist_slice",
     "coarsen_hierarchy_dist", "hec_find_mapping_method", "hec_find_mapping_method_prio", "coarsen_hierarchy_ex",
-    "hec_spectral_bisection",
+    "hec_spectral_bisection", "build_coarse_graph_ex",
 ]
 
 
@@ -112,7 +113,8 @@ def load():
         "coarsen_hierarchy_dist": (i32, [p, G, i64, u64, i64, i32, ctypes.POINTER(HecComm), i64, ctypes.POINTER(p)]),
         "hec_find_mapping_method": (i32, [p, G, i32, u64, i32, p, ctypes.POINTER(i64)]),
         "hec_find_mapping_method_prio": (i32, [p, G, i32, p, p, ctypes.POINTER(i64)]),
-        "coarsen_hierarchy_ex": (i32, [p, G, i64, u64, i64, i32, i32, ctypes.POINTER(p)]),
+        "coarsen_hierarchy_ex": (i32, [p, G, i64, u64, i64, i32, i32, i32, ctypes.POINTER(p)]),
+        "build_coarse_graph_ex": (i32, [p, G, p, i64, i32, ctypes.POINTER(p)]),
         "hec_spectral_bisection": (i32, [p, G, p, ctypes.POINTER(HecSpectralOpts), p, p, ctypes.POINTER(i64),
                                          ctypes.POINTER(i64)]),
     }

@@ -325,6 +325,11 @@ HEC_API int hec_debug_roots(hec_ctx *ctx, const hec_graph *g, const uint64_t *pr
 
 HEC_API int build_coarse_graph(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
                                hec_csr_owned **out) {
+  return build_coarse_graph_ex(ctx, g, M, n_c, HEC_BUILD_HASH, out);
+}
+
+HEC_API int build_coarse_graph_ex(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, int method,
+                                  hec_csr_owned **out) {
   if (!out) { set_error("out is NULL"); return HEC_EINVAL; }
   *out = nullptr;
   HEC_TRY(check_graph(g));
@@ -334,7 +339,7 @@ HEC_API int build_coarse_graph(hec_ctx *ctx, const hec_graph *g, const int32_t *
   hec_csr_owned *o = new (std::nothrow) hec_csr_owned();
   if (!o) { set_error("out of host memory"); return HEC_ENOMEM; }
   o->ctx = ctx;
-  int rc = build_coarse_impl(ctx, g, M, n_c, &o->c);
+  int rc = build_coarse_method_impl(ctx, g, M, n_c, method, &o->c);
   o->slice = DistSlice{0, n_c, 0, o->c.nnz_c};
   if (rc != HEC_OK) {
     free_coarse(ctx, o->c);
@@ -418,20 +423,28 @@ HEC_API void hec_csr_free(hec_csr_owned *csr) {
 }
 
 static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed, int64_t discard_below,
-                          int max_levels, const hec_comm *comm, int64_t min_nnz, int method, hec_hierarchy **out);
+                          int max_levels, const hec_comm *comm, int64_t min_nnz, int method, int build,
+                          hec_hierarchy **out);
 
 HEC_API int coarsen_hierarchy(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
                               int64_t discard_below, int max_levels, hec_hierarchy **out) {
-  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, HEC_MAP_HEC, out);
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, HEC_MAP_HEC, HEC_BUILD_HASH,
+                        out);
 }
 
 HEC_API int coarsen_hierarchy_ex(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed,
-                                 int64_t discard_below, int max_levels, int method, hec_hierarchy **out) {
-  if (method != HEC_MAP_HEC && method != HEC_MAP_HEC3 && method != HEC_MAP_HEM) {
-    set_error("unknown mapping method %d", method);
+                                 int64_t discard_below, int max_levels, int map_method, int build_method,
+                                 hec_hierarchy **out) {
+  if (map_method != HEC_MAP_HEC && map_method != HEC_MAP_HEC3 && map_method != HEC_MAP_HEM) {
+    set_error("unknown mapping method %d", map_method);
     return HEC_EINVAL;
   }
-  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, method, out);
+  if (build_method < HEC_BUILD_HASH || build_method > HEC_BUILD_AUTO) {
+    set_error("unknown construction method %d", build_method);
+    return HEC_EINVAL;
+  }
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, nullptr, 0, map_method, build_method,
+                        out);
 }
 
 static int method_common(hec_ctx *ctx, const hec_graph *g, int method, Prio prio, int32_t *M, int64_t *n_c) {
@@ -467,11 +480,13 @@ HEC_API int coarsen_hierarchy_dist(hec_ctx *ctx, const hec_graph *g0, int64_t cu
     set_error("coarsen_hierarchy_dist: invalid comm");
     return HEC_EINVAL;
   }
-  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, comm, partition_min_nnz, HEC_MAP_HEC, out);
+  return hierarchy_impl(ctx, g0, cutoff, seed, discard_below, max_levels, comm, partition_min_nnz, HEC_MAP_HEC,
+                        HEC_BUILD_HASH, out);
 }
 
 static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed, int64_t discard_below,
-                          int max_levels, const hec_comm *comm, int64_t min_nnz, int method, hec_hierarchy **out) {
+                          int max_levels, const hec_comm *comm, int64_t min_nnz, int method, int build,
+                          hec_hierarchy **out) {
   if (!out) { set_error("out is NULL"); return HEC_EINVAL; }
   *out = nullptr;
   HEC_TRY(check_graph(g0));
@@ -537,7 +552,7 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
         DistSlice sl;
         rc = build_coarse_dist_impl(ctx, &cur, M, r.n_c, comm, 1, &L.g, &sl);
       } else {
-        rc = build_coarse_impl(ctx, &cur, M, r.n_c, &L.g);
+        rc = build_coarse_method_impl(ctx, &cur, M, r.n_c, build, &L.g);
       }
     }
     if (rc != HEC_OK) {

@@ -93,14 +93,7 @@ struct DegIn {
 //   kPieceMax < U <= big_thr        CTA work blocks (windows of kWin, weight U + kRowW)
 //   U > big_thr                     skewed: key-range buckets (BUCKET mode, big_thr =
 //                                   kPieceMax) or dense accumulation (DENSE mode)
-// (HEC_BUCKET_BIG_THR: tuning hook for the skewed-row threshold in BUCKET mode,
-//  clamped to [kPieceMax, kSmallMax])
-static int64_t big_threshold_host(bool dense) {
-  if (dense) return kSmallMax;
-  const char *e = getenv("HEC_BUCKET_BIG_THR");
-  int64_t t = e ? atoll(e) : kPieceMax;
-  return t < kPieceMax ? kPieceMax : (t > kSmallMax ? kSmallMax : t);
-}
+static int64_t big_threshold_host(bool dense) { return dense ? kSmallMax : kPieceMax; }
 
 struct RowWeightIn {
   Layout L;
@@ -272,38 +265,69 @@ constexpr int kXChunk = 4096;  // positions per warp task
 // was measured 1.4x slower on C4: the walk's M[v] gathers need this kernel's
 // occupancy to hide their latency.)
 // sink of the expansion: (M[v], w) to the staging at position - P_lo
+// One-end storage (Alg 6 l.9 / l.17): the entry
+// (a, b) stays in row a only at the end with the smaller degree estimate C',
+// ties to the smaller coarse id (reading Z7); the other end's copy becomes a
+// self entry and is dropped (its weight arrives by the transpose).
+__device__ __forceinline__ bool one_end_keeps(const unsigned long long *__restrict__ Cp, int32_t a, int32_t b) {
+  const unsigned long long ca = __ldg(Cp + a), cb = __ldg(Cp + b);
+  return ca < cb || (ca == cb && a < b);
+}
+
+template <bool kOneEnd = false>
 struct StageSink {
+  static constexpr bool kRows = kOneEnd;
   const Layout &L;
   int32_t *__restrict__ Sb, *__restrict__ Sw;
   int64_t P_lo;
+  const unsigned long long *Cp;  // C' (one-end mode)
   template <int N, typename IdxT>
-  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
-    int32_t b[N], w[N];
+  __device__ __forceinline__ void store(int32_t (&b)[N], int32_t (&w)[N], const IdxT (&p)[N], unsigned ok) {
+#pragma unroll
+    for (int u = 0; u < N; ++u)
+      if (ok & (1u << u)) { __stcs(Sb + ((int64_t)p[u] - P_lo), b[u]); __stcs(Sw + ((int64_t)p[u] - P_lo), w[u]); }
+  }
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void load(int32_t (&b)[N], int32_t (&w)[N], const IdxT (&e)[N], unsigned ok) {
 #pragma unroll
     for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
 #pragma unroll
     for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
+  }
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
+    int32_t b[N], w[N];
+    load(b, w, e, ok);
+    store(b, w, p, ok);
+  }
+  template <int N, typename IdxT>
+  __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok,
+                                             const int32_t (&row)[N]) {
+    int32_t b[N], w[N];
+    load(b, w, e, ok);
 #pragma unroll
     for (int u = 0; u < N; ++u)
-      if (ok & (1u << u)) { __stcs(Sb + ((int64_t)p[u] - P_lo), b[u]); __stcs(Sw + ((int64_t)p[u] - P_lo), w[u]); }
+      if ((ok & (1u << u)) && b[u] != row[u] && !one_end_keeps(Cp, row[u], b[u])) b[u] = row[u];
+    store(b, w, p, ok);
   }
 };
 
 // skip: big_idx in DENSE mode (those rows are expanded by k_dense_accum2), else nullptr
-template <typename IdxT, int kPer>
+template <typename IdxT, int kPer, bool kOneEnd = false>
 __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
                                                int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
-                                               const int32_t *__restrict__ skip, int64_t skip_thr) {
+                                               const int32_t *__restrict__ skip, int64_t skip_thr,
+                                               const unsigned long long *__restrict__ Cp) {
   const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
   const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
   const int64_t gw = ((int64_t)blockIdx.x * kXT + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * kXT) >> 5;
-  StageSink sink{L, Sb, Sw, P_lo};
+  StageSink<kOneEnd> sink{L, Sb, Sw, P_lo, Cp};
   for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
     const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
-    x2_walk<kPer, StageSink, kPer, IdxT>(L, mstart, m_lo, m_hi, P, Pend, skip, sink, skip_thr);
+    x2_walk<kPer, StageSink<kOneEnd>, kPer, IdxT>(L, mstart, m_lo, m_hi, P, Pend, skip, sink, skip_thr);
   }
 }
 
@@ -825,6 +849,7 @@ struct DenseArgs {
   int64_t nunits;
   unsigned *ticket;
   unsigned long long *dense;  // [nbig][n_c] (zeroed)
+  const unsigned long long *Cp;  // C' (one-end mode) or nullptr
 };
 
 constexpr int kDenseUnit2 = 32768;  // DENSE units: 2048 positions per warp, one barrier per unit
@@ -837,10 +862,12 @@ constexpr int kDenseUnit2 = 32768;  // DENSE units: 2048 positions per warp, one
 // here or in k_rows); the accumulator is merged into dense[h] when the CTA
 // moves to another row.  The staging is never written for these rows.
 struct AccSink {
+  static constexpr bool kRows = false;
   const Layout &L;
   uint32_t *acc;
   int32_t a;
   bool wrap;
+  const unsigned long long *Cp;  // C' (one-end mode) or nullptr
   template <int N, typename IdxT>
   __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok) {
     (void)p;
@@ -853,7 +880,7 @@ struct AccSink {
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
 #pragma unroll
     for (int u = 0; u < N; ++u)
-      if ((ok & (1u << u)) && b[u] != a) {  // self entries dropped (L280)
+      if ((ok & (1u << u)) && b[u] != a && (!Cp || one_end_keeps(Cp, a, b[u]))) {  // self entries dropped (L280)
         const uint32_t o = atomicAdd(acc + b[u], (uint32_t)w[u]);
         wrap |= o + (uint32_t)w[u] < o;
       }
@@ -896,7 +923,7 @@ __global__ void __launch_bounds__(kT) k_dense_accum2(DenseArgs A, const int64_t 
     const int64_t Pe = min(P0 + (int64_t)kDenseUnit2, L.upos(a + 1));
     const int64_t Pw = P0 + (int64_t)wid * kSlice;
     const int64_t Pwe = min(Pw + (int64_t)kSlice, Pe);
-    AccSink sink{L, acc, a, false};
+    AccSink sink{L, acc, a, false, A.Cp};
     if (Pw < Pwe) x2_walk<8>(L, mstart, L.member_ptr[a], L.member_ptr[a + 1], Pw, Pwe, nullptr, sink);
     wrap |= sink.wrap;
     __syncthreads();
@@ -924,7 +951,8 @@ size_t ws_bytes_construct(int64_t n, int64_t nnz, int64_t n_c) {
 }
 
 int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, CoarseOut *out,
-                      int64_t a_lo, int64_t a_hi) {
+                      int64_t a_lo, int64_t a_hi, const BuildOpts *opt) {
+  const unsigned long long *Cp = opt ? opt->one_end_cp : nullptr;
   if (a_hi < 0) a_hi = n_c;
   cudaStream_t s = ctx->stream;
   const int64_t n = g->n;
@@ -990,13 +1018,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // (HEC_FORCE_WIDE_INDEX: test hook for the 64-bit instantiation)
   const bool idx32 = g->nnz < ((int64_t)1 << 32) && getenv("HEC_FORCE_WIDE_INDEX") == nullptr;
   Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi, kRbmBinAvg};
-  if (const char *e = getenv("HEC_TUNE_BINAVG")) L.bin_avg = atoll(e);  // (tuning experiment)
   const bool dense = n_c <= kDenseMax;
   // bitmap-rank items replace the bin pieces when the key range fits the
-  // shared-memory bitmap (HEC_NO_RBM: test / tuning hook for the bin-piece path)
+  // shared-memory bitmap (BuildOpts::sort_dedup, HEC_BUILD_SORT: the bin-piece / bucket-sort path)
   // rank items for every level (DENSE levels: the small rows); bins are kept
   // <= kRbmRange keys wide (row_buckets) for the bitmap-rank fallback
-  const bool rbm = getenv("HEC_NO_RBM") == nullptr;
+  const bool rbm = !(opt && opt->sort_dedup);
   const int64_t big_thr = rbm ? (int64_t)kRbmRow : big_threshold_host(dense);
   k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_thr, big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));
@@ -1086,10 +1113,14 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     const int32_t *skip = dense ? big_idx : nullptr;
     const int64_t skip_thr = dense ? 0 : INT64_MAX;
     if (grid > 0) {
-      if (idx32)
-        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr);
+      if (Cp && idx32)
+        k_expand2<uint32_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp);
+      else if (Cp)
+        k_expand2<int64_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp);
+      else if (idx32)
+        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr);
       else
-        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr);
+        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr);
       HEC_LAUNCH_CHECK();
     }
     phase_end(ctx, phx);
@@ -1137,7 +1168,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (nbig > 0 && dense) {
     unsigned long long *dn_arr = arena_take<unsigned long long>(W2, (size_t)nbig * n_c);
     HEC_CUDA_TRY(cudaMemsetAsync(dn_arr, 0, sizeof(unsigned long long) * nbig * n_c, s));
-    DenseArgs D{L, big_list, nbig, unit_ptr, unit_row, nunits, counts + 2, dn_arr};
+    DenseArgs D{L, big_list, nbig, unit_ptr, unit_row, nunits, counts + 2, dn_arr, Cp};
     int occ = 1;
     HEC_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dense_accum2, kT, 4 * (size_t)n_c));
     if (occ < 1) occ = 1;

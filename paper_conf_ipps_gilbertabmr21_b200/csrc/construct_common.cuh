@@ -141,7 +141,8 @@ constexpr int kXBig = 64;
 
 // Walk the member-edge positions [P, Pend) (all inside members [.., m_hi)):
 // sink(e[4], p[4], ok) receives, per step, up to four positions per lane (e:
-// source entry in col/wgt, p: position).  Members whose coarse row a has
+// source entry in col/wgt, p: position); a sink with kRows also receives the
+// coarse row M[member] of each position (sink(e, p, ok, row)).  Members whose coarse row a has
 // U(a) > skip_thr (and skip[a] >= 0 when skip != nullptr) are passed over: rows
 // that their own kernels walk (rank items, DENSE accumulation, unit partition).
 template <int kLong, typename Sink, int kShort = 4, typename IdxT = int64_t>
@@ -154,10 +155,12 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
     const int64_t j = i + lane;
     int64_t mp0 = L.mpre[m_hi], mp1 = mp0, rs = 0;
     bool skipped = false;
+    int32_t ra = 0;  // the member's coarse row (kRows sinks)
     if (j < m_hi) {
       mp0 = L.mpre[j];
       mp1 = L.mpre[j + 1];
       rs = mstart[j];
+      if constexpr (Sink::kRows) ra = L.M[L.members[j]];
       if (skip_thr != INT64_MAX) {
         const int32_t a = L.M[L.members[j]];
         skipped = L.U(a) > skip_thr && (!skip || skip[a] >= 0);
@@ -180,6 +183,7 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
     const int T = __shfl_sync(0xffffffffu, incl, 31);
     for (int base = 0; base < T; base += 32 * kShort) {
       IdxT e[kShort], p[kShort];
+      int32_t rw[kShort];
       unsigned ok = 0;
 #pragma unroll
       for (int u = 0; u < kShort; ++u) {
@@ -196,9 +200,11 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
         const int oex = __shfl_sync(0xffffffffu, excl, lo);
         e[u] = (IdxT)(ors + (t - oex));
         p[u] = (IdxT)(ops + (t - oex));
+        if constexpr (Sink::kRows) rw[u] = __shfl_sync(0xffffffffu, ra, lo);
         if (t < T) ok |= 1u << u;
       }
-      sink(e, p, ok);
+      if constexpr (Sink::kRows) sink(e, p, ok, rw);
+      else sink(e, p, ok);
     }
     // ---- long members, one at a time
     unsigned bm = __ballot_sync(0xffffffffu, big);
@@ -208,17 +214,21 @@ __device__ __forceinline__ void x2_walk(const Layout &L, const int64_t *__restri
       const int bd = __shfl_sync(0xffffffffu, d, src);
       const int64_t brs = __shfl_sync(0xffffffffu, rs, src);
       const int64_t bps = __shfl_sync(0xffffffffu, ps, src);
+      const int32_t bra = __shfl_sync(0xffffffffu, ra, src);
       for (int base = 0; base < bd; base += 32 * kLong) {  // kLong positions per lane in flight
         IdxT e[kLong], p[kLong];
+        int32_t rw[kLong];
         unsigned ok = 0;
 #pragma unroll
         for (int u = 0; u < kLong; ++u) {
           const int t = base + lane + 32 * u;
           e[u] = (IdxT)(brs + t);
           p[u] = (IdxT)(bps + t);
+          rw[u] = bra;
           if (t < bd) ok |= 1u << u;
         }
-        sink(e, p, ok);
+        if constexpr (Sink::kRows) sink(e, p, ok, rw);
+        else sink(e, p, ok);
       }
     }
     // the window reaches the chunk end (or the last member): done

@@ -400,10 +400,20 @@ struct CoarseOut {
 };
 size_t ws_bytes_construct(int64_t n, int64_t nnz, int64_t n_c);
 void free_coarse(hec_ctx *ctx, CoarseOut &c);
+// Construction variants: sort_dedup = the sort / bucket path for all rows
+// instead of the hash rank (HEC_BUILD_SORT); one_end_cp = C' of Alg 6 (one-end
+// storage of every coarse edge, HEC_BUILD_ONE_END's first pass).
+struct BuildOpts {
+  bool sort_dedup = false;
+  const unsigned long long *one_end_cp = nullptr;
+};
 // Coarse rows [a_lo, a_hi) only (a_hi < 0: all rows); out->n_c = a_hi - a_lo and
 // row_ptr/vwgt are indexed from a_lo, row_ptr[0] = 0 (range partition, §8(e)).
 int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c,
-                      CoarseOut *out, int64_t a_lo = 0, int64_t a_hi = -1);
+                      CoarseOut *out, int64_t a_lo = 0, int64_t a_hi = -1, const BuildOpts *opt = nullptr);
+// HEC_BUILD_* dispatch (construct_oneend.cu).
+int build_coarse_method_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_t n_c, int method,
+                             CoarseOut *out);
 // Heavy neighbours of fine rows [u0, u1) only (H indexed globally).
 int heavy_range_impl(hec_ctx *ctx, const hec_graph *g, int64_t u0, int64_t u1, int32_t *H);
 // Resolution rounds + relabel from a full heavy array H; M written for [u0, u1).

@@ -277,12 +277,18 @@ class CoarseGraph:
             pass
 
 
-def build_coarse_graph(ctx: Context, g: DeviceGraph, M: torch.Tensor, n_c: int) -> CoarseGraph:
-    """CONSTRUCTCOARSEGRAPH: G_c = P A P^T without the diagonal, rows sorted, weights summed."""
+def build_coarse_graph(ctx: Context, g: DeviceGraph, M: torch.Tensor, n_c: int, method: str = "hash") -> CoarseGraph:
+    """CONSTRUCTCOARSEGRAPH: G_c = P A P^T without the diagonal, rows sorted, weights summed.
+    method: "hash" (default), "sort", "one_end" (Alg 6's degree-based one-end storage) or "auto"."""
     h = ctypes.c_void_p()
     gc = g.c()
-    check(load().build_coarse_graph(ctx.h, ctypes.byref(gc), M.data_ptr() if g.n else None, n_c,
-                                    ctypes.byref(h)), "build_coarse_graph")
+    L = load()
+    Mp = M.data_ptr() if g.n else None
+    if method == "hash":
+        rc = L.build_coarse_graph(ctx.h, ctypes.byref(gc), Mp, n_c, ctypes.byref(h))
+    else:
+        rc = L.build_coarse_graph_ex(ctx.h, ctypes.byref(gc), Mp, n_c, _lib.BUILD_METHODS[method], ctypes.byref(h))
+    check(rc, "build_coarse_graph")
     return CoarseGraph(ctx, h)
 
 
@@ -327,18 +333,20 @@ class Hierarchy:
 
 
 def coarsen_hierarchy(ctx: Context, g0: DeviceGraph, cutoff: int, seed: int, discard_below: int = 10,
-                      max_levels: int = 200, method: str = "hec") -> Hierarchy:
+                      max_levels: int = 200, method: str = "hec", build: str = "hash") -> Hierarchy:
     """Alg 1: G_1..G_l until n_l <= cutoff (discard rule of PAPER.md:L367), every
-    level mapped by `method` ("hec" Alg 3, "hec3" Alg 5, "hem" Alg 2)."""
+    level mapped by `method` ("hec" Alg 3, "hec3" Alg 5, "hem" Alg 2) and built
+    by `build` ("hash", "sort", "one_end", "auto")."""
     h = ctypes.c_void_p()
     gc = g0.c()
     L = load()
-    if method == "hec":
+    if method == "hec" and build == "hash":
         rc = L.coarsen_hierarchy(ctx.h, ctypes.byref(gc), cutoff, seed & 0xFFFFFFFFFFFFFFFF, discard_below,
                                  max_levels, ctypes.byref(h))
     else:
         rc = L.coarsen_hierarchy_ex(ctx.h, ctypes.byref(gc), cutoff, seed & 0xFFFFFFFFFFFFFFFF, discard_below,
-                                    max_levels, _lib.MAP_METHODS[method], ctypes.byref(h))
+                                    max_levels, _lib.MAP_METHODS[method], _lib.BUILD_METHODS[build],
+                                    ctypes.byref(h))
     check(rc, "coarsen_hierarchy")
     return Hierarchy(ctx, h)
 

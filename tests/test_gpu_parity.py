@@ -309,17 +309,17 @@ def test_construct_random_labels(P, ctx):
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index"])
+@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index", "one_end"])
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
 def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     """R-MAT with random labels into nc aggregates: few labels give huge rows
     (DENSE when nc <= 32768, key-range buckets otherwise), many labels give
     warp-piece and CTA-window rows.  path=bins forces the key-range bin pieces
-    instead of the bitmap-rank items (HEC_NO_RBM test hook); path=wide_index
+    instead of the bitmap-rank items (HEC_BUILD_SORT); path=one_end the
+    degree-based one-end storage + transpose (HEC_BUILD_ONE_END); path=wide_index
     runs the member walks with 64-bit entry indices (the nnz >= 2^32 build,
     HEC_FORCE_WIDE_INDEX test hook)."""
-    if path == "bins":  # DENSE levels: small rows through the k_rows blocks instead of rank items
-        monkeypatch.setenv("HEC_NO_RBM", "1")
+    method = {"bins": "sort", "one_end": "one_end"}.get(path, "hash")
     if path == "wide_index":
         monkeypatch.setenv("HEC_FORCE_WIDE_INDEX", "1")
     rng = np.random.default_rng(15 + nc)
@@ -332,7 +332,7 @@ def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     nc = min(nc, g.n)
     M = rng.integers(0, nc, g.n).astype(np.int32)
     M[rng.permutation(g.n)[:nc]] = np.arange(nc)
-    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc, method=method)
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
@@ -382,12 +382,11 @@ def test_construct_crowded_keys(P, ctx, spread):
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["rbm", "bins"])
-def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
+@pytest.mark.parametrize("path", ["rbm", "bins", "one_end"])
+def test_construct_duplicate_heavy_rows(P, ctx, path):
     """Skewed rows whose entries repeat few keys: key-range buckets far above a
     warp piece (CTA tier) and above a CTA block (fallback), next to ordinary rows."""
-    if path == "bins":
-        monkeypatch.setenv("HEC_NO_RBM", "1")
+    method = {"bins": "sort", "one_end": "one_end"}.get(path, "hash")
     rng = np.random.default_rng(22)
     n = 60000
     hub_targets = rng.integers(0, n, 4000)
@@ -406,7 +405,7 @@ def test_construct_duplicate_heavy_rows(P, ctx, path, monkeypatch):
     M[:8] = 0  # all hubs in one coarse row
     M[hub_targets] = rng.integers(1, 40, hub_targets.size)  # targets collapse onto few keys
     M[rng.permutation(np.setdiff1d(np.arange(8, n), hub_targets))[:nc]] = np.arange(nc)
-    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc)
+    cg = P.build_coarse_graph(ctx, dev(P, g), torch.from_numpy(M).cuda(), nc, method=method)
     assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
@@ -543,6 +542,22 @@ def test_hierarchy_c1(P, ctx, golden_dir):
     # The result (M, G_c) is unaffected — compared exactly above.
     rounds = [lv.rounds for lv in Hg.levels]
     assert all(1 <= r <= k for r, k in zip(rounds, ka["rounds"])), rounds
+
+
+@pytest.mark.parametrize("build", ["sort", "one_end", "auto"])
+@pytest.mark.parametrize("which,cutoff", [("c1", 50), ("rmat14", 50), ("mesh27_24", 100)])
+def test_hierarchy_build_methods(P, ctx, build, which, cutoff):
+    """Every construction method (hash / sort / one-end) gives the
+    oracle's hierarchy bit for bit."""
+    g = {"c1": lambda: gg.config(1), "rmat14": lambda: gg.rmat(14, 16),
+         "mesh27_24": lambda: gg.mesh27(24, 24, 24)}[which]()
+    H = P.coarsen_hierarchy(ctx, dev(P, g), cutoff, SEED, build=build)
+    ref = o.hierarchy(g, cutoff, SEED)
+    assert len(H.levels) == len(ref.levels) and H.stop_reason == ref.stop_reason
+    for lv, lo in zip(H.levels, ref.levels):
+        assert np.array_equal(lv.M.cpu().numpy(), lo.M)
+        assert_csr_equal(lv.graph, lo.graph)
+    H.free()
 
 
 def test_hierarchy_c2(P, ctx):
