@@ -211,6 +211,10 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--method", default="hec", choices=["hec", "hec3", "hem"],
+                    help="mapping method of every level (SURVEY 8(f) f2/f4 ablation; default HEC, the north star)")
+    ap.add_argument("--build", default="hash", choices=["hash", "sort", "one_end", "auto"],
+                    help="construction method (SURVEY 8(f) f1 ablation)")
     args = ap.parse_args()
     rank, local_rank, world = env_rank()
     if args.impl == "reference":
@@ -269,7 +273,8 @@ def main():
         holds G_{l+1}); smaller levels replicated."""
         if world > 1:
             return D.coarsen_hierarchy_dist(ctx, graph, cfg["cutoff"], gg.COARSEN_SEED, comm=comm)
-        return P.coarsen_hierarchy(ctx, graph, cfg["cutoff"], gg.COARSEN_SEED)
+        return P.coarsen_hierarchy(ctx, graph, cfg["cutoff"], gg.COARSEN_SEED, method=args.method,
+                                   build=args.build)
 
     def step():
         h = hierarchy(dg)
@@ -395,6 +400,7 @@ def main():
             "scaling": "strong" if world > 1 else "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz, "m0": m0,
+                       "mapping": args.method, "construction": args.build,
                        "cutoff": cfg["cutoff"], "seed": gg.COARSEN_SEED,
                        "parallelism": (f"partitioned x{world} (levels with >= 64M fine entries): fine-vertex "
                                        "slices for heavy/M, coarse-row ranges for construction, NCCL all-gathers "
