@@ -48,8 +48,10 @@ def main():
         g = gg.config(cfg)
         dg = P.DeviceGraph.from_host(g)
         print(f"C{cfg} {c['name']}: n={g.n} nnz={g.nnz} (gen {time.time() - t0:.0f} s)", flush=True)
-        for method, build in [("hec", "hash"), ("hec", "sort"), ("hec", "one_end"), ("hec", "auto"),
-                              ("hec3", "hash"), ("hem", "hash")]:
+        variants = [("hec", "hash"), ("hec", "sort"), ("hec", "one_end"), ("hec", "auto"), ("hec3", "hash")]
+        if c["kind"] != "rmat":  # HEM on R-MAT runs into the 200-level cap (Table IV: 201 levels)
+            variants.append(("hem", "hash"))
+        for method, build in variants:
             levels = []
 
             def run():
@@ -66,6 +68,13 @@ def main():
             rows.append(r)
             print(f"  {method:5s} {build:8s} {ms:9.3f} ms  {r['edges_per_s'] / 1e9:6.2f} G edges/s  "
                   f"levels {levels}", flush=True)
+        # single-level mappings (level 0): HEC / HEC3 / HEM
+        for method in ("hec", "hec3", "hem"):
+            ms = timed(lambda: P.hec_find_mapping_method(ctx, dg, method, gg.COARSEN_SEED, 0), args.steps, warmup=1)
+            _, nc = P.hec_find_mapping_method(ctx, dg, method, gg.COARSEN_SEED, 0)
+            rows.append({"config": f"C{cfg}", "mapping_level0": method, "ms": ms, "n_c": nc,
+                         "GBps_algorithmic": (8 * g.nnz + 12 * g.n) / (ms / 1e3) / 1e9})
+            print(f"  level-0 mapping {method:5s} {ms:8.3f} ms  n -> n_c {g.n} -> {nc}", flush=True)
         # spectral bisection on the HEC hierarchy: fixed iterations -> SpMV rate
         h = P.coarsen_hierarchy(ctx, dg, c["cutoff"], gg.COARSEN_SEED)
         it = args.spectral_iters
