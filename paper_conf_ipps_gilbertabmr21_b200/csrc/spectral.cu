@@ -5,7 +5,7 @@
 // balanced split.  fp64 throughout.
 //
 //   per level:  d[u] = sum_v w(u,v),  sigma = 2 max d (>= lambda_max(L))
-//   iterate:    y = (sigma I - L) x = (sigma - d) x + A x     (k_lap_spmv: a warp per row)
+//   iterate:    y = (sigma I - L) x = (sigma - d) x + A x     (k_lap_spmv: vector CSR)
 //               y <- y - mean(y), y <- y / ||y||, delta = ||y - x||
 //               stop when delta < tol (L367: 1e-10) or after max_iter
 //   down:       x_fine[u] = x_coarse[M[u]]                    (L330 interpolation)
@@ -80,7 +80,11 @@ __global__ void k_sp_interp(int64_t n, const int32_t *__restrict__ M, const doub
   if (u < n) x[u] = xc[M[u]];
 }
 
-// y = (sigma - d) x + A x over buf[parity] -> buf[parity ^ 1]; partial sums of y
+// y = (sigma - d) x + A x over buf[parity] -> buf[parity ^ 1]; partial sums of y.
+// Vector CSR: a group of G lanes per row (G matched to the average degree, so
+// short mesh rows do not leave most of a warp idle), lane-strided entries,
+// shuffle reduction inside the group.
+template <int G>
 __global__ void __launch_bounds__(kSpT) k_lap_spmv(int64_t n, const int64_t *__restrict__ rp,
                                                    const int32_t *__restrict__ col, const int32_t *__restrict__ wgt,
                                                    const double *__restrict__ d, double *buf0, double *buf1,
@@ -90,21 +94,25 @@ __global__ void __launch_bounds__(kSpT) k_lap_spmv(int64_t n, const int64_t *__r
   const double *x = st->parity ? buf1 : buf0;
   double *y = st->parity ? buf0 : buf1;
   const double sigma = st->sigma;
-  const int lane = threadIdx.x & 31;
-  const int64_t w0 = (blockIdx.x * (int64_t)kSpT + threadIdx.x) >> 5, nw = ((int64_t)gridDim.x * kSpT) >> 5;
-  double acc = 0.0;  // lane 0: this warp's rows
-  for (int64_t u = w0; u < n; u += nw) {
-    double s = 0.0;
-    for (int64_t e = rp[u] + lane; e < rp[u + 1]; e += 32) s += (double)__ldg(wgt + e) * x[__ldg(col + e)];
+  const int gl = threadIdx.x & (G - 1);
+  const int64_t g0 = (blockIdx.x * (int64_t)kSpT + threadIdx.x) / G, ng = ((int64_t)gridDim.x * kSpT) / G;
+  double acc = 0.0;  // group leaders: this group's rows
+  const int64_t rows = (n + ng - 1) / ng * ng;  // every lane runs the same trip count (shuffles)
+  for (int64_t u = g0; u < rows; u += ng) {
+    double sum = 0.0;
+    if (u < n) {
+      const int64_t e1 = rp[u + 1];
+      for (int64_t e = rp[u] + gl; e < e1; e += G) sum += (double)__ldg(wgt + e) * x[__ldg(col + e)];
+    }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    if (lane == 0) {
-      const double v = (sigma - d[u]) * x[u] + s;
+    for (int o = G / 2; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+    if (gl == 0 && u < n) {
+      const double v = (sigma - d[u]) * x[u] + sum;
       y[u] = v;
       acc += v;
     }
   }
-  const double b = block_sum_d(lane == 0 ? acc : 0.0, sh);
+  const double b = block_sum_d(gl == 0 ? acc : 0.0, sh);
   if (threadIdx.x == 0) part[blockIdx.x] = b;
 }
 
@@ -282,7 +290,11 @@ extern "C" HEC_API int hec_spectral_bisection(hec_ctx *ctx, const hec_graph *g0,
     if (max_iter > 0) {
       const int64_t cap = max_iter;
       for (int64_t it = 0; it < cap && rc == HEC_OK; ++it) {
-        k_lap_spmv<<<kSpBlocks, kSpT, 0, s>>>(n, G.row_ptr, G.col, G.wgt, d, buf[0], buf[1], st, p0);
+        const int64_t avg = G.nnz / n;
+        if (avg <= 6) k_lap_spmv<4><<<kSpBlocks, kSpT, 0, s>>>(n, G.row_ptr, G.col, G.wgt, d, buf[0], buf[1], st, p0);
+        else if (avg <= 12) k_lap_spmv<8><<<kSpBlocks, kSpT, 0, s>>>(n, G.row_ptr, G.col, G.wgt, d, buf[0], buf[1], st, p0);
+        else if (avg <= 24) k_lap_spmv<16><<<kSpBlocks, kSpT, 0, s>>>(n, G.row_ptr, G.col, G.wgt, d, buf[0], buf[1], st, p0);
+        else k_lap_spmv<32><<<kSpBlocks, kSpT, 0, s>>>(n, G.row_ptr, G.col, G.wgt, d, buf[0], buf[1], st, p0);
         k_sp_center<<<kSpBlocks, kSpT, 0, s>>>(n, buf[0], buf[1], st, 1, p0, p1);
         k_sp_normalize<<<kSpBlocks, kSpT, 0, s>>>(n, buf[0], buf[1], st, 1, p1, p2);
         k_sp_finish<<<1, 32, 0, s>>>(st, p2, tol, cap);
