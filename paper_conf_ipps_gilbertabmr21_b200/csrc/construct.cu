@@ -8,25 +8,25 @@
 //  a7  bucketing: counting sort of the fine vertices by M (member_ptr, members)
 //      and the "member-edge space": fine entries regrouped by coarse row; row a
 //      owns positions [upos(a), upos(a+1)), U(a) = their number (bound on |row|).
-//  a8  rows with U <= 2040 ("small") are packed into work blocks of < 4096
-//      entries.  One CTA per block: edge-balanced expansion of (b = M[v], w) into
-//      registers through shared-memory member tables, key-range bucket sort in
-//      shared memory (one smem atomic per entry gives each entry its slot), then
-//      per-bucket insertion sort and duplicate merge with exact int64 sums (the
-//      paper's sort-based DEDUPWITHWTS, fastest on GPUs per Table II).
-//  a9  skewed rows (U > 2040):
-//        BUCKET  (n_c > 32768): the row's pairs are partitioned by key range into
-//                buckets of ~1024 entries in global memory (two passes), each
-//                bucket then is one work block of the a8 kind (the paper's
-//                segmented global sort alternative, L324); buckets that overflow
-//                a CTA go through an exact hash-based fallback.
-//        DENSE   (n_c <= 32768): persistent CTAs accumulate the row into a
-//                shared-memory dense array, merged into a dense int64 row; the
-//                row is read back in key order (no sort).
-//  a10 output placement fused into the same kernel: work blocks are taken in
-//      order and each obtains its output offset with a decoupled look-back over
-//      block totals, then writes col_c/wgt_c/row_ptr_c/vwgt_c in place (no
-//      scratch + compaction pass).
+//  a8  expansion (k_expand2): every entry's (b = M[v], w) staged once at its
+//      member-edge position (coalesced runs per coarse row); rows with U <= 124
+//      -> warp pieces (construct_pieces.cu: register bitonic sort + merge), rows
+//      with U <= 4096 -> rank items (construct_hrank.cu: smem hash merge +
+//      order-preserving bucket rank; the sort path HEC_BUILD_SORT uses the
+//      bucket-sort blocks of construct_rows.cu instead).
+//  a9  skewed rows (U > 4096):
+//        BUCKET  (n_c > 32768): the row's staged pairs are partitioned by key
+//                range into bins of ~1024 entries (k_part_count / k_part_write,
+//                the paper's segmented global sort alternative, L324); each bin
+//                is a rank item, direct-indexed (k_drank) when its key range is
+//                at most 4096 keys.
+//        DENSE   (n_c <= 32768): persistent CTAs walk the row's members and
+//                accumulate into a shared-memory dense array (k_dense_accum2),
+//                merged into a dense row read back in key order (no sort).
+//  a10 output placement: every work block stages its sorted distinct entries
+//      (in place over its input) and counts them; an exclusive scan of the
+//      block counts gives each block its output offset, and k_place copies the
+//      staged entries into the final CSR (construct_rows.cu).
 #include <stdlib.h>
 
 #include "construct_common.cuh"
