@@ -178,9 +178,6 @@ HEC_API int hec_ctx_create(hec_stream_t stream, hec_alloc_fn alloc, hec_free_fn 
   int smem = 0;
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, c->device);
   c->smem_optin = (size_t)smem;
-  int l2 = 0;
-  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, c->device);
-  c->l2_bytes = (size_t)l2;
   int major = 0, minor = 0;
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, c->device);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, c->device);

@@ -281,7 +281,6 @@ struct StageSink {
   int32_t *__restrict__ Sb, *__restrict__ Sw;
   int64_t P_lo;
   const unsigned long long *Cp;  // C' (one-end mode)
-  int32_t vlo, vhi;              // only entries with v in [vlo, vhi) (L2-blocked passes)
   template <int N, typename IdxT>
   __device__ __forceinline__ void store(int32_t (&b)[N], int32_t (&w)[N], const IdxT (&p)[N], unsigned ok) {
 #pragma unroll
@@ -289,22 +288,10 @@ struct StageSink {
       if (ok & (1u << u)) { __stcs(Sb + ((int64_t)p[u] - P_lo), b[u]); __stcs(Sw + ((int64_t)p[u] - P_lo), w[u]); }
   }
   template <int N, typename IdxT>
-  __device__ __forceinline__ void load(int32_t (&b)[N], int32_t (&w)[N], const IdxT (&e)[N], unsigned &ok) {
-    if (vlo == 0 && vhi == INT32_MAX) {
+  __device__ __forceinline__ void load(int32_t (&b)[N], int32_t (&w)[N], const IdxT (&e)[N], unsigned ok) {
 #pragma unroll
-      for (int u = 0; u < N; ++u)
-        if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
-    } else {  // L2-blocked pass: the entries of this pass's vertex range only
-#pragma unroll
-      for (int u = 0; u < N; ++u)
-        if (ok & (1u << u)) {
-          b[u] = __ldg(L.col + e[u]);  // (read again by the other pass: keep it cached)
-          if (b[u] < vlo || b[u] >= vhi) ok &= ~(1u << u);
-        }
-#pragma unroll
-      for (int u = 0; u < N; ++u)
-        if (ok & (1u << u)) w[u] = __ldcs(L.wgt + e[u]);
-    }
+    for (int u = 0; u < N; ++u)
+      if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
 #pragma unroll
     for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
@@ -317,7 +304,7 @@ struct StageSink {
   }
   template <int N, typename IdxT>
   __device__ __forceinline__ void operator()(const IdxT (&e)[N], const IdxT (&p)[N], unsigned ok,
-                                             const int32_t (&row)[N]) {  // (single pass only)
+                                             const int32_t (&row)[N]) {
     int32_t b[N], w[N];
     load(b, w, e, ok);
 #pragma unroll
@@ -332,12 +319,12 @@ template <typename IdxT, int kPer, bool kOneEnd = false>
 __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
                                                int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
                                                const int32_t *__restrict__ skip, int64_t skip_thr,
-                                               const unsigned long long *__restrict__ Cp, int32_t vlo, int32_t vhi) {
+                                               const unsigned long long *__restrict__ Cp) {
   const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
   const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
   const int64_t gw = ((int64_t)blockIdx.x * kXT + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * kXT) >> 5;
-  StageSink<kOneEnd> sink{L, Sb, Sw, P_lo, Cp, vlo, vhi};
+  StageSink<kOneEnd> sink{L, Sb, Sw, P_lo, Cp};
   for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
     const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
     x2_walk<kPer, StageSink<kOneEnd>, kPer, IdxT>(L, mstart, m_lo, m_hi, P, Pend, skip, sink, skip_thr);
@@ -1125,30 +1112,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     // everything else is staged once here
     const int32_t *skip = dense ? big_idx : nullptr;
     const int64_t skip_thr = dense ? 0 : INT64_MAX;
-    // M[v] gathers are L2 hits while 4n bytes fit comfortably in L2; beyond
-    // that (C5 level 0: M = 131 MB > 126 MB L2, every gather a DRAM sector)
-    // the expansion runs in passes over slices of the vertex range, each
-    // gathering from an L2-resident slice of M (col is read once per pass)
-    int passes = 1;
-    const char *pe = getenv("HEC_EXPAND_PASSES");  // (A/B timing hook)
-    if (pe) passes = atoi(pe) < 1 ? 1 : atoi(pe);
-    else if (!Cp && ctx->l2_bytes > 0 && (double)n * 4.0 > 0.5 * (double)ctx->l2_bytes)
-      passes = (int)((n * 4 + ctx->l2_bytes / 2 - 1) / (ctx->l2_bytes / 2));
-    for (int ps = 0; ps < passes && grid > 0; ++ps) {
-      const int32_t vlo = passes == 1 ? 0 : (int32_t)((int64_t)n * ps / passes);
-      const int32_t vhi = passes == 1 ? INT32_MAX : (int32_t)((int64_t)n * (ps + 1) / passes);
+    if (grid > 0) {
       if (Cp && idx32)
-        k_expand2<uint32_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp,
-                                                                    vlo, vhi);
+        k_expand2<uint32_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp);
       else if (Cp)
-        k_expand2<int64_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp,
-                                                                   vlo, vhi);
+        k_expand2<int64_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp);
       else if (idx32)
-        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr,
-                                                             vlo, vhi);
+        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr);
       else
-        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr,
-                                                            vlo, vhi);
+        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr);
       HEC_LAUNCH_CHECK();
     }
     phase_end(ctx, phx);

@@ -86,7 +86,6 @@ struct hec_ctx {
   int device = 0;
   int num_sms = 148;
   size_t smem_optin = 0;
-  size_t l2_bytes = 0;  // L2 capacity (cudaDevAttrL2CacheSize)
   hec::Arena ws;   // per-call workspace (reserved up front)
   hec::Arena ws2;  // construction skew-path workspace (sized after classification)
   int64_t *h_pinned = nullptr;  // pinned host scalars for D2H reads

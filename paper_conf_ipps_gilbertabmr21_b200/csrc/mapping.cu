@@ -412,10 +412,7 @@ __device__ __forceinline__ void seg_process(const SegArgs &A, int64_t k, SegWarp
 // loaded before the current span is processed, so every warp keeps a span of
 // loads in flight while it computes.
 template <bool kVec>
-#ifndef HEC_HEAVY_MINB
-#define HEC_HEAVY_MINB 2
-#endif
-__global__ void __launch_bounds__(32 * kSegWarps, HEC_HEAVY_MINB) k_heavy_seg(SegArgs A) {
+__global__ void __launch_bounds__(32 * kSegWarps, 2) k_heavy_seg(SegArgs A) {
   __shared__ SegWarpSmem smem[kSegWarps];
   const int wid = threadIdx.x >> 5;
   SegWarpSmem &W = smem[wid];

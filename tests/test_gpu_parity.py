@@ -309,7 +309,7 @@ def test_construct_random_labels(P, ctx):
         assert_csr_equal(cg.graph, o.coarsen(g, M, nc))
 
 
-@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index", "one_end", "passes3"])
+@pytest.mark.parametrize("path", ["rbm", "bins", "wide_index", "one_end"])
 @pytest.mark.parametrize("nc", [3, 40, 900, 20000, 70000])
 def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     """R-MAT with random labels into nc aggregates: few labels give huge rows
@@ -322,8 +322,6 @@ def test_construct_size_classes(P, ctx, nc, path, monkeypatch):
     method = {"bins": "sort", "one_end": "one_end"}.get(path, "hash")
     if path == "wide_index":
         monkeypatch.setenv("HEC_FORCE_WIDE_INDEX", "1")
-    if path == "passes3":  # the L2-blocked expansion (automatic when 4n > L2 / 2, e.g. C5 level 0)
-        monkeypatch.setenv("HEC_EXPAND_PASSES", "3")
     rng = np.random.default_rng(15 + nc)
     g = gg.rmat(14 if nc < 20000 else 17, 16)
     g.wgt = rng.integers(1, 1000, g.nnz).astype(np.int32)
