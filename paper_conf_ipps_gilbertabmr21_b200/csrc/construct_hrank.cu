@@ -21,45 +21,17 @@
 
 namespace hec {
 
-#ifndef HEC_HR_TAB
-#define HEC_HR_TAB 4  // hash slots per item = pow2(n) * HEC_HR_TAB / 2
-#endif
-#ifndef HEC_HR_ALIAS
-#define HEC_HR_ALIAS 0  // 1: the bucket-ordered keys share the bucket counters' memory
-#endif
-constexpr int kHrTab = HEC_HR_TAB;
 template <int NT, int PER = 8>
 struct HrSmem {
   static constexpr int kCapE = NT * PER;     // entries per item
-  static constexpr int kSlots = kCapE * kHrTab / 2;  // hash slots (load <= 2 / kHrTab)
+  static constexpr int kSlots = 2 * kCapE;   // hash slots (load <= 1/2)
   int32_t key[kSlots];
   uint32_t val[kSlots];
-#if HEC_HR_ALIAS
-  union {
-    int32_t cnt[kCapE + 1];                  // bucket counts (zeroed by the scan)
-    int32_t scr[kCapE];                      // distinct keys in bucket order (re-zeroed after use)
-  };
-#else
   int32_t cnt[kCapE + 1];                    // bucket counts (zeroed by the scan)
-  int32_t scr[kCapE];                        // distinct keys in bucket order
-#endif
   uint16_t offs[kCapE + 2];                  // bucket offsets (<= kCapE)
+  int32_t scr[kCapE];                        // distinct keys in bucket order
   int32_t wsum[NT / 32 + 1];
   int32_t nd;                                // distinct keys of the item
-};
-
-// k_hrank_big's table: always 2 kCapE (power-of-two) slots
-template <int NT, int PER = 8>
-struct HrBigSmem {
-  static constexpr int kCapE = NT * PER;
-  static constexpr int kSlots = 2 * kCapE;
-  int32_t key[kSlots];
-  uint32_t val[kSlots];
-  int32_t cnt[kCapE + 1];
-  uint16_t offs[kCapE + 2];
-  int32_t scr[kCapE];
-  int32_t wsum[NT / 32 + 1];
-  int32_t nd;
 };
 
 __device__ __forceinline__ uint32_t hr_hash(int32_t b) { return (uint32_t)b * 0x9E3779B1u; }
@@ -127,12 +99,11 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     const int32_t a = it.row, lo = it.lo;
     int32_t *const src_b = (it.bk < 0 ? scb : pbg) + it.src;
     int32_t *const src_w = (it.bk < 0 ? scw : pwg) + it.src;
-    // table geometry: NB buckets (power of two >= n), NB * kHrTab / 2 hash slots
+    // table geometry: NB buckets (power of two >= n), 2 NB hash slots
     const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
     const int NB = 1 << lg;
     const uint32_t hmask = 2u * NB - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
-    const uint32_t nslots = (uint32_t)(NB * kHrTab / 2 > 0 ? NB * kHrTab / 2 : 1);
     // any positive scale keeps the buckets monotone in b (approximate division)
     const float scale = __fdividef((float)NB, (float)(it.hi - lo));
     int32_t kb[PER], kw[PER];
@@ -152,13 +123,12 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     for (int k = 0; k < PER; ++k) {
       if (kb[k] == a) kb[k] = -1;  // self entry (L280)
       if (kb[k] < 0) continue;
-      uint32_t h = kHrTab == 4 ? (hr_hash(kb[k]) >> hshift) & hmask
-                               : (uint32_t)(((uint64_t)hr_hash(kb[k]) * nslots) >> 32);
+      uint32_t h = (hr_hash(kb[k]) >> hshift) & hmask;
       while (true) {
         const int32_t old = atomicCAS(&S.key[h], kEmpty, kb[k]);
         if (old == kEmpty) { own |= 1u << k; break; }
         if (old == kb[k]) break;
-        h = kHrTab == 4 ? (h + 1) & hmask : (h + 1 == nslots ? 0u : h + 1);
+        h = (h + 1) & hmask;
       }
       slot[k] = (int)h;
       const uint32_t o = atomicAdd(&S.val[h], (uint32_t)kw[k]);
@@ -202,12 +172,6 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     }
     if (t == 0) A.blk_cnt[it.bi] = D;
     __syncthreads();
-#if HEC_HR_ALIAS
-#pragma unroll
-    for (int k = 0; k < PER; ++k)
-      if (own & (1u << k)) S.scr[boff[k] + bpos[k]] = 0;  // the counters' zero state
-    __syncthreads();
-#endif
   }
 }
 
@@ -219,12 +183,12 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
 template <int NT>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem *__restrict__ redo,
                                                           unsigned *__restrict__ nredo) {
-  constexpr int kCapE = HrBigSmem<NT>::kCapE;
-  constexpr int kSlots = HrBigSmem<NT>::kSlots;
+  constexpr int kCapE = HrSmem<NT>::kCapE;
+  constexpr int kSlots = HrSmem<NT>::kSlots;
   constexpr int kMaxD = (3 * kSlots) / 8;  // abandon threshold (in-flight inserts stay below kSlots)
   static_assert(kMaxD + kCapE < kSlots, "probe loops must terminate");
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  HrBigSmem<NT> &S = *reinterpret_cast<HrBigSmem<NT> *>(smem_raw);
+  HrSmem<NT> &S = *reinterpret_cast<HrSmem<NT> *>(smem_raw);
   const int t = threadIdx.x;
   const int64_t nitems = *A.nlist;
   for (int i = t; i < kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
@@ -328,7 +292,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
 
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo) {
   constexpr int NT = 512;
-  const size_t smem = sizeof(HrBigSmem<NT>);
+  const size_t smem = sizeof(HrSmem<NT>);
   int occ = 1;
   HEC_TRY(kernel_occupancy(ctx, k_hrank_big<NT>, NT, smem, &occ));
   int64_t grid = (int64_t)ctx->num_sms * 2;
