@@ -30,10 +30,10 @@ int dev_alloc(hec_ctx *ctx, void **p, size_t bytes) {
     }
     return HEC_OK;
   }
-  cudaError_t e = cudaMallocAsync(p, bytes, ctx->stream);
+  cudaError_t e = cudaMallocFromPoolAsync(p, bytes, ctx->pool, ctx->stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
-    set_error("cudaMallocAsync(%zu): %s", bytes, cudaGetErrorString(e));
+    set_error("cudaMallocFromPoolAsync(%zu): %s", bytes, cudaGetErrorString(e));
     *p = nullptr;
     return e == cudaErrorMemoryAllocation ? HEC_ENOMEM : HEC_ECUDA;
   }
@@ -44,6 +44,26 @@ void dev_free(hec_ctx *ctx, void *p) {
   if (!p) return;
   if (ctx->free) ctx->free(p, (hec_stream_t)ctx->stream, ctx->user);
   else cudaFreeAsync(p, ctx->stream);
+}
+
+int out_alloc(hec_ctx *ctx, void **p, size_t bytes) {
+  Slab *sl = ctx->slab;
+  if (!sl || bytes >= kSlabDirect) return dev_alloc(ctx, p, bytes);
+  bytes = (bytes + 255) & ~(size_t)255;
+  if (sl->chunks.empty() || sl->chunks.back().used + bytes > sl->chunks.back().cap) {
+    void *c = nullptr;
+    HEC_TRY(dev_alloc(ctx, &c, kSlabChunk));
+    sl->chunks.push_back({(char *)c, kSlabChunk, 0});
+  }
+  auto &c = sl->chunks.back();
+  *p = c.base + c.used;
+  c.used += bytes;
+  return HEC_OK;
+}
+
+void out_free(hec_ctx *ctx, void *p) {
+  if (!p || (ctx->slab && ctx->slab->owns(p))) return;
+  dev_free(ctx, p);
 }
 
 int arena_reserve(hec_ctx *ctx, Arena *a, size_t bytes) {
@@ -147,10 +167,10 @@ using namespace hec;
 
 namespace hec {
 void free_coarse(hec_ctx *ctx, CoarseOut &c) {
-  dev_free(ctx, c.row_ptr);
-  dev_free(ctx, c.col);
-  dev_free(ctx, c.wgt);
-  dev_free(ctx, c.vwgt);
+  out_free(ctx, c.row_ptr);
+  out_free(ctx, c.col);
+  out_free(ctx, c.wgt);
+  out_free(ctx, c.vwgt);
   c = CoarseOut{};
 }
 }  // namespace hec
@@ -182,15 +202,30 @@ HEC_API int hec_ctx_create(hec_stream_t stream, hec_alloc_fn alloc, hec_free_fn 
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, c->device);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, c->device);
   if (e == cudaSuccess) e = cudaMallocHost((void **)&c->h_pinned, 64 * sizeof(int64_t));
+  if (e == cudaSuccess && !alloc) {
+    // no allocator callback: an own stream-ordered pool that keeps its memory
+    // (the device default pool returns freed memory at every synchronisation,
+    // so each call would pay for fresh allocations)
+    cudaMemPoolProps props{};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = c->device;
+    e = cudaMemPoolCreate(&c->pool, &props);
+    uint64_t keep = UINT64_MAX;
+    if (e == cudaSuccess) e = cudaMemPoolSetAttribute(c->pool, cudaMemPoolAttrReleaseThreshold, &keep);
+  }
   if (e != cudaSuccess) {
     set_error("CUDA init failed: %s", cudaGetErrorString(e));
     cudaGetLastError();
+    if (c->pool) cudaMemPoolDestroy(c->pool);
+    if (c->h_pinned) cudaFreeHost(c->h_pinned);
     delete c;
     return HEC_ECUDA;
   }
   if (major != 10 || minor != 0) {
     set_error("libhec is built for sm_100a (B200); device is sm_%d%d", major, minor);
     cudaFreeHost(c->h_pinned);
+    if (c->pool) cudaMemPoolDestroy(c->pool);
     delete c;
     return HEC_ECUDA;
   }
@@ -205,6 +240,8 @@ HEC_API void hec_ctx_destroy(hec_ctx *ctx) {
   dev_free(ctx, ctx->ws2.base);
   cudaStreamSynchronize(ctx->stream);
   if (ctx->h_pinned) cudaFreeHost(ctx->h_pinned);
+  // memory still held by live results is released once they are freed
+  if (ctx->pool) cudaMemPoolDestroy(ctx->pool);
   resolve_profile(ctx);
   for (auto e : ctx->prof_pool) cudaEventDestroy(e);
   delete ctx;
@@ -496,6 +533,8 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
   hec_hierarchy *h = new (std::nothrow) hec_hierarchy();
   if (!h) { set_error("out of host memory"); return HEC_ENOMEM; }
   h->ctx = ctx;
+  Slab *prev_slab = ctx->slab;
+  ctx->slab = &h->slab;
   // reserve level-0 sized workspace once; later levels are smaller
   size_t wsm = 0;
   ws_bytes_mapping_variant(g0->n, g0->nnz, &wsm);
@@ -508,7 +547,7 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
     if (cur.n <= cutoff) { h->stop_reason = HEC_STOP_CUTOFF; break; }
     if (level >= max_levels) { h->stop_reason = HEC_STOP_MAX_LEVELS; break; }
     int32_t *M = nullptr;
-    rc = dev_alloc(ctx, (void **)&M, sizeof(int32_t) * cur.n);
+    rc = out_alloc(ctx, (void **)&M, sizeof(int32_t) * cur.n);
     if (rc != HEC_OK) break;
     // one "level" phase per level: mapping + construction (SURVEY §8(d) B_l);
     // a discarded level is its mapping only (B = 8 nnz + 12 n)
@@ -526,19 +565,19 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
     if (rc == HEC_OK)
       rc = part ? find_mapping_dist_impl(ctx, &cur, prio, comm, M, &r)
                 : find_mapping_method_impl(ctx, &cur, method, prio, M, &r);
-    if (rc != HEC_OK) { dev_free(ctx, M); break; }
+    if (rc != HEC_OK) { out_free(ctx, M); break; }
     ctx->stats.rounds = r.rounds;
     ctx->stats.n_c = r.n_c;
     phase_end(ctx, ph_level);  // (extended below when the level is built)
     if (r.n_c < discard_below) {
       h->stop_reason = HEC_STOP_DISCARD;
       h->discarded_n_c = r.n_c;
-      dev_free(ctx, M);
+      out_free(ctx, M);
       break;
     }
     if (r.n_c == cur.n) {
       h->stop_reason = HEC_STOP_STALL;
-      dev_free(ctx, M);
+      out_free(ctx, M);
       break;
     }
     rc = ws_reserve(ctx, ws_bytes_construct(cur.n, cur.nnz, r.n_c));
@@ -557,7 +596,7 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
     }
     if (rc != HEC_OK) {
       free_coarse(ctx, L.g);
-      dev_free(ctx, M);
+      out_free(ctx, M);
       break;
     }
     phase_end(ctx, ph_level);
@@ -573,6 +612,7 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
     ++level;
   }
   ctx->prof_level = -1;
+  ctx->slab = prev_slab;
   if (rc != HEC_OK) {
     hec_hierarchy_free(h);
     return rc;
@@ -609,10 +649,15 @@ HEC_API int hec_hierarchy_rounds(const hec_hierarchy *h, int i) {
 
 HEC_API void hec_hierarchy_free(hec_hierarchy *h) {
   if (!h) return;
+  hec_ctx *ctx = h->ctx;
+  Slab *prev = ctx->slab;
+  ctx->slab = &h->slab;
   for (auto &L : h->levels) {
-    free_coarse(h->ctx, L.g);
-    dev_free(h->ctx, L.M);
+    free_coarse(ctx, L.g);
+    out_free(ctx, L.M);
   }
+  ctx->slab = prev;
+  for (auto &c : h->slab.chunks) dev_free(ctx, c.base);
   delete h;
 }
 

@@ -211,12 +211,17 @@ __global__ void k_block_ends(int64_t nblocks, int64_t a_hi, BlockDesc *__restric
 // member-edge positions (kUnit: partition, kCap: dense accumulation);
 // unit_ptr = exclusive scan over big rows.
 // Rows with U <= min_u get no units (BUCKET mode: partitioned by one warp).
+// UnitsIn / BucketsIn run over the n_c upper bound of the big-row count (read
+// on the device) so that their totals come back in the same host read as the
+// volumes: entries h >= nbig contribute 0.
 struct UnitsIn {
   Layout L;
   const int32_t *big_list;
+  const unsigned *nbig;
   int64_t unit;
   int64_t min_u;
   __device__ __forceinline__ int64_t operator()(int64_t h) const {
+    if (h >= (int64_t)*nbig) return 0;
     const int64_t U = L.U(big_list[h]);
     return U <= min_u ? 0 : (U + unit - 1) / unit;
   }
@@ -234,8 +239,10 @@ constexpr int kWarpBins = (int)((kWarpRowMax + 31) / 32);  // row_buckets(kWarpR
 struct BucketsIn {
   Layout L;
   const int32_t *big_list;
+  const unsigned *nbig;
   bool rbm;
   __device__ __forceinline__ int64_t operator()(int64_t h) const {
+    if (h >= (int64_t)*nbig) return 0;
     return row_buckets(L.U(big_list[h]), L.n_c, rbm, L.bin_avg);
   }
 };
@@ -960,7 +967,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   out->nnz_c = 0;
   if (n_c <= 0 || n_c > n) {
     if (n == 0 && n_c == 0) {
-      HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t)));
+      HEC_TRY(out_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t)));
       HEC_CUDA_TRY(cudaMemsetAsync(out->row_ptr, 0, sizeof(int64_t), s));
       return HEC_OK;
     }
@@ -1031,27 +1038,23 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, big_thr}, PtrOut{Sw}, st[2], Sw + n_c));
   HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr, rbm}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 4, counts + 0, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
+  HEC_TRY(chained_scan(ctx, n_c, UnitsIn{L, big_list, counts + 0, dense ? (int64_t)kDenseUnit2 : (int64_t)kUnit,
+                                          dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
+                       st[4], unit_ptr + n_c));
+  if (!dense) HEC_TRY(chained_scan(ctx, n_c, BucketsIn{L, big_list, counts + 0, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + n_c));
+  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 5, unit_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+  if (!dense) HEC_CUDA_TRY(cudaMemcpyAsync(scal + 6, bkt_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 7, blk_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
   phase_end(ctx, ph);
-  int64_t r0[5];
-  HEC_TRY(read_scalars(ctx, scal, 5, r0));
+  int64_t r0[8];
+  HEC_TRY(read_scalars(ctx, scal, 8, r0));
   if ((int)(r0[0] & 0xffffffff) & 1) {
     set_error("build_coarse_graph: M has values outside [0, n_c)");
     return HEC_EINVAL;
   }
   const int64_t small_vol = r0[1], big_vol = r0[2];
   const int64_t nbig = r0[4] & 0xffffffffLL;
-  if (nbig > 0) {
-    HEC_TRY(chained_scan(ctx, nbig, UnitsIn{L, big_list, dense ? (int64_t)kDenseUnit2 : (int64_t)kUnit,
-                                             dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
-                         st[4], unit_ptr + nbig));
-    if (!dense) HEC_TRY(chained_scan(ctx, nbig, BucketsIn{L, big_list, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + nbig));
-    HEC_CUDA_TRY(cudaMemcpyAsync(scal + 5, unit_ptr + nbig, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
-    if (!dense) HEC_CUDA_TRY(cudaMemcpyAsync(scal + 6, bkt_ptr + nbig, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
-  }
-  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 7, blk_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
-  int64_t r1[3];
-  HEC_TRY(read_scalars(ctx, scal + 5, 3, r1));
-  const int64_t nunits = r1[0], nbkt = r1[1], nblocks = r1[2];
+  const int64_t nunits = r0[5], nbkt = r0[6], nblocks = r0[7];
   ctx->stats.huge_rows = nbig;
   ctx->stats.dense_rows = dense ? nbig : 0;
 
@@ -1247,8 +1250,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   }
 
   // ---- work blocks (a8/a9 output), then placement (a10)
-  HEC_TRY(dev_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
-  HEC_TRY(dev_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
+  HEC_TRY(out_alloc(ctx, (void **)&out->row_ptr, sizeof(int64_t) * (n_out + 1)));
+  HEC_TRY(out_alloc(ctx, (void **)&out->vwgt, sizeof(int32_t) * (n_out > 0 ? n_out : 1)));
   out->n_c = n_out;
   A.row_ptr_c = out->row_ptr;
   A.vwgt_c = out->vwgt;
@@ -1317,8 +1320,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     return HEC_EOVERFLOW;
   }
   const int64_t nnz_c = out->nnz_c;
-  HEC_TRY(dev_alloc(ctx, (void **)&out->col, sizeof(int32_t) * (nnz_c > 0 ? nnz_c : 1)));
-  HEC_TRY(dev_alloc(ctx, (void **)&out->wgt, sizeof(int32_t) * (nnz_c > 0 ? nnz_c : 1)));
+  HEC_TRY(out_alloc(ctx, (void **)&out->col, sizeof(int32_t) * (nnz_c > 0 ? nnz_c : 1)));
+  HEC_TRY(out_alloc(ctx, (void **)&out->wgt, sizeof(int32_t) * (nnz_c > 0 ? nnz_c : 1)));
   A.col_c = out->col;
   A.wgt_c = out->wgt;
   const int ph_place = phase_begin(ctx, "place", 16.0 * (double)nnz_c + 16.0 * dnc);

@@ -50,18 +50,20 @@ __device__ __forceinline__ uint32_t shfl_down_k(uint32_t v, int d) { return __sh
 __device__ __forceinline__ uint64_t shfl_down_k(uint64_t v, int d) { return __shfl_down_sync(0xffffffffu, v, d); }
 
 // Exchange step between lanes (partner lane ^ lm, same register): keep the min
-// (f = 0) or the max (f = ~0, comparing complemented keys).  Branch-free: a
-// select here compiles to a divergent branch.
+// (keep_min) or the max.  The key is a min/max (one IMNMX for 32-bit keys); the
+// value follows when the kept key is the partner's.  Equal keys keep their own
+// values on both lanes, so the multiset of (key, value) pairs is preserved.
+// (The earlier complement-and-compare form spent 7 ALU operations per
+// exchange on the ALU pipe that bounds this kernel; this one spends 3.)
 template <int J, typename K>
 __device__ __forceinline__ void bitonic_lanes(K (&key)[J], int32_t (&val)[J], int lm, bool keep_min) {
-  const K f = keep_min ? (K)0 : ~(K)0;
 #pragma unroll
   for (int k = 0; k < J; ++k) {
     const K pk = shfl_xor_k(key[k], lm);
     const int32_t pv = __shfl_xor_sync(0xffffffffu, val[k], lm);
-    const bool take = (pk ^ f) < (key[k] ^ f);
-    key[k] ^= (key[k] ^ pk) & ((K)0 - (K)take);
-    val[k] ^= (val[k] ^ pv) & (int32_t)(0u - (uint32_t)take);
+    const K nk = keep_min ? (pk < key[k] ? pk : key[k]) : (pk > key[k] ? pk : key[k]);
+    if (nk != key[k]) val[k] = pv;
+    key[k] = nk;
   }
 }
 
@@ -72,14 +74,16 @@ __device__ __forceinline__ void bitonic_regs(K (&key)[J], int32_t (&val)[J], Asc
   for (int k = 0; k < J; ++k) {
     if (k & STRIDE) continue;
     const int k2 = k | STRIDE;
-    const K f = asc_of(k) ? (K)0 : ~(K)0;
-    const bool sw = (key[k2] ^ f) < (key[k] ^ f);
-    const K dk = (key[k] ^ key[k2]) & ((K)0 - (K)sw);
-    const int32_t dv = (val[k] ^ val[k2]) & (int32_t)(0u - (uint32_t)sw);
-    key[k] ^= dk;
-    key[k2] ^= dk;
-    val[k] ^= dv;
-    val[k2] ^= dv;
+    const K a = key[k], b = key[k2];
+    const K lo = a < b ? a : b, hi = a < b ? b : a;
+    const bool asc = asc_of(k);
+    const K na = asc ? lo : hi;
+    const bool sw = na != a;
+    const int32_t va = val[k], vb = val[k2];
+    key[k] = na;
+    key[k2] = asc ? hi : lo;
+    val[k] = sw ? vb : va;
+    val[k2] = sw ? va : vb;
   }
 }
 

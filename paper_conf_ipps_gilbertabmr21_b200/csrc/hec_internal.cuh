@@ -75,6 +75,25 @@ struct Arena {
   size_t cap = 0, used = 0;
 };
 
+// Output slab of one hierarchy: output buffers below kSlabDirect bytes (M,
+// row_ptr, vwgt, col, wgt of the small levels) are bump-allocated from shared
+// chunks, so a hierarchy of many small levels makes a few allocator calls
+// instead of five per level.  Freed with the hierarchy.
+struct Slab {
+  struct Chunk {
+    char *base;
+    size_t cap, used;
+  };
+  std::vector<Chunk> chunks;
+  bool owns(const void *p) const {
+    for (const auto &c : chunks)
+      if ((const char *)p >= c.base && (const char *)p < c.base + c.cap) return true;
+    return false;
+  }
+};
+constexpr size_t kSlabDirect = (size_t)16 << 20;
+constexpr size_t kSlabChunk = (size_t)64 << 20;
+
 }  // namespace hec
 
 struct hec_ctx {
@@ -88,6 +107,8 @@ struct hec_ctx {
   size_t smem_optin = 0;
   hec::Arena ws;   // per-call workspace (reserved up front)
   hec::Arena ws2;  // construction skew-path workspace (sized after classification)
+  hec::Slab *slab = nullptr;      // output slab of the hierarchy being built (out_alloc)
+  cudaMemPool_t pool = nullptr;   // own memory pool when no allocator callback is given
   int64_t *h_pinned = nullptr;  // pinned host scalars for D2H reads
   hec_stats stats{};
   // state carried between hec_build_rows_count and hec_build_rows_write
@@ -121,6 +142,9 @@ namespace hec {
 // Device memory owned by outputs goes through ctx->alloc (or cudaMallocAsync).
 int dev_alloc(hec_ctx *ctx, void **p, size_t bytes);
 void dev_free(hec_ctx *ctx, void *p);
+// output buffers: from ctx->slab when one is set and the buffer is small, else dev_alloc
+int out_alloc(hec_ctx *ctx, void **p, size_t bytes);
+void out_free(hec_ctx *ctx, void *p);  // no-op for slab memory (freed with its hierarchy)
 
 // Workspace: reserve(total) once per call (grow-only), then bump-allocate.
 int arena_reserve(hec_ctx *ctx, Arena *a, size_t bytes);
@@ -452,6 +476,7 @@ struct hec_hierarchy {
     int rounds;
   };
   std::vector<Level> levels;
+  hec::Slab slab;
   int stop_reason = HEC_STOP_CUTOFF;
   int64_t discarded_n_c = -1;
 };

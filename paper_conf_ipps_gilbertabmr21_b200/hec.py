@@ -155,11 +155,16 @@ class Context:
         if count == 0:
             return torch.empty(0, dtype=dtype, device=self.device)
         if self.torch_alloc:
-            base = self._blocks.get(int(ptr))
-            if base is None:
-                raise RuntimeError("pointer not owned by this context's allocator")
             nbytes = count * torch.empty(0, dtype=dtype).element_size()
-            return base[:nbytes].view(dtype)
+            ptr = int(ptr)
+            base = self._blocks.get(ptr)
+            if base is not None:
+                return base[:nbytes].view(dtype)
+            # small hierarchy outputs are sub-allocated from shared slab chunks
+            for p0, blk in self._blocks.items():
+                if p0 <= ptr and ptr + nbytes <= p0 + blk.numel():
+                    return blk[ptr - p0:ptr - p0 + nbytes].view(dtype)
+            raise RuntimeError("pointer not owned by this context's allocator")
         out = torch.empty(count, dtype=dtype, device=self.device)
         cudart = _cudart()
         nbytes = count * out.element_size()
