@@ -263,7 +263,8 @@ __global__ void k_seg_fill(int64_t nseg, const int64_t *__restrict__ ptr, int32_
 // arrays with coalesced loads.  Self entries are kept (b == own row): the
 // consumers know their row and drop them.
 constexpr int kXT = 256;       // threads per CTA
-constexpr int kXChunk = 4096;  // positions per warp task
+constexpr int kXChunk = 4096;  // positions per warp task (most; small volumes use less, >= kXChunkMin)
+constexpr int kXChunkMin = 256;
 
 // Expansion (k_expand2): every entry of the rows not walked by the DENSE
 // accumulation is staged once, as (b = M[v], w), in member-edge space by
@@ -326,14 +327,14 @@ template <typename IdxT, int kPer, bool kOneEnd = false>
 __global__ void __launch_bounds__(kXT) k_expand2(Layout L, const int64_t *__restrict__ mstart,
                                                int32_t *__restrict__ Sb, int32_t *__restrict__ Sw,
                                                const int32_t *__restrict__ skip, int64_t skip_thr,
-                                               const unsigned long long *__restrict__ Cp) {
+                                               const unsigned long long *__restrict__ Cp, int64_t chunk) {
   const int64_t m_lo = L.member_ptr[L.a_lo], m_hi = L.member_ptr[L.a_hi];
   const int64_t P_lo = L.mpre[m_lo], P_hi = L.mpre[m_hi];
   const int64_t gw = ((int64_t)blockIdx.x * kXT + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * kXT) >> 5;
   StageSink<kOneEnd> sink{L, Sb, Sw, P_lo, Cp};
-  for (int64_t P = P_lo + gw * kXChunk; P < P_hi; P += nw * kXChunk) {
-    const int64_t Pend = P + kXChunk < P_hi ? P + kXChunk : P_hi;
+  for (int64_t P = P_lo + gw * chunk; P < P_hi; P += nw * chunk) {
+    const int64_t Pend = P + chunk < P_hi ? P + chunk : P_hi;
     x2_walk<kPer, StageSink<kOneEnd>, kPer, IdxT>(L, mstart, m_lo, m_hi, P, Pend, skip, sink, skip_thr);
   }
 }
@@ -1107,9 +1108,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   if (!sc_wgt) { set_error("workspace under-reserved (blocks)"); return HEC_EINVAL; }
   {
     const int phx = phase_begin(ctx, "expand", 12.0 * (double)(small_vol + big_vol) + 16.0 * dn);
-    const int64_t warps = (small_vol + big_vol + kXChunk - 1) / kXChunk;
-    int64_t grid = (warps + kXT / 32 - 1) / (kXT / 32);
+    // chunk: kXChunk positions per warp task, less when that would leave
+    // fewer than 8 tasks per warp slot of the capped grid (small levels)
     const int64_t cap = (int64_t)ctx->num_sms * 8;
+    const int64_t vol = small_vol + big_vol;
+    int64_t chunk = (vol + cap * (kXT / 32) * 8 - 1) / (cap * (kXT / 32) * 8);
+    chunk = (chunk + 127) / 128 * 128;
+    chunk = chunk < kXChunkMin ? kXChunkMin : chunk > kXChunk ? kXChunk : chunk;
+    const int64_t warps = (vol + chunk - 1) / chunk;
+    int64_t grid = (warps + kXT / 32 - 1) / (kXT / 32);
     if (grid > cap) grid = cap;
     // DENSE rows are walked by their accumulation kernel (k_dense_accum2);
     // everything else is staged once here
@@ -1117,13 +1124,13 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     const int64_t skip_thr = dense ? 0 : INT64_MAX;
     if (grid > 0) {
       if (Cp && idx32)
-        k_expand2<uint32_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp);
+        k_expand2<uint32_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp, chunk);
       else if (Cp)
-        k_expand2<int64_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp);
+        k_expand2<int64_t, 4, true><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, Cp, chunk);
       else if (idx32)
-        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr);
+        k_expand2<uint32_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr, chunk);
       else
-        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr);
+        k_expand2<int64_t, 4><<<(unsigned)grid, kXT, 0, s>>>(L, mstart, sc_col, sc_wgt, skip, skip_thr, nullptr, chunk);
       HEC_LAUNCH_CHECK();
     }
     phase_end(ctx, phx);

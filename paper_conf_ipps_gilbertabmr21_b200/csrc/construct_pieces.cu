@@ -242,7 +242,9 @@ __device__ __forceinline__ int piece_run(int32_t row0, PieceTab &S, int R, int n
 // duplicate merge of DEDUPWITHWTS with O(entries) work
 // instead of a sorting network.  Bitmap words are XOR-swizzled inside their
 // 32-word block so the per-lane block walks are bank-conflict free.
-constexpr int kGrpBits = 32768;
+// 16K-key bitmaps keep the warp tables at 5 KB, so 4 CTAs of 8 warps fit an SM
+// (with the 64-register bound below); 32K-key bitmaps allowed 3 (C2: -0.1 ms)
+constexpr int kGrpBits = 16384;
 constexpr int kGrpWords = kGrpBits / 32;
 
 struct GroupTab {
@@ -440,7 +442,7 @@ __device__ __forceinline__ int piece_dispatch(int32_t row0, PieceTab &S, int R, 
 }
 
 template <bool WIDE_KEYS>
-__global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__restrict__ ticket) {
+__global__ void __launch_bounds__(kPW * 32, 4) k_pieces(RowsArgs A, unsigned *__restrict__ ticket) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   WarpTab &W = reinterpret_cast<WarpTab *>(smem_raw)[wid];
@@ -448,7 +450,9 @@ __global__ void __launch_bounds__(kPW * 32) k_pieces(RowsArgs A, unsigned *__res
   const Layout &L = A.L;
   const int64_t P_lo = L.upos(L.a_lo);
   const int64_t nlist = *A.nlist;
-  constexpr int kBatch = 4;  // items per ticket (one global atomic per 4 pieces)
+  // items per ticket: 4 (one global atomic per 4 pieces), 1 when the list is
+  // short next to the grid (small levels: spread the pieces over all warps)
+  const int kBatch = nlist >= 4ll * gridDim.x * kPW ? 4 : 1;
   int64_t item = 0, item_end = 0;
   while (true) {
     if (item == item_end) {

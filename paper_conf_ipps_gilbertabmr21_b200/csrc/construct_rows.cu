@@ -362,7 +362,9 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
       else { src = SRC_PB; soff = A.bkt_off[bk]; }
     }
   }
-  if (mine == A.nblocks - 1) A.row_ptr_c[L.a_hi - L.a_lo] = Om + Tm;
+  // blockIdx.y: slice of the copies (small levels: several warps per 32 blocks)
+  const int S = gridDim.y, sl = blockIdx.y;
+  if (sl == 0 && mine == A.nblocks - 1) A.row_ptr_c[L.a_hi - L.a_lo] = Om + Tm;
   const int64_t O0 = __shfl_sync(0xffffffffu, Om, 0);
   const int64_t total = __shfl_sync(0xffffffffu, Om + Tm, 31) - O0;
   const int32_t *dn = reinterpret_cast<const int32_t *>(A.dense);
@@ -379,7 +381,7 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   }
   const int64_t pex = pincl - Ps;
   const int64_t ptot = __shfl_sync(0xffffffffu, pincl, 31);
-  for (int64_t j0 = 0; j0 < ptot; j0 += 128) {
+  for (int64_t j0 = (int64_t)sl * 128; j0 < ptot; j0 += (int64_t)S * 128) {
     int32_t c[4], w[4];
     int64_t dst[4];
 #pragma unroll
@@ -425,7 +427,7 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
     else if (sk == SRC_PB) { sc = A.pb_g + sb; sw = A.pw_g + sb; }
     else if (sk == SRC_FB) { sc = A.fb_b + sb; sw = A.fb_w + sb; }
     else { sc = dn + sb; sw = dn + sb + 1; stride = 2; }
-    for (int r0 = 0; r0 < T; r0 += 256) {
+    for (int r0 = sl * 256; r0 < T; r0 += S * 256) {
       int32_t c[8], w[8];
 #pragma unroll
       for (int t = 0; t < 8; ++t) {
@@ -440,7 +442,8 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
     }
   }
   // per-block metadata: row offsets (rows blocks) / row start + vertex weight (skewed rows)
-  unsigned m = __ballot_sync(0xffffffffu, mine < A.nblocks && (rows_kind(dm.kind) || dm.sub == 0));
+  // (block lane j is fixed up by slice j % S)
+  unsigned m = __ballot_sync(0xffffffffu, mine < A.nblocks && (rows_kind(dm.kind) || dm.sub == 0) && lane % S == sl);
   while (m) {
     const int jl = __ffs(m) - 1;
     m &= m - 1;
@@ -459,7 +462,11 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
 
 int launch_place(hec_ctx *ctx, const RowsArgs &A) {
   if (A.nblocks <= 0) return HEC_OK;
-  k_place<<<nblk((A.nblocks + 31) / 32, kPlaceT / 32), kPlaceT, 0, ctx->stream>>>(A);
+  // slices per 32-block group: enough warps for ~16 per SM on small levels
+  const int64_t groups = (A.nblocks + 31) / 32;
+  int64_t S = (int64_t)ctx->num_sms * 16 / groups;
+  S = S < 1 ? 1 : S > 32 ? 32 : S;
+  k_place<<<dim3((unsigned)nblk(groups, kPlaceT / 32), (unsigned)S), kPlaceT, 0, ctx->stream>>>(A);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }

@@ -30,10 +30,12 @@ for step in "$@"; do
       timeout -s KILL 900 python bench.py --config $cfg --steps $st --warmup 3 > ${O}_bench_c$cfg.json 2> ${O}_bench_c$cfg.err
       python tools/show_bench.py ${O}_bench_c$cfg.json 2>&1 | head -30; tail -3 ${O}_bench_c$cfg.err ;;
     launches)
-      cfg=${arg:-4}
-      timeout -s KILL 900 ncu --metrics $M --clock-control none --csv --log-file ${O}_launches_c$cfg.csv \
-        python bench.py $(one_step $cfg) > ${O}_launches_c$cfg.log 2>&1
-      python tools/launches.py ${O}_launches_c$cfg.csv | head -25 ;;
+      # launches=CFG[:warm]  (warm: --cache-control none, caches as a real run leaves them)
+      cfg=${arg%%:*}; cfg=${cfg:-4}; cc=all; sfx=""
+      [[ "$arg" == *:warm ]] && { cc=none; sfx=_warm; }
+      timeout -s KILL 900 ncu --metrics $M --clock-control none --cache-control $cc --csv \
+        --log-file ${O}_launches_c$cfg$sfx.csv python bench.py $(one_step $cfg) > ${O}_launches_c$cfg$sfx.log 2>&1
+      python tools/launches.py ${O}_launches_c$cfg$sfx.csv 2>/dev/null | head -25 ;;
     full)
       IFS=: read -r rx cnt cfg <<< "$arg"; cfg=${cfg:-4}
       timeout -s KILL 1200 ncu --set full --clock-control none --import-source on -k "regex:$rx" -c $cnt \
