@@ -21,14 +21,21 @@
 
 namespace hec {
 
+// bucket counters / offsets are indexed through hr_p: one pad word per 32 so
+// that the scan's per-thread runs (stride 1, 2, 4 or 8 words) are bank-conflict
+// free
+__device__ __forceinline__ int hr_p(int j) { return j + (j >> 5); }
+
 template <int NT, int PER = 8>
 struct HrSmem {
   static constexpr int kCapE = NT * PER;     // entries per item
   static constexpr int kSlots = 2 * kCapE;   // hash slots (load <= 1/2)
+  static constexpr int kNB = kCapE;          // buckets at most
+  static constexpr int kCntN = kNB + kNB / 32 + 2;
   int32_t key[kSlots];
   uint32_t val[kSlots];
-  int32_t cnt[kCapE + 1];                    // bucket counts (zeroed by the scan)
-  uint16_t offs[kCapE + 2];                  // bucket offsets (<= kCapE)
+  int32_t cnt[kCntN];                        // bucket counts (zeroed by the scan), hr_p-indexed
+  uint16_t offs[kCntN + 2];                  // bucket offsets (<= kCapE), hr_p-indexed
   int32_t scr[kCapE];                        // distinct keys in bucket order
   int32_t wsum[NT / 32 + 1];
   int32_t nd;                                // distinct keys of the item
@@ -48,7 +55,7 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
 #pragma unroll
   for (int i = 0; i < PER; ++i) {
     v[i] = 0;
-    if (i < per && beg + i < nb) { v[i] = c[beg + i]; c[beg + i] = 0; }
+    if (i < per && beg + i < nb) { v[i] = c[hr_p(beg + i)]; c[hr_p(beg + i)] = 0; }
     local += v[i];
   }
   int x = local;
@@ -69,10 +76,10 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
   int run = before + x - local;
 #pragma unroll
   for (int i = 0; i < PER; ++i) {
-    if (i < per && beg + i < nb) o[beg + i] = (uint16_t)run;
+    if (i < per && beg + i < nb) o[hr_p(beg + i)] = (uint16_t)run;
     run += v[i];
   }
-  if (t == NT - 1) o[nb] = (uint16_t)total;
+  if (t == NT - 1) o[hr_p(nb)] = (uint16_t)total;
   return total;
 }
 
@@ -87,7 +94,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
   int32_t *const scb = A.sc_col, *const scw = A.sc_wgt, *const pbg = A.pb_g, *const pwg = A.pw_g;
   int *const err = A.err;
   for (int i = t; i < HrSmem<NT, PER>::kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
-  for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
+  for (int i = t; i < HrSmem<NT, PER>::kCntN; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
   __syncthreads();
   RbmItem nx{};
@@ -100,7 +107,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     int32_t *const src_b = (it.bk < 0 ? scb : pbg) + it.src;
     int32_t *const src_w = (it.bk < 0 ? scw : pwg) + it.src;
     // table geometry: NB buckets (power of two >= n), 2 NB hash slots
-    const int lg = n <= 1 ? 0 : 32 - __clz(n - 1);
+    const int lg = (n <= 1 ? 0 : 32 - __clz(n - 1));
     const int NB = 1 << lg;
     const uint32_t hmask = 2u * NB - 1u;
     const int hshift = 31 - lg;  // top lg + 1 bits of the hash
@@ -136,7 +143,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
       if (own & (1u << k)) {
         int bk = (int)__fmul_rz((float)(kb[k] - lo), scale);
         bk = bk < NB - 1 ? bk : NB - 1;
-        bpos[k] = atomicAdd(&S.cnt[bk], 1);
+        bpos[k] = atomicAdd(&S.cnt[hr_p(bk)], 1);
         slot[k] |= bk << 16;  // slot < 2^14, bucket < 2^13
       }
     }
@@ -149,7 +156,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
 #pragma unroll
     for (int k = 0; k < PER; ++k) {
       if (!(own & (1u << k))) continue;
-      boff[k] = S.offs[slot[k] >> 16];
+      boff[k] = S.offs[hr_p(slot[k] >> 16)];
       S.scr[boff[k] + bpos[k]] = kb[k];
     }
     __syncthreads();
@@ -159,7 +166,7 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     for (int k = 0; k < PER; ++k) {
       if (!(own & (1u << k))) continue;
       const int bk = slot[k] >> 16;
-      const int bend = S.offs[bk + 1];
+      const int bend = S.offs[hr_p(bk + 1)];
       int r = boff[k];
       for (int j = boff[k]; j < bend; ++j) r += S.scr[j] < kb[k];
       const int h = slot[k] & 0xffff;
@@ -192,7 +199,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
   const int t = threadIdx.x;
   const int64_t nitems = *A.nlist;
   for (int i = t; i < kSlots; i += NT) { S.key[i] = kEmpty; S.val[i] = 0u; }
-  for (int i = t; i <= kCapE; i += NT) S.cnt[i] = 0;
+  for (int i = t; i < HrSmem<NT>::kCntN; i += NT) S.cnt[i] = 0;
   if (t == 0) S.nd = 0;
   __syncthreads();
   for (int64_t ii = blockIdx.x; ii < nitems; ii += gridDim.x) {
@@ -254,7 +261,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
       if (b == kEmpty) continue;
       int bk = (int)__fmul_rz((float)(b - lo), scale);
       bk = bk < NB - 1 ? bk : NB - 1;
-      atomicAdd(&S.cnt[bk], 1);
+      atomicAdd(&S.cnt[hr_p(bk)], 1);
     }
     __syncthreads();
     hr_scan<NT>(S.cnt, S.offs, NB, S.wsum);  // counts zeroed, offsets in offs
@@ -264,7 +271,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
       if (b == kEmpty) continue;
       int bk = (int)__fmul_rz((float)(b - lo), scale);
       bk = bk < NB - 1 ? bk : NB - 1;
-      S.scr[S.offs[bk] + atomicAdd(&S.cnt[bk], 1)] = b;
+      S.scr[S.offs[hr_p(bk)] + atomicAdd(&S.cnt[hr_p(bk)], 1)] = b;
     }
     __syncthreads();
     for (int sl = t; sl < kSlots; sl += NT) {
@@ -272,8 +279,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
       if (b == kEmpty) continue;
       int bk = (int)__fmul_rz((float)(b - lo), scale);
       bk = bk < NB - 1 ? bk : NB - 1;
-      int r = S.offs[bk];
-      for (int j = S.offs[bk]; j < S.offs[bk + 1]; ++j) r += S.scr[j] < b;
+      int r = S.offs[hr_p(bk)];
+      for (int j = S.offs[hr_p(bk)]; j < S.offs[hr_p(bk + 1)]; ++j) r += S.scr[j] < b;
       const uint32_t sum = S.val[sl];
       if (sum > 0x7fffffffu) atomicOr(A.err, ERR_OVERFLOW);
       src_b[r] = b;
@@ -281,7 +288,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_hrank_big(RowsArgs A, RbmItem
     }
     __syncthreads();
     for (int sl = t; sl < kSlots; sl += NT) { S.key[sl] = kEmpty; S.val[sl] = 0u; }
-    for (int i = t; i < NB; i += NT) S.cnt[i] = 0;
+    for (int i = t; i < NB; i += NT) S.cnt[hr_p(i)] = 0;
     if (t == 0) {
       A.blk_cnt[it.bi] = D;
       S.nd = 0;
