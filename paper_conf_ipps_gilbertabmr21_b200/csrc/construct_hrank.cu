@@ -11,12 +11,15 @@
 //      half of the paper's hash-vs-sort dedup, on B200's fast smem atomics;
 //   2. counts the distinct keys per order-preserving key-range bucket
 //      (bucket = floor((b - lo) * NB / (hi - lo)), NB >= n buckets, so a bucket
-//      holds ~1 key), scans the counts, and ranks each key inside its bucket by
-//      comparison -- the rank is the key's position in the sorted row, so no
-//      sorting pass runs;
-//   3. writes (b, sum) at its rank, in place over the item's own input range.
-// Work is O(n) per item with six CTA barriers; several CTAs per SM overlap
-// them.  Items with n > NT*8 entries are left to k_rbm.
+//      holds ~1 key) and scans the counts; owners place key and sum in bucket
+//      order;
+//   3. thread t takes bucket-order positions t, t + NT, ...: the key's rank is
+//      its bucket offset plus the keys of its bucket below it (neighbouring
+//      lanes share buckets), i.e. its position in the sorted row, so no sorting
+//      pass runs; (b, sum) is written at the rank, in place over the item's own
+//      input range.
+// Work is O(n) per item with four CTA barriers; several CTAs per SM overlap
+// them.  Items with n > NT*8 entries are left to k_hrank_big / k_rbm.
 #include "construct_common.cuh"
 
 namespace hec {
@@ -152,31 +155,39 @@ __global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4
     // ---- 2. bucket offsets; owners place their key in bucket order
     const int D = hr_scan<NT, PER>(S.cnt, S.offs, NB, S.wsum);
     __syncthreads();
-    int boff[PER];
+    // owners place their key in bucket order (scr) and its sum at the same
+    // position of the (zeroed) counter array, and free their slot
 #pragma unroll
     for (int k = 0; k < PER; ++k) {
       if (!(own & (1u << k))) continue;
-      boff[k] = S.offs[hr_p(slot[k] >> 16)];
-      S.scr[boff[k] + bpos[k]] = kb[k];
-    }
-    __syncthreads();
-    // ---- 3. rank inside the bucket (its keys follow boff until the bucket
-    // changes), write at the rank, clean the owned slot
-#pragma unroll
-    for (int k = 0; k < PER; ++k) {
-      if (!(own & (1u << k))) continue;
-      const int bk = slot[k] >> 16;
-      const int bend = S.offs[hr_p(bk + 1)];
-      int r = boff[k];
-      for (int j = boff[k]; j < bend; ++j) r += S.scr[j] < kb[k];
       const int h = slot[k] & 0xffff;
-      const uint32_t sum = S.val[h];
-      if (sum > 0x7fffffffu) atomicOr(err, ERR_OVERFLOW);
-      src_b[r] = kb[k];
-      src_w[r] = (int32_t)sum;
+      const int pos = S.offs[hr_p(slot[k] >> 16)] + bpos[k];
+      S.scr[pos] = kb[k];
+      S.cnt[hr_p(pos)] = (int32_t)S.val[h];
       S.key[h] = kEmpty;
       S.val[h] = 0u;
     }
+    __syncthreads();
+    // ---- 3. thread t ranks the keys at bucket-order positions t, t + NT, ...:
+    // rank = bucket offset + keys of the bucket below it (neighbouring lanes
+    // share buckets: broadcast reads), written at the rank (near-coalesced);
+    // the sums are taken from the counter array, which is zeroed again
+    const float bscale = scale;
+    bool over = false;
+    for (int i = t; i < D; i += NT) {
+      const int32_t key = S.scr[i];
+      const uint32_t sum = (uint32_t)S.cnt[hr_p(i)];
+      S.cnt[hr_p(i)] = 0;
+      int bk = (int)__fmul_rz((float)(key - lo), bscale);
+      bk = bk < NB - 1 ? bk : NB - 1;
+      const int o0 = S.offs[hr_p(bk)], o1 = S.offs[hr_p(bk + 1)];
+      int r = o0;
+      for (int j = o0; j < o1; ++j) r += S.scr[j] < key;
+      over |= sum > 0x7fffffffu;
+      src_b[r] = key;
+      src_w[r] = (int32_t)sum;
+    }
+    if (over) atomicOr(err, ERR_OVERFLOW);
     if (t == 0) A.blk_cnt[it.bi] = D;
     __syncthreads();
   }
