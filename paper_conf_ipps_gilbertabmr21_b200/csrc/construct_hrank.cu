@@ -337,6 +337,52 @@ int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *n
 constexpr int kDrT = 256;
 static_assert(kDirectR == kDrT * 16, "16 counters per thread");
 
+// Ordered sweep of the direct counters c[0 .. R) (shared or global memory):
+// warp w takes the 32-counter rows [w Q, (w + 1) Q) (lane = counter within a
+// row: conflict-free / coalesced reads), counts the non-zero counters with
+// ballots, one CTA scan of the warp counts, then writes (lo + i, c[i]) for the
+// non-zero counters in order (contiguous positions per row: coalesced), and
+// zeroes them when `clear`.  Returns the number written (D); `wsum` holds
+// kDrT / 32 ints; the caller's next barrier protects it.
+constexpr int kDrRowSweep = 1024;  // bins with a key range up to this: dr_sweep (cost ~ range)
+template <bool kClear>
+__device__ __forceinline__ int dr_sweep(uint32_t *c, int R, int32_t lo, int32_t *__restrict__ dst_b,
+                                        int32_t *__restrict__ dst_w, int32_t *wsum, bool &over) {
+  constexpr int NW = kDrT / 32;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int rows = (R + 31) >> 5, per = (rows + NW - 1) / NW;
+  const int q0 = wid * per, q1 = min(q0 + per, rows);
+  int cnt = 0;
+  for (int q = q0; q < q1; ++q) {
+    const int i = 32 * q + lane;
+    const uint32_t v = i < R ? (kClear ? c[i] : __ldcg(c + i)) : 0u;
+    cnt += __popc(__ballot_sync(0xffffffffu, v != 0u));
+  }
+  if (lane == 0) wsum[wid] = cnt;
+  __syncthreads();
+  int base = 0, D = 0;
+#pragma unroll
+  for (int w = 0; w < NW; ++w) {
+    const int sw = wsum[w];
+    base += w < wid ? sw : 0;
+    D += sw;
+  }
+  for (int q = q0; q < q1; ++q) {
+    const int i = 32 * q + lane;
+    const uint32_t v = i < R ? (kClear ? c[i] : __ldcg(c + i)) : 0u;
+    const unsigned m = __ballot_sync(0xffffffffu, v != 0u);
+    if (v) {
+      const int p = base + __popc(m & ((1u << lane) - 1u));
+      over |= v > 0x7fffffffu;
+      dst_b[p] = lo + i;
+      dst_w[p] = (int32_t)v;
+      if (kClear) c[i] = 0u;
+    }
+    base += __popc(m);
+  }
+  return D;
+}
+
 // chunk items of the split bins (list_d items with n > kDrSplit)
 __global__ void k_drank_split(const RbmItem *__restrict__ items, const unsigned *__restrict__ nitems,
                               RbmItem *__restrict__ dc, unsigned *__restrict__ ndc, unsigned *__restrict__ nsplit) {
@@ -397,39 +443,44 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
     }
     if (wrap) atomicOr(A.err, ERR_OVERFLOW);
     __syncthreads();
-    // thread t owns counters [16 t, 16 t + 16): count, block scan, write in order
-    uint32_t v[16];
-    int c = 0;
-#pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      v[q] = val[16 * t + q];
-      c += v[q] != 0u;
-    }
-    int x = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) wsum[wid] = x;
-    __syncthreads();
-    int before = 0, D = 0;
-#pragma unroll
-    for (int w = 0; w < kDrT / 32; ++w) {
-      const int sw = wsum[w];
-      before += w < wid ? sw : 0;
-      D += sw;
-    }
-    int pos = before + x - c;
     bool over = false;
+    int D;
+    if (it.hi - lo <= kDrRowSweep) {
+      D = dr_sweep<true>(val, it.hi - lo, lo, src_b, src_w, wsum, over);
+    } else {  // wide bins: thread t owns counters [16 t, 16 t + 16) (fewer instructions)
+      uint32_t v[16];
+      int c = 0;
 #pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      if (v[q] != 0u) {
-        over |= v[q] > 0x7fffffffu;
-        src_b[pos] = lo + 16 * t + q;
-        src_w[pos] = (int32_t)v[q];
-        ++pos;
-        val[16 * t + q] = 0u;
+      for (int q = 0; q < 16; ++q) {
+        v[q] = val[16 * t + q];
+        c += v[q] != 0u;
+      }
+      int x = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      if (lane == 31) wsum[wid] = x;
+      __syncthreads();
+      int before = 0;
+      D = 0;
+#pragma unroll
+      for (int w = 0; w < kDrT / 32; ++w) {
+        const int sw = wsum[w];
+        before += w < wid ? sw : 0;
+        D += sw;
+      }
+      int pos = before + x - c;
+#pragma unroll
+      for (int q = 0; q < 16; ++q) {
+        if (v[q] != 0u) {
+          over |= v[q] > 0x7fffffffu;
+          src_b[pos] = lo + 16 * t + q;
+          src_w[pos] = (int32_t)v[q];
+          ++pos;
+          val[16 * t + q] = 0u;
+        }
       }
     }
     if (over) atomicOr(A.err, ERR_OVERFLOW);
@@ -476,12 +527,13 @@ __global__ void __launch_bounds__(kDrT) k_drank_chunks(RowsArgs A, const RbmItem
     __syncthreads();
     uint32_t *const g = gacc + (int64_t)sidx * kDirectR;
 #pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      const uint32_t x = val[16 * t + q];
+    for (int q = 0; q < 16; ++q) {  // counter q kDrT + t: conflict-free, coalesced
+      const int i = q * kDrT + t;
+      const uint32_t x = val[i];
       if (x) {
-        const uint32_t o = atomicAdd(g + 16 * t + q, x);
+        const uint32_t o = atomicAdd(g + i, x);
         wrap |= o + x < o;
-        val[16 * t + q] = 0u;
+        val[i] = 0u;
       }
     }
     if (wrap) atomicOr(A.err, ERR_OVERFLOW);
@@ -491,41 +543,9 @@ __global__ void __launch_bounds__(kDrT) k_drank_chunks(RowsArgs A, const RbmItem
     __syncthreads();
     if (!s_last) continue;
     __threadfence();
-    uint32_t v[16];
-    int c = 0;
-#pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      v[q] = __ldcg(g + 16 * t + q);
-      c += v[q] != 0u;
-    }
-    int x = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) wsum[wid] = x;
-    __syncthreads();
-    int before = 0, D = 0;
-#pragma unroll
-    for (int w = 0; w < kDrT / 32; ++w) {
-      const int sw = wsum[w];
-      before += w < wid ? sw : 0;
-      D += sw;
-    }
-    int pos = before + x - c;
     bool over = false;
     const int64_t out = it.src - (int64_t)chunk * kDrSplit;  // the bin's entries start here
-    int32_t *const dst_b = pbg + out, *const dst_w = pwg + out;
-#pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      if (v[q] != 0u) {
-        over |= v[q] > 0x7fffffffu;
-        dst_b[pos] = lo + 16 * t + q;
-        dst_w[pos] = (int32_t)v[q];
-        ++pos;
-      }
-    }
+    const int D = dr_sweep<false>(g, kDirectR, lo, pbg + out, pwg + out, wsum, over);
     if (over) atomicOr(A.err, ERR_OVERFLOW);
     if (t == 0) A.blk_cnt[it.bi] = D;
     __syncthreads();
