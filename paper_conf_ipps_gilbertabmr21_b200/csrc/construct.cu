@@ -9,7 +9,7 @@
 //      and the "member-edge space": fine entries regrouped by coarse row; row a
 //      owns positions [upos(a), upos(a+1)), U(a) = their number (bound on |row|).
 //  a8  expansion (k_expand2): every entry's (b = M[v], w) staged once at its
-//      member-edge position (coalesced runs per coarse row); rows with U <= 124
+//      member-edge position (coalesced runs per coarse row); rows with U <= 60
 //      -> warp pieces (construct_pieces.cu: register bitonic sort + merge), rows
 //      with U <= 4096 -> rank items (construct_hrank.cu: smem hash merge +
 //      order-preserving bucket rank; the sort path HEC_BUILD_SORT uses the

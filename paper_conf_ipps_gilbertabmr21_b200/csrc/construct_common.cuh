@@ -17,8 +17,9 @@ constexpr int kSmallMax = kWin - kRowW;     // rows with U <= 2040 are small
 constexpr int kMC = 1024;          // member-table chunk
 constexpr int kBucketAvg = 32;     // target entries per key-range bin of a skewed row
 constexpr int kGroupWin = 128;     // bins are grouped into pieces by windows of this weight
-constexpr int kPieceMax = 124;     // rows with U <= kPieceMax go to warp pieces
-constexpr int kPieceWin = 128;     // piece window weight (piece weight < 2*kPieceWin)
+constexpr int kPieceWin = 64;      // piece window weight (piece weight < 2*kPieceWin; 128 measured
+                                   // 2% slower on C2: the 256-slot networks cost more per entry)
+constexpr int kPieceMax = kPieceWin - 4;  // rows with U <= kPieceMax (60) go to warp pieces
 constexpr int kPieceRowW = 4;      // per-row piece weight
 constexpr int kPieceRows = kPieceWin / kPieceRowW;  // rows per piece (all start in one window)
 constexpr int kPieceCap = 256;     // entries per warp piece
