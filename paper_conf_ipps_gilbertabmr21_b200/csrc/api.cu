@@ -82,6 +82,33 @@ int arena_reserve(hec_ctx *ctx, Arena *a, size_t bytes) {
   return HEC_OK;
 }
 
+// blockIdx.y = region; 4-byte words (all regions are 4-byte multiples except
+// byte flag arrays, whose tail bytes are cleared one by one)
+__global__ void k_zero_regions(ZeroList z) {
+  const int r = blockIdx.y;
+  char *p = reinterpret_cast<char *>(z.p[r]);
+  const int64_t b = z.bytes[r];
+  const int64_t words = ((uintptr_t)p & 3) == 0 ? b >> 2 : 0;
+  uint32_t *w = reinterpret_cast<uint32_t *>(p);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
+    w[i] = 0u;
+  for (int64_t i = 4 * words + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < b;
+       i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = 0;
+}
+
+int zero_regions(hec_ctx *ctx, const ZeroList &z) {
+  if (z.n == 0) return HEC_OK;
+  int64_t mx = 0;
+  for (int i = 0; i < z.n; ++i) mx = z.bytes[i] > mx ? z.bytes[i] : mx;
+  int64_t gx = (mx / 4 + 255) / 256;
+  if (gx > 4 * (int64_t)ctx->num_sms) gx = 4 * (int64_t)ctx->num_sms;
+  if (gx < 1) gx = 1;
+  k_zero_regions<<<dim3((unsigned)gx, (unsigned)z.n), 256, 0, ctx->stream>>>(z);
+  HEC_LAUNCH_CHECK();
+  return HEC_OK;
+}
+
 int read_scalars(hec_ctx *ctx, const int64_t *dev, int count, int64_t *host_out) {
   HEC_CUDA_TRY(cudaMemcpyAsync(ctx->h_pinned, dev, sizeof(int64_t) * count, cudaMemcpyDeviceToHost,
                                ctx->stream));

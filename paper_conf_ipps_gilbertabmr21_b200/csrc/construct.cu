@@ -1000,10 +1000,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     return HEC_EINVAL;
   }
   int *err = reinterpret_cast<int *>(scal);
-  HEC_CUDA_TRY(cudaMemsetAsync(mcount, 0, sizeof(unsigned) * (n_c + 1), s));
-  HEC_CUDA_TRY(cudaMemsetAsync(vw64, 0, sizeof(unsigned long long) * (n_c + 1), s));
-  HEC_CUDA_TRY(cudaMemsetAsync(counts, 0, sizeof(unsigned) * 64, s));
-  HEC_CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(int64_t) * 32, s));
+  {
+    ZeroList z;
+    z.add(mcount, (int64_t)sizeof(unsigned) * (n_c + 1));
+    z.add(vw64, (int64_t)sizeof(unsigned long long) * (n_c + 1));
+    z.add(counts, (int64_t)sizeof(unsigned) * 64);
+    z.add(scal, (int64_t)sizeof(int64_t) * 32);
+    for (auto &x : st) z.add(x, n > n_c ? n : n_c);
+    HEC_TRY(zero_regions(ctx, z));
+  }
   const double dn = (double)n, dnc = (double)n_c;
   // ---- a7
   int ph = phase_begin(ctx, "bucket", 16.0 * dn + 4.0 * dnc);
@@ -1011,12 +1016,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     k_member_count<<<nblk(n, 256), 256, 0, s>>>(n, M, n_c, g->vwgt, mcount, vw64, err);
     HEC_LAUNCH_CHECK();
   }
-  HEC_TRY(chained_scan(ctx, n_c, CountIn{mcount}, PtrOut{member_ptr}, st[0], member_ptr + n_c));
+  HEC_TRY(chained_scan(ctx, n_c, CountIn{mcount}, PtrOut{member_ptr}, st[0], member_ptr + n_c, true));
   if (n > 0) {
     k_member_fill<<<nblk(n, 256), 256, 0, s>>>(n, n_c, M, member_ptr, mcount, members, g->row_ptr, mstart);
     HEC_LAUNCH_CHECK();
   }
-  HEC_TRY(chained_scan(ctx, n, DegIn{members, g->row_ptr, member_ptr + n_c}, PtrOut{mpre}, st[1], mpre + n));
+  HEC_TRY(chained_scan(ctx, n, DegIn{members, g->row_ptr, member_ptr + n_c}, PtrOut{mpre}, st[1], mpre + n, true));
   if (a_lo < 0 || a_lo > a_hi || a_hi > n_c) {
     set_error("coarse row range [%lld, %lld) outside [0, %lld)", (long long)a_lo, (long long)a_hi, (long long)n_c);
     return HEC_EINVAL;
@@ -1036,13 +1041,13 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   k_big_rows<<<nblk(n_c, 256), 256, 0, s>>>(L, big_thr, big_list, big_idx, counts + 0,
                                             reinterpret_cast<unsigned long long *>(scal + 1));
   HEC_LAUNCH_CHECK();
-  HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, big_thr}, PtrOut{Sw}, st[2], Sw + n_c));
-  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr, rbm}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c));
+  HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, big_thr}, PtrOut{Sw}, st[2], Sw + n_c, true));
+  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr, rbm}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c, true));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 4, counts + 0, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
   HEC_TRY(chained_scan(ctx, n_c, UnitsIn{L, big_list, counts + 0, dense ? (int64_t)kDenseUnit2 : (int64_t)kUnit,
                                           dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
-                       st[4], unit_ptr + n_c));
-  if (!dense) HEC_TRY(chained_scan(ctx, n_c, BucketsIn{L, big_list, counts + 0, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + n_c));
+                       st[4], unit_ptr + n_c, true));
+  if (!dense) HEC_TRY(chained_scan(ctx, n_c, BucketsIn{L, big_list, counts + 0, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + n_c, true));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 5, unit_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
   if (!dense) HEC_CUDA_TRY(cudaMemcpyAsync(scal + 6, bkt_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 7, blk_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
@@ -1135,7 +1140,12 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     }
     phase_end(ctx, phx);
   }
-  HEC_CUDA_TRY(cudaMemsetAsync(need_wide, 0, sizeof(int32_t) * (nblocks + 1), s));
+  {
+    ZeroList z;
+    z.add(need_wide, (int64_t)sizeof(int32_t) * (nblocks + 1));
+    z.add(st_blk, nblocks);
+    HEC_TRY(zero_regions(ctx, z));
+  }
   k_block_desc<<<nblk(n_c, 256), 256, 0, s>>>(L, blk_ptr, big_idx, dense, rbm, blk);
   HEC_LAUNCH_CHECK();
 
@@ -1198,10 +1208,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     int32_t *fb_b = arena_take<int32_t>(W2, (size_t)big_vol + 1);
     int32_t *fb_w = arena_take<int32_t>(W2, (size_t)big_vol + 1);
     if (!fb_w) { set_error("workspace under-reserved (buckets)"); return HEC_EINVAL; }
-    HEC_CUDA_TRY(cudaMemsetAsync(bkt_cnt, 0, sizeof(unsigned) * (nbkt + 1), s));
     int64_t *prow = arena_take<int64_t>(W2, nbig + 1);
     if (!prow) { set_error("workspace under-reserved (prow)"); return HEC_EINVAL; }
-    HEC_TRY(chained_scan(ctx, nbig, RowUIn{L, big_list}, PtrOut{prow}, stb, prow + nbig));
+    {
+      ZeroList z;
+      z.add(bkt_cnt, (int64_t)sizeof(unsigned) * (nbkt + 1));
+      z.add(stb, nbig);
+      HEC_TRY(zero_regions(ctx, z));
+    }
+    HEC_TRY(chained_scan(ctx, nbig, RowUIn{L, big_list}, PtrOut{prow}, stb, prow + nbig, true));
     PartArgs PA{L, big_list, nbig, unit_ptr, unit_row, bkt_ptr, sc_col, sc_wgt};
     if (nunits > 0) {  // rows above kWarpRowMax: CTA units count, per-row scan, scatter
       k_part_count<<<(unsigned)nunits, kT, sizeof(PartSmem), s>>>(PA, bkt_cnt, ubase);
@@ -1299,7 +1314,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.ticket = counts + 1;
   }
   phase_end(ctx, ph_rows);
-  HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks));
+  HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks, true));
   HEC_CUDA_TRY(cudaMemcpyAsync(scal + 12, blk_off + nblocks, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
   int64_t r2[13];
   HEC_TRY(read_scalars(ctx, scal, 13, r2));

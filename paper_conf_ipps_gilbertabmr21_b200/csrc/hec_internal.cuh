@@ -379,10 +379,12 @@ inline int64_t scan_tiles(int64_t N) {
 }
 // Launch helper: `st` must point to scan_tiles(N) descriptors + ticket (workspace).
 template <typename In, typename Out>
-int chained_scan(hec_ctx *ctx, int64_t N, In in, Out out, ScanTiles st, int64_t *total) {
+int chained_scan(hec_ctx *ctx, int64_t N, In in, Out out, ScanTiles st, int64_t *total, bool zeroed = false) {
   int64_t tiles = scan_tiles(N);
-  HEC_CUDA_TRY(cudaMemsetAsync(st.desc, 0, sizeof(uint64_t) * tiles, ctx->stream));
-  HEC_CUDA_TRY(cudaMemsetAsync(st.ticket, 0, sizeof(unsigned), ctx->stream));
+  if (!zeroed) {  // (zeroed: the caller cleared desc / ticket, e.g. in one ZeroList launch)
+    HEC_CUDA_TRY(cudaMemsetAsync(st.desc, 0, sizeof(uint64_t) * tiles, ctx->stream));
+    HEC_CUDA_TRY(cudaMemsetAsync(st.ticket, 0, sizeof(unsigned), ctx->stream));
+  }
   if (N == 0) {
     if (total) HEC_CUDA_TRY(cudaMemsetAsync(total, 0, sizeof(int64_t), ctx->stream));
     return HEC_OK;
@@ -392,6 +394,20 @@ int chained_scan(hec_ctx *ctx, int64_t N, In in, Out out, ScanTiles st, int64_t 
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }
+// Several workspace regions cleared by one launch instead of one memset each
+// (small levels are bound by the number of stream operations).
+struct ZeroList {
+  static constexpr int kMax = 20;
+  void *p[kMax];
+  int64_t bytes[kMax];
+  int n = 0;
+  void add(void *ptr, int64_t b) {
+    if (b > 0) { p[n] = ptr; bytes[n] = b; ++n; }
+  }
+  void add(ScanTiles st, int64_t N);  // a scan's tile descriptors and ticket
+};
+int zero_regions(hec_ctx *ctx, const ZeroList &z);
+
 inline ScanTiles take_scan_tiles(Arena &ar, int64_t N) {
   ScanTiles st;
   st.desc = arena_take<uint64_t>(ar, (size_t)scan_tiles(N));
@@ -399,6 +415,10 @@ inline ScanTiles take_scan_tiles(Arena &ar, int64_t N) {
   return st;
 }
 inline ScanTiles take_scan_tiles(hec_ctx *ctx, int64_t N) { return take_scan_tiles(ctx->ws, N); }
+inline void ZeroList::add(ScanTiles st, int64_t N) {
+  add(st.desc, (int64_t)sizeof(uint64_t) * scan_tiles(N));
+  add(st.ticket, (int64_t)sizeof(unsigned));
+}
 inline size_t scan_ws_bytes(int64_t N) {
   return ws_bytes((size_t)scan_tiles(N), 8) + ws_bytes(1, 4);
 }

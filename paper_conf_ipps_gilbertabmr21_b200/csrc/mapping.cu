@@ -911,11 +911,18 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   }
   const double dn = (double)n;
   int ph = phase_begin(ctx, "rounds", 5.0 * dn);
-  HEC_CUDA_TRY(cudaMemsetAsync(rootflag, 0, n, s));
-  HEC_CUDA_TRY(cudaMemsetAsync(blocked, 0, sizeof(int32_t) * n, s));
-  HEC_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(unsigned) * 4, s));
-  HEC_CUDA_TRY(cudaMemsetAsync(bar, 0, sizeof(unsigned) * 4, s));
-  HEC_CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(int64_t) * 4, s));
+  ScanTiles st = take_scan_tiles(ctx, n);  // (relabel scan below)
+  if (!st.desc || !st.ticket) { set_error("workspace under-reserved (scan)"); return HEC_EINVAL; }
+  {
+    ZeroList z;
+    z.add(rootflag, n);
+    z.add(blocked, (int64_t)sizeof(int32_t) * n);
+    z.add(cnt, (int64_t)sizeof(unsigned) * 4);
+    z.add(bar, (int64_t)sizeof(unsigned) * 4);
+    z.add(scal, (int64_t)sizeof(int64_t) * 4);
+    z.add(st, n);
+    HEC_TRY(zero_regions(ctx, z));
+  }
   k_round_init<<<nblk(n, 256), 256, 0, s>>>(n, H, prio, status, blocked);
   HEC_LAUNCH_CHECK();
 
@@ -936,9 +943,7 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   phase_end(ctx, ph);
   ph = phase_begin(ctx, "relabel", 9.0 * dn);
   // a4: labels by ascending root id; a5: inherit along H
-  ScanTiles st = take_scan_tiles(ctx, n);
-  if (!st.desc || !st.ticket) { set_error("workspace under-reserved (scan)"); return HEC_EINVAL; }
-  HEC_TRY(chained_scan(ctx, n, RootFlagIn{status}, RootLabelOut{status, lab, root_out}, st, scal));
+  HEC_TRY(chained_scan(ctx, n, RootFlagIn{status}, RootLabelOut{status, lab, root_out}, st, scal, true));
   int *long_chain = reinterpret_cast<int *>(scal + 2);
   if (u1 > u0) {  // wl0 is free after the rounds: jump targets of cut walks
     k_assign<<<nblk(u1 - u0, 256), 256, 0, s>>>(u0, u1, H, status, lab, M, wl0, long_chain);
