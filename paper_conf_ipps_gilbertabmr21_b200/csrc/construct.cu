@@ -119,7 +119,10 @@ __global__ void k_big_rows(Layout L, int64_t big_thr, int32_t *__restrict__ big_
   unsigned base = 0;
   if (m) {
     int leader = __ffs(m) - 1;
-    if (lane == leader) base = atomicAdd(nbig, (unsigned)__popc(m));
+    if (lane == leader) {
+      base = atomicAdd(nbig, (unsigned)__popc(m));
+      atomicAdd(vol + 3, (unsigned long long)__popc(m));  // the host's copy (scal[4])
+    }
     base = __shfl_sync(0xffffffffu, base, leader);
   }
   if (big) {
@@ -1042,15 +1045,11 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
                                             reinterpret_cast<unsigned long long *>(scal + 1));
   HEC_LAUNCH_CHECK();
   HEC_TRY(chained_scan(ctx, n_c, RowWeightIn{L, big_thr}, PtrOut{Sw}, st[2], Sw + n_c, true));
-  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr, rbm}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c, true));
-  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 4, counts + 0, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
+  HEC_TRY(chained_scan(ctx, n_c, BlockCountIn{L, Sw, dense, big_thr, rbm}, PtrOut{blk_ptr}, st[3], blk_ptr + n_c, true, scal + 7));
   HEC_TRY(chained_scan(ctx, n_c, UnitsIn{L, big_list, counts + 0, dense ? (int64_t)kDenseUnit2 : (int64_t)kUnit,
                                           dense ? (int64_t)0 : kWarpRowMax}, PtrOut{unit_ptr},
-                       st[4], unit_ptr + n_c, true));
-  if (!dense) HEC_TRY(chained_scan(ctx, n_c, BucketsIn{L, big_list, counts + 0, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + n_c, true));
-  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 5, unit_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
-  if (!dense) HEC_CUDA_TRY(cudaMemcpyAsync(scal + 6, bkt_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
-  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 7, blk_ptr + n_c, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+                       st[4], unit_ptr + n_c, true, scal + 5));
+  if (!dense) HEC_TRY(chained_scan(ctx, n_c, BucketsIn{L, big_list, counts + 0, rbm}, PtrOut{bkt_ptr}, st[5], bkt_ptr + n_c, true, scal + 6));
   phase_end(ctx, ph);
   int64_t r0[8];
   HEC_TRY(read_scalars(ctx, scal, 8, r0));
@@ -1237,9 +1236,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
                                                    reinterpret_cast<unsigned long long *>(scal + 10),
                                                    rbm ? INT64_MAX : (int64_t)kCap);
     HEC_LAUNCH_CHECK();
-    HEC_CUDA_TRY(cudaMemcpyAsync(scal + 9, counts + 4, sizeof(unsigned), cudaMemcpyDeviceToDevice, s));
-    int64_t rj[1];
-    HEC_TRY(read_scalars(ctx, scal + 9, 1, rj));
+    int64_t rj[1];  // counts[4] (low word; counts is 8-byte aligned)
+    HEC_TRY(read_scalars(ctx, reinterpret_cast<const int64_t *>(counts + 4), 1, rj));
     const int64_t njobs = rj[0] & 0xffffffffLL;
     if (njobs > 0) {
       k_bucket_fallback<<<ctx->num_sms, kT, sizeof(FbSmem), s>>>(jobs, njobs, bkt_off, bkt_cnt, pb, pw, fb_off,
@@ -1314,8 +1312,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.ticket = counts + 1;
   }
   phase_end(ctx, ph_rows);
-  HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks, true));
-  HEC_CUDA_TRY(cudaMemcpyAsync(scal + 12, blk_off + nblocks, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+  HEC_TRY(chained_scan(ctx, nblocks, BlkCntIn{blk_cnt}, PtrOut{blk_off}, st_blk, blk_off + nblocks, true, scal + 12));
   int64_t r2[13];
   HEC_TRY(read_scalars(ctx, scal, 13, r2));
   if ((int)(r2[0] & 0xffffffff) & ERR_WIDE) {

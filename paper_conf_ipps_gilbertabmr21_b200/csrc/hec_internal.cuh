@@ -335,10 +335,11 @@ __device__ __forceinline__ int64_t lookback(uint64_t *desc, int tile, int64_t ag
 }
 
 // Exclusive scan over i in [0, N): out(i, prefix_i) with in(i) >= 0.
-// ITEMS consecutive elements per thread; total written to *total (if non-null).
+// ITEMS consecutive elements per thread; total written to *total and *total2
+// (each if non-null; total2: a copy for a batched host read).
 template <int BLOCK, int ITEMS, typename In, typename Out>
 __global__ void __launch_bounds__(BLOCK) k_chained_scan(int64_t N, In in, Out out, ScanTiles st,
-                                                       int64_t *total) {
+                                                       int64_t *total, int64_t *total2) {
   __shared__ int s_tile;
   __shared__ int64_t s_warp[33];
   __shared__ int64_t s_prefix;
@@ -369,7 +370,10 @@ __global__ void __launch_bounds__(BLOCK) k_chained_scan(int64_t N, In in, Out ou
     run += v[i];
   }
   // the thread holding element N-1 writes the grand total
-  if (total && N > 0 && base <= N - 1 && N - 1 < base + ITEMS) *total = run;
+  if (N > 0 && base <= N - 1 && N - 1 < base + ITEMS) {
+    if (total) *total = run;
+    if (total2) *total2 = run;
+  }
 }
 
 constexpr int kScanBlock = 256, kScanItems = 8;
@@ -379,7 +383,8 @@ inline int64_t scan_tiles(int64_t N) {
 }
 // Launch helper: `st` must point to scan_tiles(N) descriptors + ticket (workspace).
 template <typename In, typename Out>
-int chained_scan(hec_ctx *ctx, int64_t N, In in, Out out, ScanTiles st, int64_t *total, bool zeroed = false) {
+int chained_scan(hec_ctx *ctx, int64_t N, In in, Out out, ScanTiles st, int64_t *total, bool zeroed = false,
+                 int64_t *total2 = nullptr) {
   int64_t tiles = scan_tiles(N);
   if (!zeroed) {  // (zeroed: the caller cleared desc / ticket, e.g. in one ZeroList launch)
     HEC_CUDA_TRY(cudaMemsetAsync(st.desc, 0, sizeof(uint64_t) * tiles, ctx->stream));
@@ -387,10 +392,11 @@ int chained_scan(hec_ctx *ctx, int64_t N, In in, Out out, ScanTiles st, int64_t 
   }
   if (N == 0) {
     if (total) HEC_CUDA_TRY(cudaMemsetAsync(total, 0, sizeof(int64_t), ctx->stream));
+    if (total2) HEC_CUDA_TRY(cudaMemsetAsync(total2, 0, sizeof(int64_t), ctx->stream));
     return HEC_OK;
   }
   k_chained_scan<kScanBlock, kScanItems><<<(unsigned)tiles, kScanBlock, 0, ctx->stream>>>(
-      N, in, out, st, total);
+      N, in, out, st, total, total2);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }

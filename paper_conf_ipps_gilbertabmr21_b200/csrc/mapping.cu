@@ -262,10 +262,13 @@ struct SegWarpSmem {
 
 // x0: aligned index of span 0 (aligned index = entry + off; col/wgt - off are
 // 16-byte aligned); entries [ebase, ebase + nnz) belong to rows [0, n) of rp.
+// (also clears the spans' head values: one launch instead of a memset)
 __global__ void k_span_coords(int64_t n, int64_t nnz, const int64_t *__restrict__ rp, int64_t ebase,
-                              int64_t x0, int64_t off, int64_t nspans, int32_t *__restrict__ cx) {
+                              int64_t x0, int64_t off, int64_t nspans, int32_t *__restrict__ cx,
+                              uint64_t *__restrict__ head) {
   const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k > nspans) return;
+  if (k < nspans) head[k] = 0ull;
   if (k == nspans) { cx[k] = (int32_t)(n - 1); return; }
   if (k == 0) { cx[k] = 0; return; }  // leading empty rows belong to span 0
   int64_t e = x0 + k * kSpan - off;
@@ -496,8 +499,7 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
     uint64_t *head = ws_take<uint64_t>(ctx, nspans + 1);
     uint64_t *mid = ws_take<uint64_t>(ctx, nspans + 1);
     if (!cx || !head || !mid) { set_error("workspace under-reserved (heavy)"); return HEC_EINVAL; }
-    HEC_CUDA_TRY(cudaMemsetAsync(head, 0, sizeof(uint64_t) * nspans, ctx->stream));
-    k_span_coords<<<nblk(nspans + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, x0, off, nspans, cx);
+    k_span_coords<<<nblk(nspans + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, x0, off, nspans, cx, head);
     HEC_LAUNCH_CHECK();
     SegArgs SA{n, nnz, rp, ebase, u0, x0, off, nspans, g->col - off, g->wgt - off, cx, H, head, mid};
     int occ[2] = {1, 1};
