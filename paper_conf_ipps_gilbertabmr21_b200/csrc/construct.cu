@@ -138,9 +138,16 @@ __global__ void k_big_rows(Layout L, int64_t big_thr, int32_t *__restrict__ big_
     vs += __shfl_xor_sync(0xffffffffu, vs, o);
     vb += __shfl_xor_sync(0xffffffffu, vb, o);
   }
+  unsigned long long mx = act ? (unsigned long long)U : 0ull;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long y = __shfl_xor_sync(0xffffffffu, mx, o);
+    mx = y > mx ? y : mx;
+  }
   if (lane == 0) {
     if (vs) atomicAdd(vol + 0, vs);
     if (vb) atomicAdd(vol + 1, vb);
+    if (mx) atomicMax(vol + 2, mx);  // scal[3]: the largest U (host skips empty rank classes)
   }
 }
 
@@ -1060,6 +1067,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   const int64_t small_vol = r0[1], big_vol = r0[2];
   const int64_t nbig = r0[4] & 0xffffffffLL;
   const int64_t nunits = r0[5], nbkt = r0[6], nblocks = r0[7];
+  const int64_t maxU = r0[3];
   ctx->stats.huge_rows = nbig;
   ctx->stats.dense_rows = dense ? nbig : 0;
 
@@ -1290,7 +1298,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     struct RankList { RbmItem *items; unsigned *n; int dir; };
     const RankList cls[5] = {{list_r3, counts + 13, 1},
         {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}, {list_r2, counts + 16, -1}};
+    // Without skewed rows every rank item is a whole row (kPieceMax < U <= maxU):
+    // classes above maxU, the multi-round class and the direct-indexed bins are
+    // empty and not launched (small levels are bound by launches); DENSE levels
+    // have no bins and no whole-row item above kHrMax2 either.
+    const bool no_bins = nbig == 0 || dense;
+    const int64_t cls_lo[5] = {kPieceMax, kHrMaxS, kHrMax0, kHrMax1, kHrMax2};
     for (int c = -1; c < 4; ++c) {
+      if (nbig == 0 && maxU <= cls_lo[c + 1]) continue;
+      if (c == 3 && no_bins) continue;
       const RankList &C = cls[c + 1];
       A.ritems = C.items;
       A.nlist = C.n;
@@ -1308,7 +1324,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     A.ritems = list_d;
     A.nlist = counts + 18;
     A.rdir = 1;
-    HEC_TRY(launch_drank(ctx, A, list_dc, counts + 19, drank_acc, drank_done, counts + 21));
+    if (!no_bins) HEC_TRY(launch_drank(ctx, A, list_dc, counts + 19, drank_acc, drank_done, counts + 21));
     A.ticket = counts + 1;
   }
   phase_end(ctx, ph_rows);
