@@ -760,6 +760,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
                         int64_t *__restrict__ grp_end,
                         WorkItem *__restrict__ list_w, int32_t *__restrict__ list_c, RbmItem *__restrict__ list_r,
                         RbmItem *__restrict__ list_r2, RbmItem *__restrict__ list_d, RbmItem *__restrict__ list_r3,
+                        RbmItem *__restrict__ list_r4,
                         unsigned *__restrict__ list_n,
                         bool rbm, bool direct, int mode,
                         const unsigned long long *__restrict__ vw64, int *__restrict__ err) {
@@ -801,7 +802,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
         ri.bk = (int32_t)bk;
       }
       // size class (k_tiers lists: list_r front/back, list_r2 front/back)
-      tier = ri.n <= kHrMaxS ? 7 : ri.n <= kHrMax0 ? 2 : ri.n <= kHrMax1 ? 3 : ri.n <= kHrMax2 ? 4 : 5;
+      tier = ri.n <= kHrMaxT ? 8 : ri.n <= kHrMaxS ? 7 : ri.n <= kHrMax0 ? 2 : ri.n <= kHrMax1 ? 3 : ri.n <= kHrMax2 ? 4 : 5;
       if (direct && ri.bk >= 0 && ri.hi - ri.lo <= kDirectR) tier = 6;  // direct-indexed bin
     } else if (d.kind != B_BUCKET) tier = 1;
     else {
@@ -823,13 +824,13 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
   }
   const int lane = threadIdx.x & 31;
   // list_n: [0] warp [1] CTA [2] list_r front [4] list_r back [5] list_r2 front [6] list_r2 back
-  //         [8] list_d [3] list_r3 (n <= kHrMaxS)
+  //         [8] list_d [3] list_r3 (n <= kHrMaxS) [12] list_r4 (n <= kHrMaxT)
 #pragma unroll
-  for (int q = 0; q < 8; ++q) {
+  for (int q = 0; q < 9; ++q) {
     const unsigned m = __ballot_sync(0xffffffffu, tier == q);
     if (!m) continue;
     const int leader = __ffs(m) - 1;
-    const int slot = q < 3 ? q : q < 6 ? q + 1 : q == 6 ? 8 : 3;
+    const int slot = q < 3 ? q : q < 6 ? q + 1 : q == 6 ? 8 : q == 7 ? 3 : 12;
     unsigned base = 0;
     if (lane == leader) base = atomicAdd(list_n + slot, (unsigned)__popc(m));
     base = __shfl_sync(0xffffffffu, base, leader);
@@ -841,6 +842,7 @@ __global__ void k_tiers(Layout L, int64_t nblocks, const BlockDesc *__restrict__
       else if (q == 5) list_r2[nblocks - pos] = ri;
       else if (q == 6) list_d[pos] = ri;
       else if (q == 7) list_r3[pos] = ri;
+      else if (q == 8) list_r4[pos] = ri;
       else if (q) list_c[pos] = (int32_t)bi;
       else list_w[pos] = it;
     }
@@ -1110,6 +1112,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   uint32_t *drank_acc = arena_take<uint32_t>(W2, (size_t)nsplit_max * kDirectR);
   unsigned *drank_done = arena_take<unsigned>(W2, nsplit_max);
   RbmItem *list_r3 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n <= kHrMaxS
+  RbmItem *list_r4 = arena_take<RbmItem>(W2, nblocks + 1);    // rank items n <= kHrMaxT
   int64_t *grp_end = arena_take<int64_t>(W2, nblocks + 1);    // BUCKET groups: end bin
   int64_t *blk_off = arena_take<int64_t>(W2, nblocks + 1);
   ScanTiles st_blk = take_scan_tiles(W2, nblocks);
@@ -1273,7 +1276,7 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     k_block_ends<<<nblk(nblocks, 256), 256, 0, s>>>(nblocks, a_hi, blk);
     HEC_LAUNCH_CHECK();
     k_tiers<<<nblk(nblocks, 256), 256, 0, s>>>(L, nblocks, blk, big_idx, bkt_ptr, A.bkt_off, A.bkt_n, A.fb_cnt, blk_cnt, grp_end, list_w,
-                                              list_c, list_r, list_r2, list_d, list_r3, counts + 10, rbm, direct, 0, vw64, err);
+                                              list_c, list_r, list_r2, list_d, list_r3, list_r4, counts + 10, rbm, direct, 0, vw64, err);
     HEC_LAUNCH_CHECK();
   }
 
@@ -1296,18 +1299,18 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
     // hash-rank size classes, then the multi-round hash rank above kHrMax2
     // entries (items with too many distinct keys -> the bitmap rank k_rbm)
     struct RankList { RbmItem *items; unsigned *n; int dir; };
-    const RankList cls[5] = {{list_r3, counts + 13, 1},
+    const RankList cls[6] = {{list_r4, counts + 22, 1}, {list_r3, counts + 13, 1},
         {list_r, counts + 12, 1}, {list_r, counts + 14, -1}, {list_r2, counts + 15, 1}, {list_r2, counts + 16, -1}};
     // Without skewed rows every rank item is a whole row (kPieceMax < U <= maxU):
     // classes above maxU, the multi-round class and the direct-indexed bins are
     // empty and not launched (small levels are bound by launches); DENSE levels
     // have no bins and no whole-row item above kHrMax2 either.
     const bool no_bins = nbig == 0 || dense;
-    const int64_t cls_lo[5] = {kPieceMax, kHrMaxS, kHrMax0, kHrMax1, kHrMax2};
-    for (int c = -1; c < 4; ++c) {
-      if (nbig == 0 && maxU <= cls_lo[c + 1]) continue;
+    const int64_t cls_lo[6] = {kPieceMax, kHrMaxT, kHrMaxS, kHrMax0, kHrMax1, kHrMax2};
+    for (int c = -2; c < 4; ++c) {
+      if (nbig == 0 && maxU <= cls_lo[c + 2]) continue;
       if (c == 3 && no_bins) continue;
-      const RankList &C = cls[c + 1];
+      const RankList &C = cls[c + 2];
       A.ritems = C.items;
       A.nlist = C.n;
       A.rdir = C.dir;

@@ -252,7 +252,7 @@ struct WorkItem {
 
 // Size classes of the rank items (k_tiers): n <= 1024, <= 2048, <= 4096 go to
 // k_hrank<128/256/512> (construct_hrank.cu), larger ones to k_rbm.
-constexpr int kHrMaxS = 512, kHrMax0 = 1024, kHrMax1 = 2048, kHrMax2 = 4096;
+constexpr int kHrMaxT = 128, kHrMaxS = 512, kHrMax0 = 1024, kHrMax1 = 2048, kHrMax2 = 4096;
 constexpr int kDirectR = 4096;  // bins with a key range this small: direct-indexed counters (k_drank)
 
 // A bitmap-rank item (construct_rbm.cu), self-contained so a CTA prefetches it:
@@ -350,7 +350,7 @@ int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide);
 int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket);  // construct_pieces.cu
 int launch_place(hec_ctx *ctx, const RowsArgs &A);
 int launch_rbm(hec_ctx *ctx, const RowsArgs &A);  // construct_rbm.cu
-int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls);  // construct_hrank.cu (cls -1..2: n <= 512/1024/2048/4096)
+int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls);  // construct_hrank.cu (cls -2..2: n <= 128/512/1024/2048/4096)
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo);  // n > 4096
 
 // bins with hi - lo <= kDirectR; bins above kDrSplit entries are cut into chunks

@@ -87,7 +87,7 @@ __device__ __forceinline__ int hr_scan(int32_t *c, uint16_t *o, int nb, int32_t 
 }
 
 template <int NT, int PER = 8>
-__global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : 4) k_hrank(RowsArgs A) {
+__global__ void __launch_bounds__(NT, PER == 8 ? (NT == 128 ? 9 : 1024 / NT) : (NT == 32 ? 32 : 4)) k_hrank(RowsArgs A) {
   constexpr int kCapE = HrSmem<NT, PER>::kCapE;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   HrSmem<NT, PER> &S = *reinterpret_cast<HrSmem<NT, PER> *>(smem_raw);
@@ -587,12 +587,13 @@ static int launch_hrank_t(hec_ctx *ctx, const RowsArgs &A) {
   return HEC_OK;
 }
 
-// One size class of items (the list in A.ritems / A.nlist): cls -1, 0, 1, 2 =
-// n <= 512, 1024, 2048, 4096 on 64-, 128-, 256-, 512-thread CTAs.
+// One size class of items (the list in A.ritems / A.nlist): cls -2, -1, 0, 1, 2 =
+// n <= 128, 512, 1024, 2048, 4096 on 32-, 64-, 128-, 256-, 512-thread CTAs.
 int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls) {
-  static_assert(HrSmem<64>::kCapE == kHrMaxS && HrSmem<128>::kCapE == kHrMax0 && HrSmem<256>::kCapE == kHrMax1 &&
+  static_assert(HrSmem<32, 4>::kCapE == kHrMaxT && HrSmem<64>::kCapE == kHrMaxS && HrSmem<128>::kCapE == kHrMax0 && HrSmem<256>::kCapE == kHrMax1 &&
                     HrSmem<512>::kCapE == kHrMax2,
                 "size classes");
+  if (cls < -1) return launch_hrank_t<32, 4>(ctx, A);  // one warp per item (rows of <= 128 entries)
   if (cls < 0) return launch_hrank_t<64>(ctx, A);  // two warps per item: barriers among 64 threads
   if (cls == 0) return launch_hrank_t<128>(ctx, A);
   if (cls == 1) return launch_hrank_t<256>(ctx, A);  // (<128, 16>: 1.6x slower, measured)
