@@ -211,6 +211,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--prof-steps", type=int, default=-1,
+                    help="steps of the instrumented per-level pass (default min(steps, 5); 0: none, e.g. under ncu)")
     ap.add_argument("--method", default="hec", choices=["hec", "hec3", "hem"],
                     help="mapping method of every level (SURVEY 8(f) f2/f4 ablation; default HEC, the north star)")
     ap.add_argument("--build", default="hash", choices=["hash", "sort", "one_end", "auto"],
@@ -301,7 +303,7 @@ def main():
     launches = ctx.launches()
     # ---- instrumented pass (same step, per-phase / per-level CUDA events): the
     # per-level breakdown and the roofline come from here
-    prof_steps = max(1, min(args.steps, 5))
+    prof_steps = max(1, min(args.steps, 5)) if args.prof_steps < 0 else args.prof_steps
     ctx.set_profiling(True)
     ctx.profile_reset()
     torch.cuda.synchronize()
@@ -311,7 +313,8 @@ def main():
         step()
     ep1.record(stream)
     torch.cuda.synchronize()
-    ms_prof = ep0.elapsed_time(ep1) / prof_steps
+    ms_prof = ep0.elapsed_time(ep1) / prof_steps if prof_steps else 0.0
+    prof_steps = max(prof_steps, 1)  # (divisor of the empty profile below)
     prof = ctx.profile()
     prof_lv = ctx.profile(by_level=True)
     ctx.set_profiling(False)
@@ -349,7 +352,7 @@ def main():
     achieved = b_dom / (t_dom / 1e3) / 1e9 if t_dom > 0 else 0.0
     traffic, stamp = traffic_from_profiles(args.config, l_dom, part_dom)
     phases = {k: {"ms_per_step": v["ms"] / prof_steps, "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] else 0,
-                  "share": v["ms"] / (ms_prof * prof_steps)}
+                  "share": v["ms"] / (ms_prof * prof_steps) if ms_prof else 0.0}
               for k, v in sorted(prof.items(), key=lambda kv: -kv[1]["ms"]) if k != "level"}
 
     # ---- e2e through host buffers

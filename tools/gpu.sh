@@ -14,7 +14,7 @@ TAG=$1; shift
 mkdir -p gpurun_out
 O=gpurun_out/$TAG
 M=gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum
-one_step() { echo "--steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline --config $1"; }
+one_step() { echo "--steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline --prof-steps 0 --config $1"; }
 for step in "$@"; do
   name=${step%%=*}; arg=""; [[ "$step" == *=* ]] && arg=${step#*=}
   echo "== $step"
