@@ -78,8 +78,10 @@ class Comm:
         self.rank, self.world = dist.get_rank(group), dist.get_world_size(group)
         self.device = device or torch.device("cuda", torch.cuda.current_device())
         self.error = None
+        self.calls = 0  # collective calls made by libhec through this communicator
 
         def _cb(send, recv, nbytes, stream, user):
+            self.calls += 1
             try:
                 allgather_bytes(send, recv, int(nbytes), self.group, self.device)
                 return 0

@@ -103,3 +103,60 @@ def test_dist_matches_single_gpu(which, tmp_path):
         assert np.array_equal(d["svw"][:a1 - a0], vw1[a0:a1])
         covered += a1 - a0
     assert covered == nc0
+
+
+def _nccl_worker(port, which, outdir, q):
+    import torch.distributed as dist
+    import paper_conf_ipps_gilbertabmr21_b200 as P
+    from paper_conf_ipps_gilbertabmr21_b200 import dist as D
+    try:
+        torch.cuda.set_device(0)
+        init(0, 1, port, "nccl")
+        g, _ = _graph(which)
+        ctx = P.Context()
+        comm = D.Comm(None, torch.device("cuda", 0))
+        dg = P.DeviceGraph.from_host(g)
+        # level 0 through the partitioned calls (coarsen_hierarchy_dist runs
+        # unpartitioned at world 1; these always exchange through the callback)
+        M, nc = D.hec_find_mapping_dist(ctx, dg, SEED, 0, comm)
+        G1 = D.build_coarse_graph_dist(ctx, dg, M, nc, comm, gather_full=True)
+        rp, col, wgt, vw = G1.graph.to_host()
+        assert comm.error is None, comm.error
+        np.savez(os.path.join(outdir, f"nccl_{which}.npz"), M=M.cpu().numpy(), nc=np.array([nc]), rp=rp, col=col,
+                 wgt=wgt, vw=vw, calls=np.array([comm.calls]))
+        G1.free()
+        ctx.close()
+        q.put("ok")
+    except Exception:  # noqa: BLE001
+        import traceback
+        q.put(traceback.format_exc())
+    finally:
+        if torch.distributed.is_initialized():
+            dist.destroy_process_group()
+
+
+def test_dist_nccl_collective_path(tmp_path):
+    """The all-gather callback over NCCL (all_gather_into_tensor on device
+    buffers; the gloo tests take the host path): one rank on the box's one GPU,
+    level 0 through hec_find_mapping_dist / build_coarse_graph_dist, bit-exact
+    vs the single-GPU calls."""
+    import paper_conf_ipps_gilbertabmr21_b200 as P
+    which = "rmat14"
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_nccl_worker, args=(free_port(), which, str(tmp_path), q))
+    p.start()
+    res = q.get(timeout=600)
+    p.join(timeout=60)
+    assert res == "ok", res
+    g, _ = _graph(which)
+    c = P.Context()
+    dg = P.DeviceGraph.from_host(g)
+    M0, nc0 = P.hec_find_mapping(c, dg, SEED, 0)
+    G1 = P.build_coarse_graph(c, dg, M0, nc0)
+    rp, col, wgt, vw = G1.graph.to_host()
+    d = np.load(tmp_path / f"nccl_{which}.npz")
+    assert int(d["calls"][0]) > 0 and int(d["nc"][0]) == nc0
+    assert np.array_equal(d["M"], M0.cpu().numpy())
+    assert np.array_equal(d["rp"], rp) and np.array_equal(d["col"], col)
+    assert np.array_equal(d["wgt"], wgt) and np.array_equal(d["vw"], vw)
