@@ -1292,7 +1292,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   HEC_TRY(launch_pieces(ctx, A, counts + 5));
   A.list = list_c;
   A.nlist = counts + 11;
-  HEC_TRY(launch_rows(ctx, A, false));
+  // (rank-item levels without skewed rows have only PIECE / RBM blocks: no CTA list)
+  if (!(rbm && nbig == 0)) HEC_TRY(launch_rows(ctx, A, false));
   if (rbm) {
     A.ticket = counts + 30;  // (unused by the rank kernels)
     A.rcap = nblocks + 1;

@@ -467,6 +467,32 @@ static size_t heavy_ws(int64_t n, int64_t nnz) {
 
 // Heavy neighbours of rows [u0, u1): ebase = row_ptr[u0] and nnz of the range are
 // read from the device when the range is partial (one small synchronous read).
+// Small graphs (nnz <= kHeavyRowsMax): one warp per row, lanes stride the row's
+// entries, warp max of the packed key -- one launch instead of the span
+// coordinates + segmented pass + fixup (small levels are launch-bound).
+constexpr int64_t kHeavyRowsMax = 1 << 18;
+__global__ void k_heavy_rows(int64_t n, const int64_t *__restrict__ rp, int64_t vbase,
+                             const int32_t *__restrict__ col, const int32_t *__restrict__ wgt,
+                             int32_t *__restrict__ H) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {
+    const int64_t s = rp[r], e = rp[r + 1];
+    uint64_t best = 0;
+    for (int64_t i = s + lane; i < e; i += 32) {
+      const int32_t w = __ldg(wgt + i);
+      const uint64_t k = w ? pack_key(w, __ldg(col + i)) : 0ull;  // weight 0 never wins (strict >, L116)
+      best = k > best ? k : best;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const uint64_t y = __shfl_xor_sync(0xffffffffu, best, o);
+      best = y > best ? y : best;
+    }
+    if (lane == 0) H[vbase + r] = best ? key_vertex(best) : (int32_t)(vbase + r);  // isolated -> itself
+  }
+}
+
 static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 0, int64_t u1 = -1) {
   if (u1 < 0) u1 = g->n;
   const int64_t n = u1 - u0;
@@ -484,6 +510,14 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
   const int64_t *rp = g->row_ptr + u0;
   if (nnz == 0) {
     k_fill_identity<<<nblk(n, 256), 256, 0, ctx->stream>>>(n, u0, H);
+    HEC_LAUNCH_CHECK();
+    return HEC_OK;
+  }
+  // (HEC_HEAVY_SEG / HEC_HEAVY_TILES: test hooks that keep small graphs on the span / tile kernels)
+  if (nnz <= kHeavyRowsMax && getenv("HEC_HEAVY_SEG") == nullptr && getenv("HEC_HEAVY_TILES") == nullptr) {
+    const int64_t want = (n + 7) / 8;  // 8 warps per CTA, a row per warp
+    const int64_t grid = want < (int64_t)ctx->num_sms * 8 ? want : (int64_t)ctx->num_sms * 8;
+    k_heavy_rows<<<(unsigned)grid, 256, 0, ctx->stream>>>(n, rp, u0, g->col, g->wgt, H);
     HEC_LAUNCH_CHECK();
     return HEC_OK;
   }

@@ -67,8 +67,13 @@ def prio_tensor(pr):
 
 
 # ------------------------------------------------------------------ a1
+@pytest.mark.parametrize("path", ["default", "spans"])
 @pytest.mark.parametrize("which", ["grid", "mesh27_small", "rmat12", "rmat16", "random"])
-def test_heavy_parity(P, ctx, which):
+def test_heavy_parity(P, ctx, which, path, monkeypatch):
+    """default: graphs of <= 2^18 entries take the warp-per-row kernel, larger
+    ones the segmented span kernel; spans: the span kernel for all (test hook)."""
+    if path == "spans":
+        monkeypatch.setenv("HEC_HEAVY_SEG", "1")
     rng = np.random.default_rng(11)
     if which == "grid":
         gs = [gg.grid2d(64, 64), gg.grid2d(1, 7), gg.grid2d(3, 1000)]
@@ -115,14 +120,17 @@ def scattered_isolated_graph(n, rng, deg=6, iso_frac=0.1):
     return gg.from_edges(n, [(u, v, w) for (u, v), w in edges.items()])
 
 
-@pytest.mark.parametrize("path", ["spans", "tiles"])
+@pytest.mark.parametrize("path", ["default", "spans", "tiles"])
 @pytest.mark.parametrize("phase", [0, 1, 2, 3, "mixed"])
 def test_heavy_isolated_and_unaligned(P, ctx, path, phase, monkeypatch):
     """a1 with empty rows anywhere and col/wgt views that start 0-3 int32 past a
-    16-byte boundary (same phase: segmented span kernel; different phases: the
-    tile kernel).  path=tiles forces the merge-path tile kernel (test hook)."""
+    16-byte boundary (default: warp-per-row kernel for the small graphs; spans:
+    the segmented span kernel, scalar loads when the phases differ; tiles: the
+    merge-path tile kernel; test hooks)."""
     if path == "tiles":
         monkeypatch.setenv("HEC_HEAVY_TILES", "1")
+    if path == "spans":
+        monkeypatch.setenv("HEC_HEAVY_SEG", "1")
     rng = np.random.default_rng(31 if phase == "mixed" else 31 + phase)
     for n in (6, 700, 20000):
         g = scattered_isolated_graph(n, rng)
