@@ -548,6 +548,7 @@ HEC_API int coarsen_hierarchy_dist(hec_ctx *ctx, const hec_graph *g0, int64_t cu
                         HEC_BUILD_HASH, out);
 }
 
+constexpr int64_t kFuseHeavyAvgU = 256;
 static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uint64_t seed, int64_t discard_below,
                           int max_levels, const hec_comm *comm, int64_t min_nnz, int method, int build,
                           hec_hierarchy **out) {
@@ -592,6 +593,11 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
     if (rc == HEC_OK)
       rc = part ? find_mapping_dist_impl(ctx, &cur, prio, comm, M, &r)
                 : find_mapping_method_impl(ctx, &cur, method, prio, M, &r);
+    if (ctx->hk_map) {  // this level's heavy keys (fused into the previous placement) are used
+      dev_free(ctx, ctx->hk_map);
+      ctx->hk_map = nullptr;
+      ctx->hk_map_col = nullptr;
+    }
     if (rc != HEC_OK) { out_free(ctx, M); break; }
     ctx->stats.rounds = r.rounds;
     ctx->stats.n_c = r.n_c;
@@ -618,7 +624,28 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
         DistSlice sl;
         rc = build_coarse_dist_impl(ctx, &cur, M, r.n_c, comm, 1, &L.g, &sl);
       } else {
+        // G_{l+1}'s heavy-neighbour keys computed by its placement (k_place),
+        // so the next level's mapping skips its a1 pass over G_{l+1}
+        unsigned long long *hk = nullptr;
+        // (only when rows average >= kFuseHeavyAvgU entries: otherwise most entries sit in
+        // multi-row piece blocks, whose per-entry row search costs more than the a1 pass)
+        // (HEC_FUSE_HEAVY_ALL: test hook, every level regardless of the row volume)
+        const bool fuse = method == HEC_MAP_HEC && build == HEC_BUILD_HASH &&
+                          (cur.nnz >= kFuseHeavyAvgU * r.n_c || getenv("HEC_FUSE_HEAVY_ALL") != nullptr);
+        if (fuse &&
+            dev_alloc(ctx, (void **)&hk, sizeof(unsigned long long) * (r.n_c > 0 ? r.n_c : 1)) != HEC_OK)
+          hk = nullptr;  // (optional: the mapping then runs its own a1 pass)
+        ctx->hk_build = hk;
+        ctx->hk_built = false;
         rc = build_coarse_method_impl(ctx, &cur, M, r.n_c, build, &L.g);
+        ctx->hk_build = nullptr;
+        if (hk && rc == HEC_OK && ctx->hk_built) {
+          ctx->hk_map = hk;
+          ctx->hk_map_col = L.g.col;
+          ctx->hk_map_n = L.g.n_c;
+        } else if (hk) {
+          dev_free(ctx, hk);
+        }
       }
     }
     if (rc != HEC_OK) {
@@ -640,6 +667,11 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
   }
   ctx->prof_level = -1;
   ctx->slab = prev_slab;
+  if (ctx->hk_map) {  // keys of a level the loop did not map (cutoff / cap)
+    dev_free(ctx, ctx->hk_map);
+    ctx->hk_map = nullptr;
+    ctx->hk_map_col = nullptr;
+  }
   if (rc != HEC_OK) {
     hec_hierarchy_free(h);
     return rc;

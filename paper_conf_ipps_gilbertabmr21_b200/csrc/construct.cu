@@ -1364,7 +1364,15 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   A.col_c = out->col;
   A.wgt_c = out->wgt;
   const int ph_place = phase_begin(ctx, "place", 16.0 * (double)nnz_c + 16.0 * dnc);
-  HEC_TRY(launch_place(ctx, A));
+  // heavy keys of G_{l+1} fused into the placement (hierarchy, hash construction
+  // of the whole row range only)
+  bool hk_done = false;
+  if (ctx->hk_build && rbm && !Cp && a_lo == 0 && a_hi == n_c) {
+    HEC_CUDA_TRY(cudaMemsetAsync(ctx->hk_build, 0, sizeof(unsigned long long) * n_c, s));
+    A.hkey = ctx->hk_build;
+  }
+  HEC_TRY(launch_place(ctx, A, &hk_done));
+  ctx->hk_built = hk_done;
   phase_end(ctx, ph_place);
   // rows phase: staged / partitioned entries read (8 B each; DENSE rows were
   // accumulated in rows_skew), distinct entries staged (8 B), row_ptr_c + vwgt_c

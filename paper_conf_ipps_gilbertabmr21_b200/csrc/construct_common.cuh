@@ -342,13 +342,16 @@ struct RowsArgs {
   int32_t rdir;           // +1: items ritems[0 .. n); -1: ritems[rcap - 1], ritems[rcap - 2], ...
   int64_t rcap;
   const unsigned *nlist;  // device count of `list` / `items`
+  // k_place only: max packed key (w << 32 | ~b) per coarse row a at hkey[a - a_lo]
+  // (zeroed; the next level's heavy neighbours, Alg 3 l.6-10), or nullptr
+  unsigned long long *hkey;
 };
 
 // Work-block kernel and placement launchers (construct_rows.cu).
 // Work-block kernels take their blocks from A.list / *A.nlist (device count).
 int launch_rows(hec_ctx *ctx, const RowsArgs &A, bool wide);
 int launch_pieces(hec_ctx *ctx, const RowsArgs &A, unsigned *ticket);  // construct_pieces.cu
-int launch_place(hec_ctx *ctx, const RowsArgs &A);
+int launch_place(hec_ctx *ctx, const RowsArgs &A, bool *hkey_done = nullptr);
 int launch_rbm(hec_ctx *ctx, const RowsArgs &A);  // construct_rbm.cu
 int launch_hrank(hec_ctx *ctx, const RowsArgs &A, int cls);  // construct_hrank.cu (cls -2..2: n <= 128/512/1024/2048/4096)
 int launch_hrank_big(hec_ctx *ctx, const RowsArgs &A, RbmItem *redo, unsigned *nredo);  // n > 4096

@@ -337,6 +337,42 @@ constexpr int kPlaceT = 256;
 enum : int { SRC_SC = 0, SRC_PB = 1, SRC_FB = 2, SRC_DENSE = 3 };
 
 constexpr int kPlaceBig = 96;
+
+// Heavy-neighbour keys of the graph being placed (fused: the next level's a1
+// pass over G_{l+1} is not run).  key = w << 32 | ~b, the row's maximum = its
+// heaviest neighbour, ties to the smallest id (Alg 3 l.6-10, reading Z1).
+__device__ __forceinline__ unsigned long long place_key(int32_t w, int32_t b) {
+  return ((unsigned long long)(uint32_t)w << 32) | (unsigned long long)(~(uint32_t)b);
+}
+// Row of block-relative entry r: the block's row unless it is a rows block
+// holding several rows (row_ptr_c still block-relative: k_place fixes it after
+// its copies, in the same warp).
+__device__ __forceinline__ int32_t place_row(const RowsArgs &A, int kind, int32_t row0, int32_t row1, int64_t r) {
+  if (!rows_kind(kind) || row1 - row0 <= 1) return row0;
+  int32_t lo = row0, hi = row1 - 1;  // last row starting at or before r
+  while (lo < hi) {
+    const int32_t mid = (lo + hi + 1) >> 1;
+    if (A.row_ptr_c[mid - A.L.a_lo] <= r) lo = mid;
+    else hi = mid - 1;
+  }
+  return lo;
+}
+// The warp's 32 entries at consecutive output positions (rows non-decreasing
+// over the valid lanes): segmented max per row, one atomicMax per row segment.
+__device__ __forceinline__ void place_key_flush(const RowsArgs &A, bool valid, int32_t row, unsigned long long key) {
+  const int lane = threadIdx.x & 31;
+  unsigned long long v = valid ? key : 0ull;
+  int32_t rw = valid ? row : -1;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(0xffffffffu, v, o);
+    const int32_t ry = __shfl_up_sync(0xffffffffu, rw, o);
+    if (lane >= o && ry == rw && y > v) v = y;
+  }
+  const int32_t rn = __shfl_down_sync(0xffffffffu, rw, 1);
+  if (valid && (lane == 31 || rn != rw) && v) atomicMax(A.hkey + (rw - A.L.a_lo), v);
+}
+
 __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   const int lane = threadIdx.x & 31;
   const int64_t b0 = ((int64_t)blockIdx.x * (kPlaceT / 32) + (threadIdx.x >> 5)) * 32;
@@ -385,6 +421,7 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
     int32_t c[4], w[4];
     int64_t dst[4];
 #pragma unroll
+    int32_t prow[4];
     for (int t = 0; t < 4; ++t) {
       const int64_t j = j0 + lane + 32 * t;
       int k = 0;  // last lane whose packed range starts at or before j
@@ -397,11 +434,23 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
       const int64_t sb = __shfl_sync(0xffffffffu, soff, k);
       const int64_t r = j - __shfl_sync(0xffffffffu, pex, k);  // index inside the block
       dst[t] = __shfl_sync(0xffffffffu, Om, k) + r;
+      if (A.hkey) {
+        const int kk = __shfl_sync(0xffffffffu, dm.kind, k);
+        const int32_t r0 = __shfl_sync(0xffffffffu, dm.row0, k), r1 = __shfl_sync(0xffffffffu, dm.row1, k);
+        prow[t] = j < ptot ? place_row(A, kk, r0, r1, r) : -1;
+      }
       if (j < ptot) {
         if (sk == SRC_SC) { c[t] = __ldcs(A.sc_col + sb + r); w[t] = __ldcs(A.sc_wgt + sb + r); }
         else if (sk == SRC_PB) { c[t] = __ldcs(A.pb_g + sb + r); w[t] = __ldcs(A.pw_g + sb + r); }
         else if (sk == SRC_FB) { c[t] = __ldcs(A.fb_b + sb + r); w[t] = __ldcs(A.fb_w + sb + r); }
         else { c[t] = dn[sb + 2 * r]; w[t] = dn[sb + 2 * r + 1]; }  // interleaved (b, w) pairs
+      }
+    }
+    if (A.hkey) {
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const bool ok = j0 + lane + 32 * t < ptot;
+        place_key_flush(A, ok, prow[t], ok ? place_key(w[t], c[t]) : 0ull);
       }
     }
 #pragma unroll
@@ -427,6 +476,9 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
     else if (sk == SRC_PB) { sc = A.pb_g + sb; sw = A.pw_g + sb; }
     else if (sk == SRC_FB) { sc = A.fb_b + sb; sw = A.fb_w + sb; }
     else { sc = dn + sb; sw = dn + sb + 1; stride = 2; }
+    const int bkind = __shfl_sync(0xffffffffu, dm.kind, jl);
+    const int32_t brow0 = __shfl_sync(0xffffffffu, dm.row0, jl), brow1 = __shfl_sync(0xffffffffu, dm.row1, jl);
+    const bool one_row = !rows_kind(bkind) || brow1 - brow0 <= 1;
     for (int r0 = sl * 256; r0 < T; r0 += S * 256) {
       int32_t c[8], w[8];
 #pragma unroll
@@ -438,6 +490,31 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
       for (int t = 0; t < 8; ++t) {
         const int r = r0 + lane + 32 * t;
         if (r < T) { __stcs(A.col_c + O + r, c[t]); __stcs(A.wgt_c + O + r, w[t]); }
+      }
+      if (A.hkey) {
+        if (one_row) {  // one row: lane maxima, warp maximum, one atomic per 256 entries
+          unsigned long long m = 0ull;
+#pragma unroll
+          for (int t = 0; t < 8; ++t)
+            if (r0 + lane + 32 * t < T) {
+              const unsigned long long key = place_key(w[t], c[t]);
+              m = key > m ? key : m;
+            }
+#pragma unroll
+          for (int o = 16; o > 0; o >>= 1) {
+            const unsigned long long y = __shfl_xor_sync(0xffffffffu, m, o);
+            m = y > m ? y : m;
+          }
+          if (lane == 0 && m) atomicMax(A.hkey + (brow0 - L.a_lo), m);
+        } else {
+#pragma unroll
+          for (int t = 0; t < 8; ++t) {
+            const int r = r0 + lane + 32 * t;
+            const bool ok = r < T;
+            place_key_flush(A, ok, ok ? place_row(A, bkind, brow0, brow1, r) : -1,
+                            ok ? place_key(w[t], c[t]) : 0ull);
+          }
+        }
       }
     }
   }
@@ -460,13 +537,19 @@ __global__ void __launch_bounds__(kPlaceT) k_place(RowsArgs A) {
   }
 }
 
-int launch_place(hec_ctx *ctx, const RowsArgs &A) {
+int launch_place(hec_ctx *ctx, const RowsArgs &A, bool *hkey_done) {
+  if (hkey_done) *hkey_done = false;
   if (A.nblocks <= 0) return HEC_OK;
   // slices per 32-block group: enough warps for ~16 per SM on small levels
   const int64_t groups = (A.nblocks + 31) / 32;
   int64_t S = (int64_t)ctx->num_sms * 16 / groups;
   S = S < 1 ? 1 : S > 32 ? 32 : S;
-  k_place<<<dim3((unsigned)nblk(groups, kPlaceT / 32), (unsigned)S), kPlaceT, 0, ctx->stream>>>(A);
+  // heavy keys only with one slice per group: a rows block's offsets are then
+  // read (row search) and fixed up by the same warp
+  RowsArgs B = A;
+  if (S != 1) B.hkey = nullptr;
+  if (hkey_done) *hkey_done = B.hkey != nullptr;
+  k_place<<<dim3((unsigned)nblk(groups, kPlaceT / 32), (unsigned)S), kPlaceT, 0, ctx->stream>>>(B);
   HEC_LAUNCH_CHECK();
   return HEC_OK;
 }

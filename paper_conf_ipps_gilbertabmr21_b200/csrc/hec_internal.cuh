@@ -113,6 +113,15 @@ struct hec_ctx {
   hec_stats stats{};
   // state carried between hec_build_rows_count and hec_build_rows_write
   struct DistState *dist = nullptr;
+  // heavy-neighbour keys fused into the placement of G_{l+1} (hierarchy only):
+  // hk_build: target of the build in progress (k_place), hk_built: it was filled;
+  // hk_map / hk_map_col / hk_map_n: keys of the graph whose col array is hk_map_col,
+  // used by the next mapping instead of its a1 pass
+  unsigned long long *hk_build = nullptr;
+  bool hk_built = false;
+  unsigned long long *hk_map = nullptr;
+  const int32_t *hk_map_col = nullptr;
+  int64_t hk_map_n = 0;
   // profiling (hec_ctx_set_profiling)
   int64_t launches = 0;
   int prof_on = 0;

@@ -1003,6 +1003,15 @@ static int resolve_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *H, Prio
   return HEC_OK;
 }
 
+// H from the heavy keys the previous level's placement left (k_place): the
+// row maximum of w << 32 | ~v, 0 for an empty row (-> itself)
+__global__ void k_hkey_to_H(int64_t n, const unsigned long long *__restrict__ hk, int32_t *__restrict__ H) {
+  const int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (u >= n) return;
+  const unsigned long long k = hk[u];
+  H[u] = k ? key_vertex(k) : (int32_t)u;
+}
+
 int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, uint8_t *root_out,
                       int32_t *H_out, MapResult *res) {
   const int64_t n = g->n;
@@ -1012,9 +1021,16 @@ int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, u
   int32_t *H = H_out ? H_out : ws_take<int32_t>(ctx, n);
   if (!H) { set_error("workspace under-reserved (mapping)"); return HEC_EINVAL; }
   const double dn = (double)n, dnnz = (double)g->nnz;
-  int ph = phase_begin(ctx, "heavy", 8.0 * dnnz + 8.0 * (dn + 1) + 4.0 * dn);
-  HEC_TRY(run_heavy(ctx, g, H));
-  phase_end(ctx, ph);
+  if (ctx->hk_map && ctx->hk_map_col == g->col && ctx->hk_map_n == n) {
+    int ph = phase_begin(ctx, "heavy", 12.0 * dn);  // keys computed with the placement of g
+    k_hkey_to_H<<<nblk(n, 256), 256, 0, ctx->stream>>>(n, ctx->hk_map, H);
+    HEC_LAUNCH_CHECK();
+    phase_end(ctx, ph);
+  } else {
+    int ph = phase_begin(ctx, "heavy", 8.0 * dnnz + 8.0 * (dn + 1) + 4.0 * dn);
+    HEC_TRY(run_heavy(ctx, g, H));
+    phase_end(ctx, ph);
+  }
   return resolve_impl(ctx, g, H, prio, 0, n, M, root_out, res);
 }
 

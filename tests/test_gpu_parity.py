@@ -572,6 +572,15 @@ def test_hierarchy_c2(P, ctx):
     check_hierarchy(P, ctx, gg.config(2), 1000)
 
 
+def test_hierarchy_c2_fused_heavy_everywhere(P, ctx, monkeypatch):
+    """The next level's heavy neighbours computed by the placement (k_place) on
+    every large-enough level, also where most entries sit in multi-row piece
+    blocks (per-entry row search; HEC_FUSE_HEAVY_ALL test hook; by default only
+    levels averaging >= 256 entries per coarse row fuse)."""
+    monkeypatch.setenv("HEC_FUSE_HEAVY_ALL", "1")
+    check_hierarchy(P, ctx, gg.config(2), 1000)
+
+
 @pytest.mark.parametrize("scale", [10, 12, 16, 18])
 def test_hierarchy_rmat(P, ctx, scale):
     check_hierarchy(P, ctx, gg.rmat(scale, 16), 50)
