@@ -24,8 +24,10 @@ PROF = os.path.join(ROOT, "profiles")
 
 # kernels of the mapping (a1-a5); every other libhec kernel belongs to the construction
 MAPPING = ("k_span_coords", "k_heavy", "k_fill_identity", "k_tile_coords", "k_round_init", "k_rounds",
-           "RootFlagIn", "k_assign", "k_jump")
-LEVEL_START = ("k_span_coords", "k_tile_coords", "k_fill_identity")  # first launch of each level's mapping
+           "RootFlagIn", "k_assign", "k_jump", "k_hkey_to_H")
+# first launch of each level's mapping (k_hkey_to_H: keys fused into the previous placement;
+# k_heavy_rows: small graphs)
+LEVEL_START = ("k_span_coords", "k_tile_coords", "k_fill_identity", "k_hkey_to_H", "k_heavy_rows")
 
 
 def part_of(name):
