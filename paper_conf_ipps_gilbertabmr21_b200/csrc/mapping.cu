@@ -1022,7 +1022,7 @@ int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, u
   if (!H) { set_error("workspace under-reserved (mapping)"); return HEC_EINVAL; }
   const double dn = (double)n, dnnz = (double)g->nnz;
   if (ctx->hk_map && ctx->hk_map_col == g->col && ctx->hk_map_n == n) {
-    int ph = phase_begin(ctx, "heavy", 12.0 * dn);  // keys computed with the placement of g
+    int ph = phase_begin(ctx, "heavy", 20.0 * dn);  // keys (8 B) in, H out; computed with the placement of g
     k_hkey_to_H<<<nblk(n, 256), 256, 0, ctx->stream>>>(n, ctx->hk_map, H);
     HEC_LAUNCH_CHECK();
     phase_end(ctx, ph);
