@@ -18,6 +18,8 @@
 // flagged blocks with the 64-bit (WIDE) instantiation.
 #include <type_traits>
 
+#include <stdlib.h>
+
 #include "construct_common.cuh"
 
 namespace hec {
@@ -544,6 +546,7 @@ int launch_place(hec_ctx *ctx, const RowsArgs &A, bool *hkey_done) {
   const int64_t groups = (A.nblocks + 31) / 32;
   int64_t S = (int64_t)ctx->num_sms * 16 / groups;
   S = S < 1 ? 1 : S > 32 ? 32 : S;
+  if (getenv("HEC_PLACE_ONE_SLICE") != nullptr) S = 1;  // test hook: fused heavy keys on small levels
   // heavy keys only with one slice per group: a rows block's offsets are then
   // read (row search) and fixed up by the same warp
   RowsArgs B = A;

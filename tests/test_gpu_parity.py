@@ -572,6 +572,17 @@ def test_hierarchy_c2(P, ctx):
     check_hierarchy(P, ctx, gg.config(2), 1000)
 
 
+@pytest.mark.parametrize("which", ["c1", "rmat12", "mesh27_16"])
+def test_hierarchy_fused_heavy_small(P, ctx, which, monkeypatch):
+    """The fused heavy keys on small graphs: every placement in one slice per
+    32-block group and every level fused (HEC_PLACE_ONE_SLICE, HEC_FUSE_HEAVY_ALL
+    test hooks), bit-exact vs the oracle."""
+    monkeypatch.setenv("HEC_FUSE_HEAVY_ALL", "1")
+    monkeypatch.setenv("HEC_PLACE_ONE_SLICE", "1")
+    g = {"c1": lambda: gg.config(1), "rmat12": lambda: gg.rmat(12, 16), "mesh27_16": lambda: gg.mesh27(16, 16, 16)}[which]()
+    check_hierarchy(P, ctx, g, 50)
+
+
 def test_hierarchy_c2_fused_heavy_everywhere(P, ctx, monkeypatch):
     """The next level's heavy neighbours computed by the placement (k_place) on
     every large-enough level, also where most entries sit in multi-row piece

@@ -18,18 +18,23 @@ def main():
     import torch
     torch.cuda.set_device(0)
     ctx = P.Context(torch_alloc=False)
-    for name, g, cut in (("c1", gg.config(1), 50), ("rmat12", gg.rmat(12, 16), 50),
-                         ("mesh27_16", gg.mesh27(16, 16, 16), 50)):
-        h = P.coarsen_hierarchy(ctx, P.DeviceGraph.from_host(g), cut, gg.COARSEN_SEED)
-        ref = o.hierarchy(g, cut, gg.COARSEN_SEED)
-        assert len(h.levels) == len(ref.levels), name
-        for lv, lo in zip(h.levels, ref.levels):
-            rp, col, wgt, vw = lv.graph.to_host()
-            assert np.array_equal(lv.M.cpu().numpy(), lo.M), name
-            assert np.array_equal(rp, lo.graph.row_ptr) and np.array_equal(col, lo.graph.col), name
-            assert np.array_equal(wgt, lo.graph.wgt) and np.array_equal(vw, lo.graph.vwgt), name
-        print(name, "levels", len(h.levels), "bit-exact", flush=True)
-        h.free()
+    cases = [("c1", gg.config(1), 50), ("rmat12", gg.rmat(12, 16), 50), ("mesh27_16", gg.mesh27(16, 16, 16), 50)]
+    # second pass: the next level's heavy keys fused into every placement (test hooks)
+    for fused in (False, True):
+        if fused:
+            os.environ["HEC_FUSE_HEAVY_ALL"] = "1"
+            os.environ["HEC_PLACE_ONE_SLICE"] = "1"
+        for name, g, cut in cases:
+            h = P.coarsen_hierarchy(ctx, P.DeviceGraph.from_host(g), cut, gg.COARSEN_SEED)
+            ref = o.hierarchy(g, cut, gg.COARSEN_SEED)
+            assert len(h.levels) == len(ref.levels), name
+            for lv, lo in zip(h.levels, ref.levels):
+                rp, col, wgt, vw = lv.graph.to_host()
+                assert np.array_equal(lv.M.cpu().numpy(), lo.M), name
+                assert np.array_equal(rp, lo.graph.row_ptr) and np.array_equal(col, lo.graph.col), name
+                assert np.array_equal(wgt, lo.graph.wgt) and np.array_equal(vw, lo.graph.vwgt), name
+            print(name, "fused" if fused else "", "levels", len(h.levels), "bit-exact", flush=True)
+            h.free()
     ctx.close()
     print("sanitize_run ok")
 
