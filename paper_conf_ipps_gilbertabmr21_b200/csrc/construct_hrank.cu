@@ -448,12 +448,18 @@ __global__ void __launch_bounds__(kDrT) k_drank(RowsArgs A) {
     if (it.hi - lo <= kDrRowSweep) {
       D = dr_sweep<true>(val, it.hi - lo, lo, src_b, src_w, wsum, over);
     } else {  // wide bins: thread t owns counters [16 t, 16 t + 16) (fewer instructions)
+      const int R = it.hi - lo;
       uint32_t v[16];
       int c = 0;
+      if (16 * t < R) {  // (counters at or past R are never touched: zero)
 #pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        v[q] = val[16 * t + q];
-        c += v[q] != 0u;
+        for (int q = 0; q < 16; ++q) {
+          v[q] = val[16 * t + q];
+          c += v[q] != 0u;
+        }
+      } else {
+#pragma unroll
+        for (int q = 0; q < 16; ++q) v[q] = 0u;
       }
       int x = c;
 #pragma unroll
