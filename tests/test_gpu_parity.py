@@ -597,7 +597,13 @@ def test_hierarchy_rmat(P, ctx, scale):
     check_hierarchy(P, ctx, gg.rmat(scale, 16), 50)
 
 
-def test_hierarchy_edge_cases(P, ctx):
+@pytest.mark.parametrize("fused", [False, True])
+def test_hierarchy_edge_cases(P, ctx, fused, monkeypatch):
+    """fused: the heavy keys of every level from its placement (test hooks),
+    including rows of G_{l+1} left empty by isolated vertices (key 0 -> itself)."""
+    if fused:
+        monkeypatch.setenv("HEC_FUSE_HEAVY_ALL", "1")
+        monkeypatch.setenv("HEC_PLACE_ONE_SLICE", "1")
     empty = gg.Graph(np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0, np.int32), np.zeros(0, np.int32))
     Hg = P.coarsen_hierarchy(ctx, P.DeviceGraph.from_host(empty), 50, SEED)
     assert Hg.levels == [] and Hg.stop_reason == P.STOP_CUTOFF
