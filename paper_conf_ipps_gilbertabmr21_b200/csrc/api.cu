@@ -637,7 +637,9 @@ static int hierarchy_impl(hec_ctx *ctx, const hec_graph *g0, int64_t cutoff, uin
           hk = nullptr;  // (optional: the mapping then runs its own a1 pass)
         ctx->hk_build = hk;
         ctx->hk_built = false;
+        ctx->build_unit_wgt = r.unit_weights ? cur.wgt : nullptr;  // the expansion need not read them
         rc = build_coarse_method_impl(ctx, &cur, M, r.n_c, build, &L.g);
+        ctx->build_unit_wgt = nullptr;
         ctx->hk_build = nullptr;
         if (hk && rc == HEC_OK && ctx->hk_built) {
           ctx->hk_map = hk;

@@ -309,7 +309,7 @@ struct StageSink {
   __device__ __forceinline__ void load(int32_t (&b)[N], int32_t (&w)[N], const IdxT (&e)[N], unsigned ok) {
 #pragma unroll
     for (int u = 0; u < N; ++u)
-      if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
+      if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = L.unit_w ? 1 : __ldcs(L.wgt + e[u]); }
 #pragma unroll
     for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
@@ -894,7 +894,7 @@ struct AccSink {
     int32_t b[N], w[N];
 #pragma unroll
     for (int u = 0; u < N; ++u)
-      if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = __ldcs(L.wgt + e[u]); }
+      if (ok & (1u << u)) { b[u] = __ldcs(L.col + e[u]); w[u] = L.unit_w ? 1 : __ldcs(L.wgt + e[u]); }
 #pragma unroll
     for (int u = 0; u < N; ++u)
       if (ok & (1u << u)) b[u] = __ldg(L.M + b[u]);
@@ -1042,7 +1042,8 @@ int build_coarse_impl(hec_ctx *ctx, const hec_graph *g, const int32_t *M, int64_
   // 32-bit entry / position indices in the member walks when nnz < 2^32
   // (HEC_FORCE_WIDE_INDEX: test hook for the 64-bit instantiation)
   const bool idx32 = g->nnz < ((int64_t)1 << 32) && getenv("HEC_FORCE_WIDE_INDEX") == nullptr;
-  Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi, kRbmBinAvg};
+  Layout L{n_c, member_ptr, members, mpre, g->row_ptr, g->col, g->wgt, M, a_lo, a_hi, kRbmBinAvg,
+           ctx->build_unit_wgt != nullptr && ctx->build_unit_wgt == g->wgt};
   const bool dense = n_c <= kDenseMax;
   // bitmap-rank items replace the bin pieces when the key range fits the
   // shared-memory bitmap (BuildOpts::sort_dedup, HEC_BUILD_SORT: the bin-piece / bucket-sort path)

@@ -114,6 +114,7 @@ struct Layout {
   const int32_t *M;
   int64_t a_lo, a_hi;  // coarse rows produced by this call (range partition, §8(e))
   int64_t bin_avg;     // target entries per key-range bin of a skewed row (rank items)
+  bool unit_w = false;  // every weight of the fine graph is 1 (a1's flag): weights not read
   __device__ __forceinline__ bool active(int64_t a) const { return a >= a_lo && a < a_hi; }
   __device__ __forceinline__ int64_t upos(int64_t a) const { return mpre[member_ptr[a]]; }
   __device__ __forceinline__ int64_t U(int64_t a) const { return upos(a + 1) - upos(a); }

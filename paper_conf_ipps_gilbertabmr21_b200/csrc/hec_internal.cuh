@@ -117,6 +117,10 @@ struct hec_ctx {
   // hk_build: target of the build in progress (k_place), hk_built: it was filled;
   // hk_map / hk_map_col / hk_map_n: keys of the graph whose col array is hk_map_col,
   // used by the next mapping instead of its a1 pass
+  // weight array of the graph being built whose weights are all 1 (the a1 pass's
+  // flag; hierarchy only; nested builds on other graphs read their weights)
+  const int32_t *build_unit_wgt = nullptr;
+  bool unit_flag_armed = false;  // the a1 span pass of the current mapping sets h_pinned[63]
   unsigned long long *hk_build = nullptr;
   bool hk_built = false;
   unsigned long long *hk_map = nullptr;
@@ -442,6 +446,7 @@ inline size_t scan_ws_bytes(int64_t N) {
 struct MapResult {
   int64_t n_c = 0;
   int rounds = 0;
+  bool unit_weights = false;  // the a1 span pass saw only weights of 1
 };
 int ws_bytes_mapping(int64_t n, int64_t nnz, size_t *bytes);
 // M (device) and optional root (device u8) outputs; uses workspace already reserved.

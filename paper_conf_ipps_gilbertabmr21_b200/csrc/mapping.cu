@@ -297,6 +297,7 @@ struct SegArgs {
   const int32_t *cx;
   int32_t *H;
   uint64_t *head_key, *mid_key;
+  volatile int *nonunit;  // pinned host flag: set when a weight other than 1 is seen (or nullptr)
 };
 
 // lane's 16 consecutive entries of span k (4 x 16 B of col and of wgt, or scalars)
@@ -424,16 +425,20 @@ __global__ void __launch_bounds__(32 * kSegWarps, 2) k_heavy_seg(SegArgs A) {
   if (k >= A.nspans) return;
   int cc[16], ww[16];
   seg_load<kVec>(A, k, cc, ww);
+  bool nu = false;
   while (true) {
     const int64_t kn = k + nw;
     int nc[16], nw_[16];
     if (kn < A.nspans) seg_load<kVec>(A, kn, nc, nw_);
     seg_process(A, k, W, cc, ww);
+#pragma unroll
+    for (int q = 0; q < 16; ++q) nu |= (unsigned)ww[q] > 1u;  // (entries outside the range read 0)
     if (kn >= A.nspans) break;
     k = kn;
 #pragma unroll
     for (int q = 0; q < 16; ++q) { cc[q] = nc[q]; ww[q] = nw_[q]; }
   }
+  if (A.nonunit && __any_sync(0xffffffffu, nu) && (threadIdx.x & 31) == 0) *A.nonunit = 1;
 }
 
 // Rows that end in span k but began in an earlier span s0: max of span k's head
@@ -535,7 +540,12 @@ static int run_heavy(hec_ctx *ctx, const hec_graph *g, int32_t *H, int64_t u0 = 
     if (!cx || !head || !mid) { set_error("workspace under-reserved (heavy)"); return HEC_EINVAL; }
     k_span_coords<<<nblk(nspans + 1, 256), 256, 0, ctx->stream>>>(n, nnz, rp, ebase, x0, off, nspans, cx, head);
     HEC_LAUNCH_CHECK();
-    SegArgs SA{n, nnz, rp, ebase, u0, x0, off, nspans, g->col - off, g->wgt - off, cx, H, head, mid};
+    // unit-weight flag (pinned host word, written by the kernel, read after the
+    // mapping's host read): only for whole graphs
+    volatile int *flag = (u0 == 0 && u1 == g->n) ? reinterpret_cast<volatile int *>(ctx->h_pinned + 63) : nullptr;
+    if (flag) *flag = 0;
+    ctx->unit_flag_armed = flag != nullptr;
+    SegArgs SA{n, nnz, rp, ebase, u0, x0, off, nspans, g->col - off, g->wgt - off, cx, H, head, mid, flag};
     int occ[2] = {1, 1};
     if (vec) HEC_TRY(kernel_occupancy(ctx, k_heavy_seg<true>, 32 * kSegWarps, 0, &occ[1]));
     else HEC_TRY(kernel_occupancy(ctx, k_heavy_seg<false>, 32 * kSegWarps, 0, &occ[0]));
@@ -1028,10 +1038,16 @@ int find_mapping_impl(hec_ctx *ctx, const hec_graph *g, Prio prio, int32_t *M, u
     phase_end(ctx, ph);
   } else {
     int ph = phase_begin(ctx, "heavy", 8.0 * dnnz + 8.0 * (dn + 1) + 4.0 * dn);
+    ctx->unit_flag_armed = false;
     HEC_TRY(run_heavy(ctx, g, H));
     phase_end(ctx, ph);
   }
-  return resolve_impl(ctx, g, H, prio, 0, n, M, root_out, res);
+  const bool armed = ctx->unit_flag_armed;
+  ctx->unit_flag_armed = false;
+  HEC_TRY(resolve_impl(ctx, g, H, prio, 0, n, M, root_out, res));
+  // (resolve_impl's host read synchronised the stream: the span kernel's flag is final)
+  res->unit_weights = armed && *reinterpret_cast<volatile int *>(ctx->h_pinned + 63) == 0;
+  return HEC_OK;
 }
 
 int heavy_range_impl(hec_ctx *ctx, const hec_graph *g, int64_t u0, int64_t u1, int32_t *H) {
